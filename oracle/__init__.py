@@ -1,0 +1,174 @@
+"""CPU oracle for the batched Jacobi-preconditioned BiCGSTAB (ctypes wrapper).
+
+TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+cpu_baseline / ``--impl reference`` legs of bench.py may import this package.
+The product package (paper_conf_ipps_kashinksla22_b200) never imports it and
+shares no code with it (see oracle.c for the algorithm and its citations).
+
+Functions mirror oracle.c:
+  spmv, dense_solve, banded_solve, bandwidth, bicgstab (one system, with
+  optional invariant trace), batch_bicgstab, batch_banded (host threads).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+STOP_REL_B = 0
+STOP_ABS = 1
+CONVERGED, MAXITER, BREAKDOWN = 0, 1, 2
+
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c with gcc (no BLAS, no CUDA, IEEE fp64, no FMA contraction)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        cmd = ["gcc", "-O2", "-std=c11", "-D_GNU_SOURCE", "-ffp-contract=off", "-fno-fast-math",
+               "-fPIC", "-shared", "-o", _LIB + ".tmp", _SRC, "-lpthread", "-lm"]
+        subprocess.check_call(cmd)
+        os.replace(_LIB + ".tmp", _LIB)
+    return _LIB
+
+
+class Result(C.Structure):
+    _fields_ = [("iters", C.c_int32), ("status", C.c_int32), ("restarts", C.c_int32),
+                ("exit_kind", C.c_int32), ("resnorm", C.c_double),
+                ("recursive", C.c_double), ("tau", C.c_double)]
+
+
+_P = C.c_void_p
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            L = C.CDLL(build())
+            L.oracle_spmv_csr.argtypes = [C.c_int, _P, _P, _P, _P, _P]
+            L.oracle_spmv_csr.restype = None
+            L.oracle_dense_solve.argtypes = [C.c_int, _P, _P]
+            L.oracle_dense_solve.restype = C.c_int
+            L.oracle_bandwidth.argtypes = [C.c_int, _P, _P, C.POINTER(C.c_int), C.POINTER(C.c_int)]
+            L.oracle_bandwidth.restype = None
+            L.oracle_banded_solve.argtypes = [C.c_int, _P, _P, _P, _P, _P]
+            L.oracle_banded_solve.restype = C.c_int
+            L.oracle_bicgstab.argtypes = [C.c_int, _P, _P, _P, _P, _P, C.c_double, C.c_int,
+                                          C.c_int, C.c_int, _P, C.POINTER(Result), _P]
+            L.oracle_bicgstab.restype = C.c_int
+            L.oracle_batch_bicgstab.argtypes = [C.c_int, C.c_int, C.c_int, _P, _P, _P, _P, _P,
+                                                C.c_double, C.c_int, C.c_int, C.c_int,
+                                                _P, _P, _P, _P, _P, C.c_int]
+            L.oracle_batch_bicgstab.restype = C.c_int
+            L.oracle_batch_banded.argtypes = [C.c_int, C.c_int, C.c_int, _P, _P, _P, _P, _P,
+                                              _P, C.c_int]
+            L.oracle_batch_banded.restype = C.c_int
+            _lib = L
+    return _lib
+
+
+def _i32(a):
+    return np.ascontiguousarray(a, dtype=np.int32)
+
+
+def _f64(a):
+    return np.ascontiguousarray(a, dtype=np.float64)
+
+
+def _ptr(a):
+    return None if a is None else a.ctypes.data
+
+
+def spmv(row_ptr, col_idx, val, x):
+    rp, ci, v, xx = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(x)
+    n = rp.size - 1
+    y = np.empty(n)
+    lib().oracle_spmv_csr(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(xx), _ptr(y))
+    return y
+
+
+def dense_solve(A, b):
+    A = np.array(A, dtype=np.float64, order="C")
+    x = np.array(b, dtype=np.float64)
+    info = lib().oracle_dense_solve(A.shape[0], _ptr(A), _ptr(x))
+    if info:
+        raise np.linalg.LinAlgError(f"zero pivot at {info - 1}")
+    return x
+
+
+def bandwidth(row_ptr, col_idx):
+    rp, ci = _i32(row_ptr), _i32(col_idx)
+    kl, ku = C.c_int(), C.c_int()
+    lib().oracle_bandwidth(rp.size - 1, _ptr(rp), _ptr(ci), C.byref(kl), C.byref(ku))
+    return kl.value, ku.value
+
+
+def banded_solve(row_ptr, col_idx, val, b):
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(b)
+    x = np.empty(rp.size - 1)
+    info = lib().oracle_banded_solve(rp.size - 1, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x))
+    if info:
+        raise np.linalg.LinAlgError(f"banded LU: zero pivot / error {info}")
+    return x
+
+
+def bicgstab(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, stop=STOP_REL_B,
+             true_res_check=True, trace=False):
+    """One system through Algorithm 1.  Returns (x, Result[, trace])."""
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(b)
+    n = rp.size - 1
+    x0a = None if x0 is None else _f64(x0)
+    x = np.empty(n)
+    R = Result()
+    tr = np.full(max(maxiter, 1), np.nan) if trace else None
+    rc = lib().oracle_bicgstab(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x0a), float(tol),
+                               int(maxiter), int(stop), int(bool(true_res_check)), _ptr(x),
+                               C.byref(R), _ptr(tr))
+    if rc:
+        raise MemoryError("oracle_bicgstab")
+    if trace:
+        return x, R, tr[: R.iters]
+    return x, R
+
+
+def batch_bicgstab(row_ptr, col_idx, values, b, x0=None, tol=1e-10, maxiter=1000,
+                   stop=STOP_REL_B, true_res_check=True, threads=0):
+    """Alg. 1 on every system (values [batch, nnz] CSR order).
+    Returns dict(x, iters, resnorm, status, restarts)."""
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(values), _f64(b)
+    batch, nnz = v.shape
+    n = rp.size - 1
+    x0a = None if x0 is None else _f64(x0)
+    out = dict(x=np.empty((batch, n)), iters=np.empty(batch, np.int32),
+               resnorm=np.empty(batch), status=np.empty(batch, np.int32),
+               restarts=np.empty(batch, np.int32))
+    rc = lib().oracle_batch_bicgstab(n, nnz, batch, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb),
+                                     _ptr(x0a), float(tol), int(maxiter), int(stop),
+                                     int(bool(true_res_check)), _ptr(out["x"]),
+                                     _ptr(out["iters"]), _ptr(out["resnorm"]),
+                                     _ptr(out["status"]), _ptr(out["restarts"]), int(threads))
+    if rc:
+        raise MemoryError("oracle_batch_bicgstab")
+    return out
+
+
+def batch_banded(row_ptr, col_idx, values, b, threads=0):
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(values), _f64(b)
+    batch, nnz = v.shape
+    n = rp.size - 1
+    x = np.empty((batch, n))
+    st = np.empty(batch, np.int32)
+    rc = lib().oracle_batch_banded(n, nnz, batch, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb),
+                                   _ptr(x), _ptr(st), int(threads))
+    if rc or np.any(st != 0):
+        raise np.linalg.LinAlgError("batch banded LU failed")
+    return x
