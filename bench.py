@@ -1,0 +1,475 @@
+#!/usr/bin/env python
+"""Benchmark: systems solved per second for batched Jacobi-BiCGSTAB on B200.
+
+Metric (BASELINE.json): "systems solved/sec (992-row XGC matrices, tol 1e-10)
+at 1/2/4/8 B200; % roofline".  Workload at N = 1: BASELINE.json configs[3]'s
+batch of 10^5 XGC-shaped systems (50/50 ion/electron, 32x31 grid, 9-point
+stencil, fp64, zero initial guess, tol 1e-10 relative to ||b||), which fits
+one GPU; with N GPUs each rank solves its own 10^5-system slice (weak
+scaling, no collective on the solve path).
+
+One "step" = one bsolve_run over the rank's whole batch (one kernel launch).
+Timed region: W untimed warm-up steps, then K steps bracketed by barrier +
+cuda synchronize, CUDA events on the launching stream, max over ranks.
+Inputs (8.7 GB per rank) exceed the 126 MB L2, so no flush is needed.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "systems solved/sec (992-row XGC matrices, tol 1e-10)"
+UNIT = "systems/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--batch", type=int, default=100_000, help="systems per GPU (weak scaling)")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    ap.add_argument("--nx", type=int, default=32)
+    ap.add_argument("--ny", type=int, default=31)
+    ap.add_argument("--format", choices=["ell", "csr"], default="ell")
+    ap.add_argument("--placement", choices=["auto", "smem", "stream"], default="auto")
+    ap.add_argument("--tol", type=float, default=1e-10)
+    ap.add_argument("--maxiter", type=int, default=1000)
+    ap.add_argument("--seed", type=int, default=20220530)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0,
+                    help="target wall seconds of the oracle sample")
+    ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- clocks --
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([c.strip() for c in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"],
+                    "samples": 0}
+        def f(x):
+            try:
+                return float(x)
+            except ValueError:
+                return None
+        sm = [f(r[1]) for r in self.rows if f(r[1])]
+        mx = [f(r[2]) for r in self.rows if f(r[2])]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[5:9]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        pw = [f(r[3]) for r in self.rows if f(r[3])]
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------- inputs --
+def make_inputs(g0, count, args, pinned):
+    """Generate systems g0..g0+count-1 into (pinned) host buffers, ELL/CSR."""
+    import torch
+    import xgcgen as X
+    pat = X.stencil_pattern(args.nx, args.ny)
+    W = pat.max_row_nnz
+    per = W * pat.n if args.format == "ell" else pat.nnz
+    vals = torch.empty((count, per), dtype=torch.float64, pin_memory=pinned)
+    b = torch.empty((count, pat.n), dtype=torch.float64, pin_memory=pinned)
+    vn, bn = vals.numpy(), b.numpy()
+    _, src = X.ell_layout(pat.row_ptr, pat.col_idx)
+    ok = src >= 0
+    CH = 8192
+    for c0 in range(0, count, CH):
+        c1 = min(count, c0 + CH)
+        Bt = X.make_batch(g0 + c0, c1 - c0, pattern=pat, seed=args.seed)
+        if args.format == "ell":
+            blk = vn[c0:c1]
+            blk[:, ~ok] = 0.0
+            blk[:, ok] = Bt.values[:, src[ok]]
+        else:
+            vn[c0:c1] = Bt.values
+        bn[c0:c1] = Bt.b
+    return pat, vals, b
+
+
+def make_csr_sample(g0, count, args):
+    import xgcgen as X
+    pat = X.stencil_pattern(args.nx, args.ny)
+    return pat, X.make_batch(g0, count, pattern=pat, seed=args.seed)
+
+
+# ------------------------------------------------------- cpu baseline --
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_sample_rate(g0, max_count, args, target_s, kind="bicgstab"):
+    """Time the oracle (as it stands) on a bounded sample; returns dict."""
+    import oracle as O
+    cores = host_cores()
+    # calibrate on a small sample, then size the sample to ~target_s of wall time
+    n_cal = min(max_count, max(2 * cores, 64))
+    pat, Bc = make_csr_sample(g0, n_cal, args)
+    t0 = time.perf_counter()
+    if kind == "bicgstab":
+        O.batch_bicgstab(pat.row_ptr, pat.col_idx, Bc.values, Bc.b, tol=args.tol,
+                         maxiter=args.maxiter, threads=cores)
+    else:
+        O.batch_banded(pat.row_ptr, pat.col_idx, Bc.values, Bc.b, threads=cores)
+    dt = time.perf_counter() - t0
+    rate = n_cal / max(dt, 1e-9)
+    count = int(min(max_count, max(n_cal, rate * target_s)))
+    count -= count % 2  # keep the ion/electron mix 50/50
+    count = max(count, 2)
+    pat, Bs = make_csr_sample(g0, count, args)
+    t0 = time.perf_counter()
+    if kind == "bicgstab":
+        out = O.batch_bicgstab(pat.row_ptr, pat.col_idx, Bs.values, Bs.b, tol=args.tol,
+                               maxiter=args.maxiter, threads=cores)
+    else:
+        out = {"x": O.batch_banded(pat.row_ptr, pat.col_idx, Bs.values, Bs.b, threads=cores)}
+    dt = time.perf_counter() - t0
+    return {"value": count / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "algorithm": "Alg. 1 BiCGSTAB + Jacobi (oracle/oracle.c)" if kind == "bicgstab"
+            else "banded LU with partial pivoting, dgbsv-like (oracle/oracle.c)",
+            "sample": f"systems g={g0}..{g0 + count - 1} of the same workload "
+                      f"({count} systems, {dt:.1f} s wall, one system per task over "
+                      f"{cores} host threads)",
+            "cpu": cpu_model(), "_out": out, "_count": count, "_csr": Bs}
+
+
+# --------------------------------------------------------------- reference --
+def run_reference(args, rank, world):
+    """--impl reference: the oracle (as it stands) on the host cores."""
+    if rank != 0:
+        return
+    per_rank = args.batch if args.scaling == "weak" else args.batch // world
+    cal = oracle_sample_rate(0, per_rank, args, target_s=min(5.0, args.cpu_seconds))
+    count = cal["_count"]
+    import oracle as O
+    pat, Bs = make_csr_sample(0, count, args)
+    cores = host_cores()
+    times = []
+    for s in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        O.batch_bicgstab(pat.row_ptr, pat.col_idx, Bs.values, Bs.b, tol=args.tol,
+                         maxiter=args.maxiter, threads=cores)
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            times.append(dt)
+    ms = 1e3 * statistics.mean(times)
+    value = count / (ms * 1e-3)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_dict(args, world, per_rank),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"{count} systems (g=0..{count - 1}) of the workload per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "note": "CPU oracle (oracle/oracle.c, Alg. 1) on the host cores; the paper has no "
+                "public code and this tier has no installable reference",
+    }
+    emit(line, args)
+
+
+def config_dict(args, world, per_rank):
+    n = args.nx * args.ny
+    return {"workload": f"xgc{n}_9pt_mix_zero_guess",
+            "description": "BASELINE configs[3]: 10^5-system batch of XGC-shaped 9-point "
+                           "stencil systems per GPU, 50/50 ion/electron, x0 = 0",
+            "batch_per_gpu": per_rank, "global_batch": per_rank * world, "n": n,
+            "grid": f"{args.nx}x{args.ny}", "format": args.format, "placement": args.placement,
+            "tol": args.tol, "stop": "rel_b", "maxiter": args.maxiter, "x0": "zero",
+            "parallelism": f"batch-partitioned x{world} (one process per GPU, no solve-path "
+                           f"collective)",
+            "l2": "inputs larger than L2 (no flush needed)", "seed": args.seed}
+
+
+def emit(line, args):
+    s = json.dumps(line)
+    print(s, flush=True)
+    if args.out:
+        with open(args.out, "a") as f:
+            f.write(s + "\n")
+
+
+# -------------------------------------------------------------------- ours --
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_kashinksla22_b200 import Solver, probe_smem_bandwidth
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    per_rank = args.batch if args.scaling == "weak" else args.batch // world
+    g0 = rank * per_rank
+    pat, vals_h, b_h = make_inputs(g0, per_rank, args, pinned=True)
+    n, nnz, W = pat.n, pat.nnz, pat.max_row_nnz
+    S = Solver(pat.row_ptr, pat.col_idx, per_rank, format=args.format,
+               placement=args.placement, device=local_rank)
+    vals = vals_h.to(dev, non_blocking=False)
+    b = b_h.to(dev)
+    out = S.alloc_outputs()
+    x, it, res, st = out
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(max(args.warmup, 0)):
+        S.run(vals, b, None, args.tol, args.maxiter, out=out)
+    barrier()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    launch_ms = []
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            e_a = torch.cuda.Event(enable_timing=True)
+            e_b = torch.cuda.Event(enable_timing=True)
+            e_a.record(stream)
+            S.run(vals, b, None, args.tol, args.maxiter, out=out)
+            e_b.record(stream)
+            launch_ms.append((e_a, e_b))
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    total_ms = ev0.elapsed_time(ev1)
+    kern_ms = [a.elapsed_time(bb) for a, bb in launch_ms]
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    value = per_rank * world * args.steps / (total_ms * 1e-3)
+
+    # ---- stats of the last step (outside the timed region) ------------------
+    it_h = it.cpu().numpy()
+    st_h = st.cpu().numpy()
+    res_h = res.cpu().numpy()
+    if world > 1:
+        its = [torch.empty_like(it) for _ in range(world)]
+        dist.all_gather(its, it)
+        sts = [torch.empty_like(st) for _ in range(world)]
+        dist.all_gather(sts, st)
+        it_all = torch.cat(its).cpu().numpy()
+        st_all = torch.cat(sts).cpu().numpy()
+    else:
+        it_all, st_all = it_h, st_h
+    sum_iters_rank = int(it_h.astype(np.int64).sum())
+
+    # ---- roofline (dominant kernel = the one solve kernel per step) ---------
+    import json as _json
+    peaks = {}
+    try:
+        peaks = _json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    info = S.info
+    num_sms = info["num_sms"]
+    sm_max_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+    kern_avg_s = statistics.mean(kern_ms) * 1e-3
+    smem_bytes_iter = 2 * (16 * nnz + 8 * n)
+    smem_bytes_launch = smem_bytes_iter * sum_iters_rank
+    smem_peak = 128.0 * num_sms * sm_max_mhz * 1e6      # guide: 128 B/clk/SM
+    smem_achieved = smem_bytes_launch / kern_avg_s
+    vals_bytes = vals.element_size() * vals.numel() / per_rank
+    hbm_bytes_sys = vals_bytes + 8 * n + 8 * n + 4 + 8 + 1   # values, b, x, iters, resnorm, status
+    hbm_achieved = hbm_bytes_sys * per_rank / kern_avg_s
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0)) * 1e9
+    try:
+        probe_bw, probe_hz = probe_smem_bandwidth(local_rank)
+    except Exception:
+        probe_bw, probe_hz = None, None
+    clocks = clk.summary()
+    roofline = {
+        "bound": "smem", "achieved": smem_achieved / 1e9, "peak": smem_peak / 1e9,
+        "unit": "GB/s", "frac": smem_achieved / smem_peak, "traffic": None,
+        "kernel": "bicgstab_kernel (one launch per step)",
+        "algorithmic_bytes_per_launch": smem_bytes_launch,
+        "algorithmic_bytes_per_unit": f"{smem_bytes_iter} B per BiCGSTAB iteration "
+                                      f"(2 SpMVs x (16 B x nnz + 8 B x n))",
+        "units_per_launch": sum_iters_rank,
+        "peak_source": f"derived: 128 B/clk/SM x {num_sms} SMs x {sm_max_mhz:.0f} MHz "
+                       f"(B300_MICROARCH smem crossbar; no SMEM figure in MEASURED_PEAKS)",
+        "peak_measured_probe": None if probe_bw is None else probe_bw / 1e9,
+        "probe_sm_mhz": None if probe_hz is None else probe_hz / 1e6,
+        "kernel_ms_avg": kern_avg_s * 1e3,
+        "hbm": {"achieved": hbm_achieved / 1e9, "peak": hbm_peak / 1e9, "unit": "GB/s",
+                "frac": hbm_achieved / hbm_peak, "bytes_per_system": hbm_bytes_sys,
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
+    }
+    if clocks.get("sm_mhz"):
+        roofline["frac_at_observed_clock"] = smem_achieved / (128.0 * num_sms *
+                                                              clocks["sm_mhz"] * 1e6)
+
+    # ---- e2e through the public host API (pinned host buffers) -------------
+    e2e = None
+    if not args.no_e2e:
+        x_h = torch.empty((per_rank, n), dtype=torch.float64, pin_memory=True).numpy()
+        i_h = torch.empty(per_rank, dtype=torch.int32, pin_memory=True).numpy()
+        r_h = torch.empty(per_rank, dtype=torch.float64, pin_memory=True).numpy()
+        s_h = torch.empty(per_rank, dtype=torch.int8, pin_memory=True).numpy()
+        vn, bn = vals_h.numpy(), b_h.numpy()
+        outs = (x_h, i_h, r_h, s_h)
+        S.run_host(vn, bn, None, args.tol, args.maxiter, out=outs)  # warm-up (allocates)
+        e2e_steps = max(1, min(args.steps, 3))
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(e2e_steps):
+            S.run_host(vn, bn, None, args.tol, args.maxiter, out=outs)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        dt = float(tt.item())
+        h2d = int(vn.nbytes + bn.nbytes)
+        d2h = int(x_h.nbytes + i_h.nbytes + r_h.nbytes + s_h.nbytes)
+        e2e = {"value": per_rank * world * e2e_steps / dt, "unit": UNIT,
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+               "api": "bsolve_run_host (C ABI, chunked H2D/solve/D2H pipeline)",
+               "bitwise_equal_to_device_path": bool(np.array_equal(i_h, it_h) and
+                                                    np.array_equal(r_h, res_h))}
+
+    # ---- cpu baseline (rank 0, N = 1 only) -------------------------------------
+    cpu = None
+    parity = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cb = oracle_sample_rate(g0, per_rank, args, target_s=args.cpu_seconds)
+        o = cb.pop("_out")
+        cnt = cb.pop("_count")
+        cb.pop("_csr")
+        cpu = cb
+        xo = x[:cnt].cpu().numpy()
+        bnrm = np.linalg.norm(b_h.numpy()[:cnt], axis=1)
+        parity = {"systems_checked": cnt,
+                  "max_iter_diff": int(np.abs(o["iters"][:cnt].astype(int) -
+                                              it_h[:cnt].astype(int)).max()),
+                  "status_equal": bool(np.array_equal(o["status"][:cnt], st_h[:cnt])),
+                  "max_rel_x_diff_vs_oracle_bicgstab": float(np.max(
+                      np.linalg.norm(xo - o["x"], axis=1) / np.linalg.norm(o["x"], axis=1))),
+                  "max_true_rel_residual_gpu": float(np.max(res_h[:cnt] / bnrm))}
+        try:
+            cbl = oracle_sample_rate(g0, per_rank, args, target_s=args.cpu_seconds / 2,
+                                     kind="banded")
+            for k in ("_out", "_count", "_csr"):
+                cbl.pop(k)
+            cpu["banded_lu"] = cbl
+        except Exception as e:  # noqa: BLE001
+            cpu["banded_lu"] = {"error": str(e)}
+
+    ion = it_all[0::2] if (g0 % 2 == 0) else it_all[1::2]
+    ele = it_all[1::2] if (g0 % 2 == 0) else it_all[0::2]
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_dict(args, world, per_rank),
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+        "gpu_launches": args.steps,
+        "plan": info,
+        "solve_stats": {"iters_mean_ion": float(np.mean(ion)), "iters_mean_electron":
+                        float(np.mean(ele)), "iters_max": int(it_all.max()),
+                        "all_converged": bool(np.all(st_all == 0)),
+                        "max_true_rel_residual_rank0": float(np.max(
+                            res_h / np.linalg.norm(b_h.numpy(), axis=1)))},
+        "parity_sample": parity,
+        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms)},
+    }
+    if rank == 0:
+        emit(line, args)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

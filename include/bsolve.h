@@ -1,0 +1,194 @@
+/*
+ * bsolve.h -- C ABI of the B200-native batched sparse iterative solver.
+ *
+ * What it computes (per system i of a batch, independently):
+ *   x_i ~= A_i^{-1} b_i by Algorithm 1 of Kashi et al., IPDPS 2022
+ *   (Sec. IV-D): BiCGSTAB (van der Vorst [18],
+ *   PAPER.md:1240-1243) right-preconditioned with scalar Jacobi
+ *   D_i^{-1} = diag(A_i)^{-1}, stopping each
+ *   system on its own when the residual 2-norm falls below
+ *   tau.  All A_i share ONE sparsity pattern
+ *   (BatchCsr/BatchEll, Sec. IV-A); only values differ.
+ *   The readings of the garbled/silent points of Alg. 1 are DESIGN.md R1-R19.
+ *
+ * Conventions for every entry point
+ *   - Return value: BSOLVE_OK (0) or a negative bsolve_error code.  No C++
+ *     exception ever crosses this ABI.  On error, bsolve_last_error() returns
+ *     a thread-local, human-readable message.
+ *   - Argument validation happens before any CUDA call, synchronously.
+ *   - "device" pointers are CUDA device (or managed) memory of the handle's
+ *     device, 8-byte aligned for double; "host" pointers are ordinary host
+ *     memory (pinned memory makes bsolve_run_host faster but is optional).
+ *   - Asynchronous entry points (bsolve_run, bsolve_spmv, bsolve_csr_to_ell)
+ *     only enqueue work on `stream` (a cudaStream_t; NULL = legacy default
+ *     stream) and never synchronise it.  Numerical outcomes are per system
+ *     and land in iters/resnorm/status on that stream; non-convergence is NOT
+ *     an error return.
+ *   - A handle may be used from one host thread / stream at a time.
+ *   - Everything is fp64 (the paper's precision: LAPACK dgbsv, FP64 peaks in
+ *     Table I, tol 1e-10).
+ */
+#ifndef BSOLVE_H
+#define BSOLVE_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- codes -- */
+typedef enum bsolve_error {
+  BSOLVE_OK = 0,
+  BSOLVE_ERR_INVALID = -1,     /* bad argument: NULL, n<=0, batch<0, tol<0 or
+                                  NaN, maxiter<0, wrong device, bad options    */
+  BSOLVE_ERR_PATTERN = -2,     /* row_ptr not monotone/not starting at 0,
+                                  column out of range, duplicate or unsorted
+                                  column, missing diagonal entry              */
+  BSOLVE_ERR_UNSUPPORTED = -3, /* valid request this build cannot run, e.g.
+                                  forced SMEM placement that does not fit,
+                                  row longer than 32 entries                  */
+  BSOLVE_ERR_CUDA = -4,        /* a CUDA runtime call failed (message has it) */
+  BSOLVE_ERR_NOMEM = -5        /* host or device allocation failed           */
+} bsolve_error;
+
+/* Layout of the per-system `values` array (Fig. 3). */
+enum {
+  BSOLVE_FMT_AUTO = 0, /* resolves to ELL                                      */
+  BSOLVE_FMT_CSR = 1,  /* values[i*nnz + e]: entry e in the CSR order of
+                          (row_ptr, col_idx)  (BatchCsr)     */
+  BSOLVE_FMT_ELL = 2   /* values[i*W*n + k*n + r]: slot k of row r, column-
+                          major (BatchEll).  Slot k
+                          of row r is the k-th CSR entry of row r; slots past
+                          the row's length are padding and MUST hold 0.0.
+                          W = max entries per row (bsolve_info.ell_width).    */
+};
+
+/* Where the matrix values live while a system iterates (PAPER.md:708-721,
+ * 738-813: the paper's automatic shared-memory configuration). */
+enum {
+  BSOLVE_PLACE_AUTO = 0,   /* SMEM if one system's values fit, else STREAM   */
+  BSOLVE_PLACE_SMEM = 1,   /* staged once into shared memory by TMA bulk copy */
+  BSOLVE_PLACE_STREAM = 2  /* re-read from global memory (L2/L1) every SpMV   */
+};
+
+/* Stopping criterion (R5). */
+enum {
+  BSOLVE_STOP_REL_B = 0, /* ||r||_2 < tol * ||b||_2  (default)                */
+  BSOLVE_STOP_ABS = 1    /* ||r||_2 < tol            (paper's experiments,
+                            PAPER.md:869-870)                                  */
+};
+
+/* Per-system outcome written to status[] (R10). */
+enum {
+  BSOLVE_SYS_CONVERGED = 0, /* final TRUE ||b - A x||_2 < tau                 */
+  BSOLVE_SYS_MAXITER = 1,   /* maxiter iterations done without convergence    */
+  BSOLVE_SYS_BREAKDOWN = 2  /* a BiCGSTAB denominator was 0 or non-finite;
+                               x is the last finite iterate                   */
+};
+
+typedef struct bsolve_options {
+  int format;              /* BSOLVE_FMT_*                 (default AUTO)     */
+  int placement;           /* BSOLVE_PLACE_*               (default AUTO)     */
+  int stop;                /* BSOLVE_STOP_*                (default REL_B)    */
+  int true_residual_check; /* 1: recompute ||b - A x|| at exit and restart if
+                              it is >= tau (R4); 0: trust the
+                              recursive residual of Alg. 1  (default 1)       */
+  int device;              /* CUDA device ordinal, -1 = current (default -1)  */
+  int block_threads;       /* threads per CTA, 0 = auto (default 0)          */
+} bsolve_options;
+
+typedef struct bsolve_info {
+  int n, nnz, batch;
+  int ell_width;           /* W = max entries in a row                        */
+  int format, placement;   /* resolved BSOLVE_FMT_* / BSOLVE_PLACE_*          */
+  int block_threads;       /* CTA size used by the solve kernel               */
+  int rows_per_thread;     /* rows each thread owns                           */
+  int smem_bytes;          /* dynamic shared memory per CTA                   */
+  int ctas_per_sm;         /* resident CTAs per SM (occupancy calculator)     */
+  int num_sms;             /* SMs on the device                               */
+  int grid;                /* CTAs launched per bsolve_run                    */
+  int kl, ku;              /* lower / upper bandwidth of the pattern          */
+  int device;
+} bsolve_info;
+
+typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */
+
+/* Fill *opt with the defaults listed above. */
+void bsolve_default_options(bsolve_options *opt);
+
+/* Analyse one shared sparsity pattern and build a solve plan.
+ *   out      [out] receives the handle (NULL on failure).
+ *   n        rows (= columns) of every A_i, n >= 1.
+ *   batch    number of systems each bsolve_run solves, batch >= 0.
+ *   row_ptr  HOST, n+1 int32, row_ptr[0] = 0, non-decreasing.
+ *   col_idx  HOST, row_ptr[n] int32, strictly increasing inside each row,
+ *            every row containing its diagonal (Jacobi needs a_rr).
+ *   opt      NULL for defaults.
+ * The handle copies what it needs; the caller keeps ownership of the arrays.
+ * Errors: INVALID, PATTERN, UNSUPPORTED, CUDA, NOMEM. */
+int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t *row_ptr,
+                  const int32_t *col_idx, const bsolve_options *opt);
+
+/* Solve all `batch` systems (one asynchronous kernel launch).
+ *   values   DEVICE, batch * nnz (CSR) or batch * W * n (ELL) doubles.
+ *   b        DEVICE, batch * n doubles (read only).
+ *   x0       DEVICE, batch * n doubles, or NULL for the zero guess; may alias
+ *            x (warm start "x in/out").
+ *   tol      >= 0, finite.  maxiter >= 0 (0 returns x = x0, iters = 0).
+ *   x        DEVICE, batch * n doubles (out).
+ *   iters    DEVICE, batch int32 (out): executions of "v <- A p^" (R8).
+ *   resnorm  DEVICE, batch doubles (out): final TRUE ||b - A x||_2, absolute.
+ *   status   DEVICE, batch int8 (out) or NULL: BSOLVE_SYS_*.
+ *   stream   cudaStream_t or NULL.
+ * Caller owns all buffers; they must stay valid until the stream reaches
+ * this work.  b = 0 under REL_B gives x = 0, iters = 0, CONVERGED. */
+int bsolve_run(bsolve_handle h, const double *values, const double *b, const double *x0,
+               double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
+               int8_t *status, void *stream);
+
+/* Same computation with HOST buffers (same shapes as bsolve_run; x0 and
+ * status may be NULL).  The library streams the batch through the device in
+ * chunks: host->device copies, solve and device->host copies of successive
+ * chunks overlap on internal streams.  Synchronous: returns when x, iters,
+ * resnorm, status are written.  Pinned (page-locked) host memory is needed
+ * for the copies to overlap; pageable memory works but serialises. */
+int bsolve_run_host(bsolve_handle h, const double *values, const double *b, const double *x0,
+                    double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
+                    int8_t *status);
+
+/* Batched SpMV y_i = A_i x_i for `batch` systems (
+ * the Fig. 7 microbenchmark).  values in the handle's
+ * format; x, y DEVICE batch * n doubles (y must not alias x). Asynchronous. */
+int bsolve_spmv(bsolve_handle h, const double *values, const double *x, double *y, int batch,
+                void *stream);
+
+/* Re-layout CSR-ordered values (batch * nnz) into the handle's ELL layout
+ * (batch * W * n, zero padding).  DEVICE pointers, must not overlap.
+ * Asynchronous.  Bit-exact: a pure permutation with zero fill. */
+int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, double *ell_values, int batch,
+                      void *stream);
+
+/* Describe the plan (see bsolve_info). */
+int bsolve_query(bsolve_handle h, bsolve_info *info);
+
+/* Copy the ELL column indices (W * n int32, column-major, padding slots hold
+ * their own row) to HOST memory `out`. */
+int bsolve_ell_cols(bsolve_handle h, int32_t *out);
+
+/* Release the handle and its device memory.  NULL-safe; returns BSOLVE_OK. */
+int bsolve_destroy(bsolve_handle h);
+
+/* Message of the last non-OK return on the calling thread ("" if none). */
+const char *bsolve_last_error(void);
+
+/* Measure this device's shared-memory load bandwidth (bytes/s) with a
+ * streaming LDS.128 kernel over all SMs; used as a measured roofline
+ * denominator by bench.py.  Synchronous.  Writes *bytes_per_s and the SM
+ * clock the kernel saw (*sm_hz, from clock64 over the event time). */
+int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BSOLVE_H */

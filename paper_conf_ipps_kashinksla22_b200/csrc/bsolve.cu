@@ -1,0 +1,569 @@
+// bsolve.cu -- host side of the C ABI declared in include/bsolve.h.
+//
+// bsolve_create analyses the shared pattern once (validation, diagonal slot
+// per row, ELL column indices, bandwidth) and chooses the kernel variant
+// (format x placement x rows-per-thread x CTA size) and its dynamic shared
+// memory -- the B200 analogue of the paper's automatic shared-memory
+// configuration and block-size tuning (Sec. IV-D;
+// PAPER.md:836-850, Sec. IV-E).  bsolve_run validates arguments and enqueues
+// ONE kernel launch on the caller's stream.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/bsolve.h"
+#include "kernels.cuh"
+
+using namespace bsolve;
+
+// ------------------------------------------------------------- errors --
+static thread_local std::string g_err;
+
+static int fail(int code, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CUDA_TRY(call)                                                                    \
+  do {                                                                                    \
+    cudaError_t e_ = (call);                                                              \
+    if (e_ != cudaSuccess)                                                                \
+      return fail(BSOLVE_ERR_CUDA, "%s failed: %s", #call, cudaGetErrorString(e_));       \
+  } while (0)
+
+// ------------------------------------------------------- kernel table --
+typedef void (*solve_fn)(const SolveParams);
+
+struct Variant {
+  int fmt, place, wb, r, nt;
+  solve_fn fn;
+};
+
+#define V_(F, PL, WB, R, NT, MB) \
+  {F, PL, WB, R, NT, (solve_fn)bicgstab_kernel<F, PL, WB, R, NT, MB>}
+#define V_FP(WB, R, NT, MB)                                                     \
+  V_(FMT_ELL, PLACE_SMEM, WB, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, R, NT, MB), \
+      V_(FMT_CSR, PLACE_SMEM, WB, R, NT, MB), V_(FMT_CSR, PLACE_STREAM, WB, R, NT, MB)
+
+static const Variant kVariants[] = {
+    V_FP(9, 1, 256, 2),  V_FP(9, 2, 256, 2),  V_FP(9, 4, 256, 2),  V_FP(9, 4, 512, 1),
+    V_FP(16, 1, 256, 2), V_FP(16, 2, 256, 2), V_FP(16, 4, 256, 2), V_FP(16, 4, 512, 1),
+};
+
+static const Variant *find_variant(int fmt, int place, int wb, int r, int nt) {
+  for (const Variant &v : kVariants)
+    if (v.fmt == fmt && v.place == place && v.wb == wb && v.r == r && v.nt == nt) return &v;
+  return nullptr;
+}
+
+// ------------------------------------------------------------- handle --
+struct bsolve_plan {
+  int n = 0, nnz = 0, batch = 0, W = 0, wb = 0;
+  int fmt = 0, place = 0, stop = 0, trc = 1, device = 0;
+  int nt = 0, r = 0, smem_bytes = 0, smem_vals = 0, n_pad = 0, ctas_per_sm = 0, num_sms = 0;
+  int kl = 0, ku = 0;
+  long long sys_stride = 0;
+  const Variant *var = nullptr;
+  std::vector<int32_t> h_ell_col;  // [W][n]
+  std::vector<int32_t> h_csr2ell;  // [W][n] -> CSR entry or -1
+  int32_t *d_ell_col = nullptr, *d_row_ptr = nullptr, *d_diag = nullptr, *d_src = nullptr;
+  // bsolve_run_host pipeline (lazily allocated)
+  static constexpr int kSlots = 3;
+  cudaStream_t hs[kSlots] = {nullptr, nullptr, nullptr};
+  int h_chunk = 0;
+  double *h_val[kSlots] = {}, *h_b[kSlots] = {}, *h_x0[kSlots] = {}, *h_x[kSlots] = {},
+         *h_res[kSlots] = {};
+  int32_t *h_it[kSlots] = {};
+  int8_t *h_st[kSlots] = {};
+};
+
+extern "C" void bsolve_default_options(bsolve_options *o) {
+  if (!o) return;
+  o->format = BSOLVE_FMT_AUTO;
+  o->placement = BSOLVE_PLACE_AUTO;
+  o->stop = BSOLVE_STOP_REL_B;
+  o->true_residual_check = 1;
+  o->device = -1;
+  o->block_threads = 0;
+}
+
+static void free_plan(bsolve_plan *h) {
+  if (!h) return;
+  int cur = -1;
+  cudaGetDevice(&cur);
+  cudaSetDevice(h->device);
+  cudaFree(h->d_ell_col);
+  cudaFree(h->d_row_ptr);
+  cudaFree(h->d_diag);
+  cudaFree(h->d_src);
+  for (int s = 0; s < bsolve_plan::kSlots; ++s) {
+    if (h->hs[s]) cudaStreamDestroy(h->hs[s]);
+    cudaFree(h->h_val[s]);
+    cudaFree(h->h_b[s]);
+    cudaFree(h->h_x0[s]);
+    cudaFree(h->h_x[s]);
+    cudaFree(h->h_res[s]);
+    cudaFree(h->h_it[s]);
+    cudaFree(h->h_st[s]);
+  }
+  if (cur >= 0) cudaSetDevice(cur);
+  delete h;
+}
+
+// Validate the shared CSR pattern; fills diag slot per row. Pure host code.
+static int validate_pattern(int n, const int32_t *rp, const int32_t *ci, std::vector<int32_t> &diag,
+                            int &W) {
+  if (rp[0] != 0) return fail(BSOLVE_ERR_PATTERN, "row_ptr[0] = %d, expected 0", rp[0]);
+  diag.assign(n, -1);
+  W = 0;
+  for (int i = 0; i < n; ++i) {
+    if (rp[i + 1] < rp[i])
+      return fail(BSOLVE_ERR_PATTERN, "row_ptr decreases at row %d (%d -> %d)", i, rp[i], rp[i + 1]);
+    W = std::max(W, rp[i + 1] - rp[i]);
+    for (int e = rp[i]; e < rp[i + 1]; ++e) {
+      const int c = ci[e];
+      if (c < 0 || c >= n)
+        return fail(BSOLVE_ERR_PATTERN, "col_idx[%d] = %d out of range [0, %d)", e, c, n);
+      if (e > rp[i] && c <= ci[e - 1])
+        return fail(BSOLVE_ERR_PATTERN, "row %d: columns not strictly increasing at entry %d", i, e);
+      if (c == i) diag[i] = e - rp[i];
+    }
+    if (diag[i] < 0) return fail(BSOLVE_ERR_PATTERN, "row %d has no diagonal entry", i);
+  }
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t *row_ptr,
+                             const int32_t *col_idx, const bsolve_options *opt_in) {
+  g_err.clear();
+  if (!out) return fail(BSOLVE_ERR_INVALID, "out is NULL");
+  *out = nullptr;
+  if (n <= 0) return fail(BSOLVE_ERR_INVALID, "n = %d must be >= 1", n);
+  if (batch < 0) return fail(BSOLVE_ERR_INVALID, "batch = %d must be >= 0", batch);
+  if (!row_ptr || !col_idx) return fail(BSOLVE_ERR_INVALID, "row_ptr/col_idx is NULL");
+  bsolve_options opt;
+  bsolve_default_options(&opt);
+  if (opt_in) opt = *opt_in;
+  if (opt.format < BSOLVE_FMT_AUTO || opt.format > BSOLVE_FMT_ELL)
+    return fail(BSOLVE_ERR_INVALID, "bad format %d", opt.format);
+  if (opt.placement < BSOLVE_PLACE_AUTO || opt.placement > BSOLVE_PLACE_STREAM)
+    return fail(BSOLVE_ERR_INVALID, "bad placement %d", opt.placement);
+  if (opt.stop != BSOLVE_STOP_REL_B && opt.stop != BSOLVE_STOP_ABS)
+    return fail(BSOLVE_ERR_INVALID, "bad stop mode %d", opt.stop);
+  if (opt.block_threads != 0 && opt.block_threads != 256 && opt.block_threads != 512)
+    return fail(BSOLVE_ERR_INVALID, "block_threads must be 0, 256 or 512 (got %d)",
+                opt.block_threads);
+
+  std::vector<int32_t> diag;
+  int W = 0;
+  int rc = validate_pattern(n, row_ptr, col_idx, diag, W);
+  if (rc) return rc;
+  const int nnz = row_ptr[n];
+  if (W > 16)
+    return fail(BSOLVE_ERR_UNSUPPORTED, "rows with %d > 16 entries are not supported", W);
+  if ((long long)n * 8 >= 65536)
+    return fail(BSOLVE_ERR_UNSUPPORTED, "n = %d too large (packed 16-bit gather offsets need n < 8192)", n);
+
+  bsolve_plan *h = new (std::nothrow) bsolve_plan();
+  if (!h) return fail(BSOLVE_ERR_NOMEM, "host allocation failed");
+  h->n = n;
+  h->nnz = nnz;
+  h->batch = batch;
+  h->W = W;
+  h->wb = W <= 9 ? 9 : 16;
+  h->fmt = opt.format == BSOLVE_FMT_CSR ? FMT_CSR : FMT_ELL;
+  h->stop = opt.stop;
+  h->trc = opt.true_residual_check ? 1 : 0;
+  h->sys_stride = h->fmt == FMT_ELL ? (long long)W * n : nnz;
+
+  // bandwidth (for bsolve_info; the banded structure is not used by the solve)
+  for (int i = 0; i < n; ++i)
+    for (int e = row_ptr[i]; e < row_ptr[i + 1]; ++e) {
+      h->kl = std::max(h->kl, i - col_idx[e]);
+      h->ku = std::max(h->ku, col_idx[e] - i);
+    }
+  // ELL columns: slot k of row i = k-th CSR entry; padding -> own row
+  h->h_ell_col.assign((size_t)W * n, 0);
+  h->h_csr2ell.assign((size_t)W * n, -1);
+  for (int i = 0; i < n; ++i)
+    for (int k = 0; k < W; ++k) {
+      const int e = row_ptr[i] + k;
+      const bool real = e < row_ptr[i + 1];
+      h->h_ell_col[(size_t)k * n + i] = real ? col_idx[e] : i;
+      h->h_csr2ell[(size_t)k * n + i] = real ? e : -1;
+    }
+
+  // ---- device + variant choice -------------------------------------------
+  int dev = opt.device;
+  if (dev < 0) {
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) {
+      delete h;
+      return fail(BSOLVE_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(e));
+    }
+  }
+  h->device = dev;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  auto fail_free = [&](int code) {
+    free_plan(h);
+    if (prev >= 0) cudaSetDevice(prev);
+    return code;
+  };
+  cudaError_t ce = cudaSetDevice(dev);
+  if (ce != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_CUDA, "cudaSetDevice(%d): %s", dev, cudaGetErrorString(ce)));
+  cudaDeviceProp prop;
+  ce = cudaGetDeviceProperties(&prop, dev);
+  if (ce != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_CUDA, "cudaGetDeviceProperties: %s", cudaGetErrorString(ce)));
+  h->num_sms = prop.multiProcessorCount;
+  const int smem_optin = (int)prop.sharedMemPerBlockOptin;
+
+  // rows per thread / CTA size: prefer 256 threads (2 CTAs per SM fit the
+  // register file at <= 128 regs/thread), 512 threads for 1025..2048 rows.
+  int nt = opt.block_threads;
+  if (nt == 0) nt = n <= 1024 ? 256 : 512;
+  int r = (n + nt - 1) / nt;
+  if (r == 3) r = 4;
+  if (nt == 512) r = 4;  // the 512-thread variants own 4 rows per thread
+  if (r > 4)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                          "n = %d needs more than 4 rows per thread at %d threads", n, nt));
+  h->nt = nt;
+  h->r = r;
+  h->n_pad = (n + 1) & ~1;
+  h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
+  const int nwarp = nt / 32;
+  const int tail = h->n_pad * 8 + 2 * nwarp * 4 * 8 + 16;
+  const long long smem_need = (long long)h->smem_vals * 8 + tail;
+  int place = opt.placement;
+  if (place == BSOLVE_PLACE_AUTO) place = smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM;
+  else place = place == BSOLVE_PLACE_SMEM ? PLACE_SMEM : PLACE_STREAM;
+  if (place == PLACE_SMEM && smem_need > smem_optin)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                          "SMEM placement needs %lld B of shared memory, device allows %d",
+                          smem_need, smem_optin));
+  h->place = place;
+  h->smem_bytes = (int)(place == PLACE_SMEM ? smem_need : tail);
+  h->var = find_variant(h->fmt, place, h->wb, r, nt);
+  if (!h->var)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
+                          h->fmt, place, h->wb, r, nt));
+  ce = cudaFuncSetAttribute((const void *)h->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            h->smem_bytes);
+  if (ce != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+  cudaFuncSetAttribute((const void *)h->var->fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                       cudaSharedmemCarveoutMaxShared);
+  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var->fn, nt, h->smem_bytes);
+  if (ce != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_CUDA, "occupancy query: %s", cudaGetErrorString(ce)));
+  if (h->ctas_per_sm < 1)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "kernel variant cannot be resident on an SM"));
+
+  // ---- device copy of the pattern ------------------------------------------
+  std::vector<int32_t> rp(row_ptr, row_ptr + n + 1);
+  const size_t ell_b = sizeof(int32_t) * (size_t)W * n;
+  if (cudaMalloc(&h->d_ell_col, ell_b) != cudaSuccess ||
+      cudaMalloc(&h->d_src, ell_b) != cudaSuccess ||
+      cudaMalloc(&h->d_row_ptr, sizeof(int32_t) * (n + 1)) != cudaSuccess ||
+      cudaMalloc(&h->d_diag, sizeof(int32_t) * n) != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_NOMEM, "device allocation of the pattern failed"));
+  if (cudaMemcpy(h->d_ell_col, h->h_ell_col.data(), ell_b, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(h->d_src, h->h_csr2ell.data(), ell_b, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(h->d_row_ptr, rp.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice) !=
+          cudaSuccess ||
+      cudaMemcpy(h->d_diag, diag.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice) != cudaSuccess)
+    return fail_free(fail(BSOLVE_ERR_CUDA, "copy of the pattern to the device failed"));
+  if (prev >= 0) cudaSetDevice(prev);
+  *out = h;
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_destroy(bsolve_handle h) {
+  free_plan(h);
+  return BSOLVE_OK;
+}
+
+extern "C" const char *bsolve_last_error(void) { return g_err.c_str(); }
+
+extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
+  if (!h || !info) return fail(BSOLVE_ERR_INVALID, "NULL handle or info");
+  info->n = h->n;
+  info->nnz = h->nnz;
+  info->batch = h->batch;
+  info->ell_width = h->W;
+  info->format = h->fmt == FMT_ELL ? BSOLVE_FMT_ELL : BSOLVE_FMT_CSR;
+  info->placement = h->place == PLACE_SMEM ? BSOLVE_PLACE_SMEM : BSOLVE_PLACE_STREAM;
+  info->block_threads = h->nt;
+  info->rows_per_thread = h->r;
+  info->smem_bytes = h->smem_bytes;
+  info->ctas_per_sm = h->ctas_per_sm;
+  info->num_sms = h->num_sms;
+  info->grid = h->batch;
+  info->kl = h->kl;
+  info->ku = h->ku;
+  info->device = h->device;
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_ell_cols(bsolve_handle h, int32_t *out) {
+  if (!h || !out) return fail(BSOLVE_ERR_INVALID, "NULL handle or out");
+  std::memcpy(out, h->h_ell_col.data(), sizeof(int32_t) * h->h_ell_col.size());
+  return BSOLVE_OK;
+}
+
+// ------------------------------------------------------------------ run --
+static int check_run_args(bsolve_handle h, const double *values, const double *b, double tol,
+                          int maxiter, const double *x, const int32_t *iters,
+                          const double *resnorm) {
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (h->batch > 0 && (!values || !b || !x || !iters || !resnorm))
+    return fail(BSOLVE_ERR_INVALID, "values, b, x, iters and resnorm must be non-NULL");
+  if (!(tol >= 0.0) || !std::isfinite(tol))
+    return fail(BSOLVE_ERR_INVALID, "tol = %g must be finite and >= 0", tol);
+  if (maxiter < 0) return fail(BSOLVE_ERR_INVALID, "maxiter = %d must be >= 0", maxiter);
+  return BSOLVE_OK;
+}
+
+static int launch_solve(bsolve_handle h, const double *values, const double *b, const double *x0,
+                        double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
+                        int8_t *status, int count, cudaStream_t stream) {
+  if (count <= 0) return BSOLVE_OK;
+  SolveParams P;
+  P.values = values;
+  P.b = b;
+  P.x0 = x0;
+  P.x = x;
+  P.iters = iters;
+  P.resnorm = resnorm;
+  P.status = status;
+  P.ell_col = h->d_ell_col;
+  P.row_ptr = h->d_row_ptr;
+  P.diag_slot = h->d_diag;
+  P.sys_stride = h->sys_stride;
+  P.tol = tol;
+  P.n = h->n;
+  P.W = h->W;
+  P.batch = count;
+  P.maxiter = maxiter;
+  P.stop = h->stop;
+  P.trc = h->trc;
+  P.smem_vals = h->smem_vals;
+  P.n_pad = h->n_pad;
+  h->var->fn<<<count, h->nt, h->smem_bytes, stream>>>(P);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));
+  return BSOLVE_OK;
+}
+
+static int check_device_ptr(bsolve_handle h, const void *p, const char *name) {
+  if (!p) return BSOLVE_OK;
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BSOLVE_ERR_INVALID, "%s is not a CUDA pointer (%s)", name, cudaGetErrorString(e));
+  }
+  if (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged)
+    return fail(BSOLVE_ERR_INVALID, "%s must be device memory", name);
+  if (a.type == cudaMemoryTypeDevice && a.device != h->device)
+    return fail(BSOLVE_ERR_INVALID, "%s lives on device %d, handle is on device %d", name, a.device,
+                h->device);
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_run(bsolve_handle h, const double *values, const double *b, const double *x0,
+                          double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
+                          int8_t *status, void *stream) {
+  g_err.clear();
+  int rc = check_run_args(h, values, b, tol, maxiter, x, iters, resnorm);
+  if (rc) return rc;
+  if (h->batch == 0) return BSOLVE_OK;
+  const void *ptrs[] = {values, b, x0, x, iters, resnorm, status};
+  const char *names[] = {"values", "b", "x0", "x", "iters", "resnorm", "status"};
+  for (int i = 0; i < 7; ++i)
+    if ((rc = check_device_ptr(h, ptrs[i], names[i]))) return rc;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  rc = launch_solve(h, values, b, x0, tol, maxiter, x, iters, resnorm, status, h->batch,
+                    (cudaStream_t)stream);
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  return rc;
+}
+
+extern "C" int bsolve_run_host(bsolve_handle h, const double *values, const double *b,
+                               const double *x0, double tol, int maxiter, double *x, int32_t *iters,
+                               double *resnorm, int8_t *status) {
+  g_err.clear();
+  int rc = check_run_args(h, values, b, tol, maxiter, x, iters, resnorm);
+  if (rc) return rc;
+  if (h->batch == 0) return BSOLVE_OK;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  const int n = h->n;
+  const long long ss = h->sys_stride;
+  if (h->h_chunk == 0) {
+    // ~64 MB of values per chunk, rounded to whole waves of resident CTAs
+    const long long wave = (long long)h->num_sms * h->ctas_per_sm;
+    long long c = std::max<long long>(wave, (64ll << 20) / (ss * 8));
+    c = (c + wave - 1) / wave * wave;
+    c = std::min<long long>(c, h->batch);
+    h->h_chunk = (int)std::max<long long>(c, 1);
+    for (int s = 0; s < bsolve_plan::kSlots; ++s) {
+      CUDA_TRY(cudaStreamCreateWithFlags(&h->hs[s], cudaStreamNonBlocking));
+      const size_t c_ = (size_t)h->h_chunk;
+      if (cudaMalloc(&h->h_val[s], c_ * ss * 8) != cudaSuccess ||
+          cudaMalloc(&h->h_b[s], c_ * n * 8) != cudaSuccess ||
+          cudaMalloc(&h->h_x0[s], c_ * n * 8) != cudaSuccess ||
+          cudaMalloc(&h->h_x[s], c_ * n * 8) != cudaSuccess ||
+          cudaMalloc(&h->h_res[s], c_ * 8) != cudaSuccess ||
+          cudaMalloc(&h->h_it[s], c_ * 4) != cudaSuccess ||
+          cudaMalloc(&h->h_st[s], c_) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(BSOLVE_ERR_NOMEM, "device allocation for the host pipeline failed");
+      }
+    }
+  }
+  const int C = h->h_chunk;
+  int k = 0;
+  for (long long s0 = 0; s0 < h->batch; s0 += C, ++k) {
+    const int cnt = (int)std::min<long long>(C, h->batch - s0);
+    const int sl = k % bsolve_plan::kSlots;
+    cudaStream_t st = h->hs[sl];
+    CUDA_TRY(cudaMemcpyAsync(h->h_val[sl], values + s0 * ss, (size_t)cnt * ss * 8,
+                             cudaMemcpyHostToDevice, st));
+    CUDA_TRY(cudaMemcpyAsync(h->h_b[sl], b + s0 * n, (size_t)cnt * n * 8, cudaMemcpyHostToDevice, st));
+    if (x0)
+      CUDA_TRY(cudaMemcpyAsync(h->h_x0[sl], x0 + s0 * n, (size_t)cnt * n * 8,
+                               cudaMemcpyHostToDevice, st));
+    rc = launch_solve(h, h->h_val[sl], h->h_b[sl], x0 ? h->h_x0[sl] : nullptr, tol, maxiter,
+                      h->h_x[sl], h->h_it[sl], h->h_res[sl], h->h_st[sl], cnt, st);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(x + s0 * n, h->h_x[sl], (size_t)cnt * n * 8, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaMemcpyAsync(iters + s0, h->h_it[sl], (size_t)cnt * 4, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaMemcpyAsync(resnorm + s0, h->h_res[sl], (size_t)cnt * 8, cudaMemcpyDeviceToHost, st));
+    if (status)
+      CUDA_TRY(cudaMemcpyAsync(status + s0, h->h_st[sl], (size_t)cnt, cudaMemcpyDeviceToHost, st));
+  }
+  for (int s = 0; s < bsolve_plan::kSlots; ++s) CUDA_TRY(cudaStreamSynchronize(h->hs[s]));
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_spmv(bsolve_handle h, const double *values, const double *x, double *y,
+                           int batch, void *stream) {
+  g_err.clear();
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (batch < 0) return fail(BSOLVE_ERR_INVALID, "batch = %d must be >= 0", batch);
+  if (batch == 0) return BSOLVE_OK;
+  if (!values || !x || !y) return fail(BSOLVE_ERR_INVALID, "values, x and y must be non-NULL");
+  if (x == y) return fail(BSOLVE_ERR_INVALID, "y must not alias x");
+  int rc;
+  const void *ptrs[] = {values, x, y};
+  const char *names[] = {"values", "x", "y"};
+  for (int i = 0; i < 3; ++i)
+    if ((rc = check_device_ptr(h, ptrs[i], names[i]))) return rc;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  const size_t sm = sizeof(double) * h->n;
+  if (h->fmt == FMT_ELL) {
+    if (sm > 48 * 1024)
+      CUDA_TRY(cudaFuncSetAttribute((const void *)spmv_kernel<FMT_ELL, 256>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    spmv_kernel<FMT_ELL, 256><<<batch, 256, sm, (cudaStream_t)stream>>>(
+        values, x, y, h->d_ell_col, h->d_row_ptr, h->n, h->W, h->sys_stride);
+  } else {
+    if (sm > 48 * 1024)
+      CUDA_TRY(cudaFuncSetAttribute((const void *)spmv_kernel<FMT_CSR, 256>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    spmv_kernel<FMT_CSR, 256><<<batch, 256, sm, (cudaStream_t)stream>>>(
+        values, x, y, h->d_ell_col, h->d_row_ptr, h->n, h->W, h->sys_stride);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "spmv launch: %s", cudaGetErrorString(e));
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, double *ell_values,
+                                 int batch, void *stream) {
+  g_err.clear();
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (batch < 0) return fail(BSOLVE_ERR_INVALID, "batch = %d must be >= 0", batch);
+  if (batch == 0) return BSOLVE_OK;
+  if (!csr_values || !ell_values) return fail(BSOLVE_ERR_INVALID, "NULL values");
+  int rc;
+  if ((rc = check_device_ptr(h, csr_values, "csr_values"))) return rc;
+  if ((rc = check_device_ptr(h, ell_values, "ell_values"))) return rc;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  const long long slots = (long long)h->W * h->n;
+  const long long total = slots * batch;
+  const int blocks = (int)std::min<long long>((total + 255) / 256, (long long)h->num_sms * 16);
+  csr_to_ell_kernel<<<blocks, 256, 0, (cudaStream_t)stream>>>(csr_values, ell_values, h->d_src,
+                                                               slots, h->nnz, total);
+  cudaError_t e = cudaGetLastError();
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "csr_to_ell launch: %s", cudaGetErrorString(e));
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz) {
+  g_err.clear();
+  if (!bytes_per_s || !sm_hz) return fail(BSOLVE_ERR_INVALID, "NULL output");
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (device < 0) device = prev;
+  CUDA_TRY(cudaSetDevice(device));
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, device));
+  const int grid = prop.multiProcessorCount * 2, iters = 1 << 14;
+  constexpr int NT = 512;
+  double *sink = nullptr;
+  long long *cyc = nullptr;
+  CUDA_TRY(cudaMalloc(&sink, sizeof(double) * grid));
+  CUDA_TRY(cudaMalloc(&cyc, sizeof(long long) * grid));
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  smem_probe_kernel<NT><<<grid, NT>>>(64, sink, cyc);  // warm-up
+  cudaEventRecord(e0);
+  smem_probe_kernel<NT><<<grid, NT>>>(iters, sink, cyc);
+  cudaEventRecord(e1);
+  cudaError_t e = cudaEventSynchronize(e1);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  std::vector<long long> hc(grid);
+  cudaMemcpy(hc.data(), cyc, sizeof(long long) * grid, cudaMemcpyDeviceToHost);
+  cudaFree(sink);
+  cudaFree(cyc);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (prev >= 0) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "smem probe: %s", cudaGetErrorString(e));
+  const double bytes = (double)grid * NT * iters * 4 * 32;
+  *bytes_per_s = bytes / (ms * 1e-3);
+  long long mx = 0;
+  for (long long c : hc) mx = std::max(mx, c);
+  *sm_hz = (double)mx / (ms * 1e-3);
+  return BSOLVE_OK;
+}

@@ -1,0 +1,515 @@
+// kernels.cuh -- sm_100a device code of the batched Jacobi-BiCGSTAB solver.
+//
+// One CTA solves one system end to end: the whole
+// Algorithm 1 loop runs inside a single kernel launch
+// and each system stops on its own.
+//
+// B200 design:
+//  * the system's matrix values (71,424 B for the 992-row 9-point ELL case)
+//    are staged ONCE into shared memory with a TMA bulk copy
+//    (cp.async.bulk + mbarrier complete_tx) while the threads load b, x0 and
+//    the shared pattern; every SpMV then reads values and the gathered vector
+//    from SMEM (PLACE_SMEM).  PLACE_STREAM re-reads values from global
+//    memory (L2/L1) instead, for systems whose values do not fit.
+//  * every BiCGSTAB vector lives in REGISTERS: thread t owns rows t + j*NT,
+//    j < R.  Only the vector being multiplied (p^ or s^) is published to a
+//    shared "gather" buffer for the SpMV.
+//  * column indices are held in registers as packed 16-bit byte offsets into
+//    the gather buffer (read once per CTA from the shared pattern in L2).
+//  * dot products and norms are fused into the vector updates and reduced
+//    warp-shuffle -> one __syncthreads -> redundant per-thread final sum over
+//    the NT/32 warp partials, so every reduction costs exactly one barrier
+//    and all threads hold bitwise-identical scalars (uniform control flow,
+//    deterministic results independent of batch partitioning).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace bsolve {
+
+enum { FMT_CSR = 1, FMT_ELL = 2 };
+enum { PLACE_SMEM = 1, PLACE_STREAM = 2 };
+enum { STOP_REL_B = 0, STOP_ABS = 1 };
+enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
+
+struct SolveParams {
+  const double *values;     // [batch][sys_stride]
+  const double *b;          // [batch][n]
+  const double *x0;         // [batch][n] or nullptr
+  double *x;                // [batch][n]
+  int32_t *iters;           // [batch]
+  double *resnorm;          // [batch]
+  int8_t *status;           // [batch] or nullptr
+  const int32_t *ell_col;   // [W][n] shared pattern, column-major
+  const int32_t *row_ptr;   // [n+1]
+  const int32_t *diag_slot; // [n] slot of the diagonal entry in its row
+  long long sys_stride;     // doubles per system in `values`
+  double tol;
+  int n, W, batch, maxiter, stop, trc;
+  int smem_vals;            // doubles of SMEM reserved for values (even)
+  int n_pad;                // doubles of the gather buffer (even)
+};
+
+// ------------------------------------------------------------ PTX helpers --
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count)
+               : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
+               "r"(bytes)
+               : "memory");
+}
+// TMA bulk copy global -> shared, completion counted on `bar` in bytes.
+__device__ __forceinline__ void tma_bulk_g2s(void *dst, const void *src, uint32_t bytes,
+                                             uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
+
+// Block-wide sum of K doubles: warp butterfly (all lanes end bitwise equal),
+// lane 0 publishes, ONE barrier, then every thread sums the NWARP partials
+// in warp order.  `buf` alternates between two scratch halves so that the
+// next reduction never overwrites partials a slow thread is still reading.
+template <int K, int NWARP>
+__device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf, int lane,
+                                          int warp) {
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v[k] += __shfl_xor_sync(0xffffffffu, v[k], o);
+  }
+  double *S = sred + buf * (NWARP * 4);
+  if (lane == 0) {
+#pragma unroll
+    for (int k = 0; k < K; ++k) S[warp * 4 + k] = v[k];
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    double a = 0.0;
+#pragma unroll
+    for (int w = 0; w < NWARP; ++w) a += S[w * 4 + k];
+    v[k] = a;
+  }
+  buf ^= 1;
+}
+
+// Per-thread view of its rows of the shared pattern.
+template <int WB, int R>
+struct RowMeta {
+  uint32_t cpk[R][(WB + 1) / 2]; // packed 16-bit byte offsets (col*8) into the gather buffer
+  int vbase[R];                  // ELL: row; CSR: row_ptr[row]
+  int vlen[R];                   // CSR row length
+  bool act[R];                   // row < n
+};
+
+// y = A * g for this thread's rows; g is the shared gather buffer sg;
+// values come from V (shared or global).
+// Extract the 16-bit field at bit `pos` of `pk`.  volatile: keeps the unpack
+// inside the SpMV loop instead of letting the compiler hoist 2x as many
+// unpacked offsets into registers (which spills at R = 4).
+template <int POS>
+__device__ __forceinline__ uint32_t field16(uint32_t pk) {
+  uint32_t v;
+  asm volatile("bfe.u32 %0, %1, %2, 16;" : "=r"(v) : "r"(pk), "n"(POS));
+  return v;
+}
+
+template <int FMT, int PLACE, int WB, int R, int NT>
+__device__ __forceinline__ void spmv_rows(const double *__restrict__ V, const double *sg, int n,
+                                          int W, const RowMeta<WB, R> &m, double (&y)[R]) {
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+  const double *Vt = V + threadIdx.x;  // ELL: slot k of row tid + j*NT at Vt[k*n + j*NT]
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    double acc = 0.0;
+    if (m.act[j]) {
+#pragma unroll
+      for (int k = 0; k < WB; ++k) {
+        if (k < W) {
+          const uint32_t off = (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+          const double g = *reinterpret_cast<const double *>(gb + off);
+          if (FMT == FMT_ELL) {
+            const double a = (PLACE == PLACE_STREAM) ? __ldg(Vt + (size_t)k * n + j * NT)
+                                                     : Vt[k * n + j * NT];
+            acc = fma(a, g, acc);
+          } else {
+            if (k < m.vlen[j]) {
+              const double a = (PLACE == PLACE_STREAM) ? __ldg(V + m.vbase[j] + k)
+                                                       : V[m.vbase[j] + k];
+              acc = fma(a, g, acc);
+            }
+          }
+        }
+      }
+    }
+    y[j] = acc;
+  }
+}
+
+// ------------------------------------------------------------ the solver --
+// Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
+//   [values: smem_vals doubles (PLACE_SMEM only)] [gather: n_pad doubles]
+//   [reduction scratch: 2*NWARP*4 doubles] [mbarrier: 8 B]
+template <int FMT, int PLACE, int WB, int R, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
+  constexpr int NWARP = NT / 32;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sg = sval + (PLACE == PLACE_SMEM ? P.smem_vals : 0);
+  double *sred = sg + P.n_pad;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 2 * NWARP * 4);
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int n = P.n, W = P.W;
+  const long long sys = blockIdx.x;
+  const double *gval = P.values + sys * P.sys_stride;
+
+  // ---- a1: stage this system's values into SMEM (TMA bulk copy) ----------
+  bool use_tma = false;
+  if (PLACE == PLACE_SMEM) {
+    const uint32_t bytes = static_cast<uint32_t>(P.sys_stride * 8);
+    use_tma = (bytes % 16u == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0);
+    if (use_tma) {
+      if (tid == 0) {
+        mbar_init(mbar, 1);
+        fence_mbar_init();
+      }
+      __syncthreads();
+      if (tid == 0) {
+        mbar_arrive_expect_tx(mbar, bytes);
+        constexpr uint32_t CH = 32768;
+        for (uint32_t off = 0; off < bytes; off += CH)
+          tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off,
+                       reinterpret_cast<const unsigned char *>(gval) + off,
+                       bytes - off < CH ? bytes - off : CH, mbar);
+      }
+    } else {
+      // unaligned system block (odd nnz in CSR): plain cooperative copy
+      for (long long i = tid; i < P.sys_stride; i += NT) sval[i] = __ldg(gval + i);
+    }
+  }
+  const double *V = (PLACE == PLACE_SMEM) ? sval : gval;
+
+  // ---- pattern + right-hand side + initial guess into registers ----------
+  RowMeta<WB, R> m;
+  double x[R], r[R], rh[R], p[R], v[R], d[R];
+  const double *bsys = P.b + sys * n;
+  int dsl[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    const int row = tid + j * NT;
+    m.act[j] = row < n;
+#pragma unroll
+    for (int k = 0; k < (WB + 1) / 2; ++k) m.cpk[j][k] = 0u;
+    m.vbase[j] = 0;
+    m.vlen[j] = 0;
+    dsl[j] = 0;
+    r[j] = 0.0;
+    x[j] = 0.0;
+    if (m.act[j]) {
+#pragma unroll
+      for (int k = 0; k < WB; ++k) {
+        if (k < W) {
+          const uint32_t off = static_cast<uint32_t>(__ldg(P.ell_col + (size_t)k * n + row)) * 8u;
+          m.cpk[j][k >> 1] |= (k & 1) ? (off << 16) : off;
+        }
+      }
+      if (FMT == FMT_ELL) {
+        m.vbase[j] = row;
+        m.vlen[j] = W;
+      } else {
+        m.vbase[j] = __ldg(P.row_ptr + row);
+        m.vlen[j] = __ldg(P.row_ptr + row + 1) - m.vbase[j];
+      }
+      dsl[j] = __ldg(P.diag_slot + row);
+      r[j] = __ldg(bsys + row);  // r holds b until the initial residual is formed
+      if (P.x0) x[j] = __ldg(P.x0 + sys * n + row);
+    }
+  }
+  if (PLACE == PLACE_SMEM) {
+    if (use_tma) mbar_wait_parity(mbar, 0);
+    else __syncthreads();
+  }
+
+  // ---- a2: scalar Jacobi d = 1/a_rr (zero diagonal -> 1, DESIGN R11) -----
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    d[j] = 1.0;
+    if (m.act[j]) {
+      const int pos = (FMT == FMT_ELL) ? dsl[j] * n + m.vbase[j] : m.vbase[j] + dsl[j];
+      const double a = (PLACE == PLACE_STREAM) ? __ldg(V + pos) : V[pos];
+      d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+    }
+  }
+
+  int buf = 0;
+  // ---- a3: r = b - A x0 ; r^ = r ; ||b|| --------------------------------
+  double red3[2] = {0.0, 0.0};
+#pragma unroll
+  for (int j = 0; j < R; ++j) red3[0] += r[j] * r[j];  // b.b
+  if (P.x0) {
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (m.act[j]) sg[tid + j * NT] = x[j];
+    __syncthreads();
+    double q[R];
+    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+#pragma unroll
+    for (int j = 0; j < R; ++j) r[j] = r[j] - q[j];
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    rh[j] = r[j];
+    p[j] = 0.0;
+    v[j] = 0.0;
+    red3[1] += r[j] * r[j];
+  }
+  block_sum<2, NWARP>(red3, sred, buf, lane, warp);
+  const double bnorm = sqrt(red3[0]);
+  const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
+  double rnorm = sqrt(red3[1]);
+  double rho = red3[1];  // r^ . r with r^ = r
+
+  double *xout = P.x + sys * n;
+  if (P.stop == STOP_REL_B && bnorm == 0.0) {
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (m.act[j]) xout[tid + j * NT] = 0.0;
+    if (tid == 0) {
+      P.iters[sys] = 0;
+      P.resnorm[sys] = 0.0;
+      if (P.status) P.status[sys] = SYS_CONVERGED;
+    }
+    return;
+  }
+
+  int it = 0, st = -1, exit_kind = 0;
+  double rho_old = 1.0, alpha = 1.0, omega = 1.0;
+  double final_res = -1.0;
+  for (;;) {
+    exit_kind = 0;
+    while (it < P.maxiter) {
+      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1
+      if (bad(rho)) { st = SYS_BREAKDOWN; break; }
+      const double beta = (rho / rho_old) * (alpha / omega);  // R2
+      // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        p[j] = r[j] + beta * (p[j] - omega * v[j]);
+        if (m.act[j]) sg[tid + j * NT] = d[j] * p[j];
+      }
+      __syncthreads();
+      // a6: v = A p^
+      spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, v);
+      ++it;
+      // a7: alpha = rho / (r^ . v)
+      double rv[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
+      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
+      if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
+      alpha = rho / rv[0];                                 // R3
+      // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
+      // barrier in the reduction above separates them)
+      double s[R], ss[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        s[j] = r[j] - alpha * v[j];
+        ss[0] += s[j] * s[j];
+        if (m.act[j]) sg[tid + j * NT] = d[j] * s[j];
+      }
+      block_sum<1, NWARP>(ss, sred, buf, lane, warp);      // also publishes s^
+      if (sqrt(ss[0]) < tau) {                             // stop test 2
+#pragma unroll
+        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
+        exit_kind = 2;
+        break;
+      }
+      // a9: t = A s^
+      double t[R];
+      spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, t);
+      // a10: omega = (t.s)/(t.t); x, r updates
+      double ts[2] = {0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        ts[0] += t[j] * s[j];
+        ts[1] += t[j] * t[j];
+      }
+      block_sum<2, NWARP>(ts, sred, buf, lane, warp);
+      if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
+      omega = ts[0] / ts[1];
+      if (bad(omega)) { st = SYS_BREAKDOWN; break; }
+      double rr[2] = {0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
+        r[j] = s[j] - omega * t[j];
+        rr[0] += r[j] * r[j];
+        rr[1] += rh[j] * r[j];
+      }
+      rho_old = rho;
+      // next iteration's ||r|| and rho = r^ . r in the same single barrier
+      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
+      rnorm = sqrt(rr[0]);
+      rho = rr[1];
+    }
+    if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
+    // ---- a11: true-residual guard (DESIGN R4) -----------------------------
+    // (gather buffer is free: its last readers passed a barrier already)
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (m.act[j]) sg[tid + j * NT] = x[j];
+    __syncthreads();
+    double q[R], tr[1] = {0.0};
+    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
+      tr[0] += q[j] * q[j];
+    }
+    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
+    final_res = sqrt(tr[0]);
+    if (final_res < tau || it >= P.maxiter) break;
+    // restart from the true residual, keep counting iterations
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      r[j] = q[j];
+      rh[j] = q[j];
+      p[j] = 0.0;
+      v[j] = 0.0;
+    }
+    rho_old = alpha = omega = 1.0;
+    rnorm = final_res;
+    rho = tr[0];
+    final_res = -1.0;
+  }
+
+  if (final_res < 0.0) {
+    // final TRUE residual ||b - A x|| (always reported, R4)
+    __syncthreads();  // previous gather readers done before overwriting
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (m.act[j]) sg[tid + j * NT] = x[j];
+    __syncthreads();
+    double q[R], tr[1] = {0.0};
+    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
+      tr[0] += q[j] * q[j];
+    }
+    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
+    final_res = sqrt(tr[0]);
+  }
+  if (st != SYS_BREAKDOWN) {
+    if (P.trc) st = final_res < tau ? SYS_CONVERGED : SYS_MAXITER;
+    else st = exit_kind != 0 ? SYS_CONVERGED : SYS_MAXITER;
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j)
+    if (m.act[j]) xout[tid + j * NT] = x[j];
+  if (tid == 0) {
+    P.iters[sys] = it;
+    P.resnorm[sys] = final_res;
+    if (P.status) P.status[sys] = static_cast<int8_t>(st);
+  }
+}
+
+// -------------------------------------------------- standalone batched SpMV --
+// y_i = A_i x_i (Fig. 7).  One CTA per system; x_i is
+// staged into SMEM for the gather, values stream from global (coalesced for
+// ELL: consecutive rows of one slot are contiguous).
+template <int FMT, int NT>
+__global__ void __launch_bounds__(NT) spmv_kernel(const double *__restrict__ values,
+                                                  const double *__restrict__ xin,
+                                                  double *__restrict__ y,
+                                                  const int32_t *__restrict__ ell_col,
+                                                  const int32_t *__restrict__ row_ptr, int n,
+                                                  int W, long long sys_stride) {
+  extern __shared__ __align__(16) double sx[];
+  const long long sys = blockIdx.x;
+  const double *V = values + sys * sys_stride;
+  for (int i = threadIdx.x; i < n; i += NT) sx[i] = __ldg(xin + sys * n + i);
+  __syncthreads();
+  for (int row = threadIdx.x; row < n; row += NT) {
+    double acc = 0.0;
+    if (FMT == FMT_ELL) {
+      for (int k = 0; k < W; ++k)
+        acc = fma(__ldg(V + (size_t)k * n + row), sx[__ldg(ell_col + (size_t)k * n + row)], acc);
+    } else {
+      const int a = __ldg(row_ptr + row), e = __ldg(row_ptr + row + 1);
+      for (int q = a; q < e; ++q)
+        acc = fma(__ldg(V + q), sx[__ldg(ell_col + (size_t)(q - a) * n + row)], acc);
+    }
+    y[sys * n + row] = acc;
+  }
+}
+
+// ------------------------------------------------------- CSR -> ELL values --
+__global__ void csr_to_ell_kernel(const double *__restrict__ csr, double *__restrict__ ell,
+                                  const int32_t *__restrict__ src, long long slots, int nnz,
+                                  long long total) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const long long sys = i / slots, pos = i - sys * slots;
+    const int e = __ldg(src + pos);
+    ell[i] = e >= 0 ? __ldg(csr + sys * nnz + e) : 0.0;
+  }
+}
+
+// -------------------------------------------------- SMEM bandwidth probe --
+// Every thread streams conflict-free 16-byte shared loads; the sum is kept
+// live through a conditional store.  bytes = grid * NT * ITERS * 4 * 16.
+template <int NT>
+__global__ void __launch_bounds__(NT) smem_probe_kernel(int iters, double *sink,
+                                                        long long *cycles) {
+  __shared__ __align__(32) double4 buf[1024];
+  for (int i = threadIdx.x; i < 1024; i += NT)
+    buf[i] = make_double4(i, i + 1, i + 2, i + 3);
+  __syncthreads();
+  const long long c0 = clock64();
+  double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+  int idx = threadIdx.x;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const double4 q = buf[(idx + u * NT) & 1023];
+      a0 += q.x;
+      a1 += q.y;
+      a2 += q.z;
+      a3 += q.w;
+    }
+    idx = (idx + 32) & 1023;
+  }
+  const long long c1 = clock64();
+  const double s = a0 + a1 + a2 + a3;
+  if (s == -1.0) sink[blockIdx.x] = s;
+  if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+}
+
+}  // namespace bsolve

@@ -1,0 +1,67 @@
+"""Shared helpers of the GPU parity tests: run the C-ABI path and the oracle on
+the same seeded inputs and compare with the tolerances of BASELINE.json
+north_star:
+  * true relative residual ||b - A x|| / ||b|| <= 1e-10 (REL_B, tol 1e-10)
+  * ||x - x_direct|| / ||x_direct|| <= 1e-8 against the oracle's banded LU
+  * |iters_gpu - iters_oracle| <= 2 against the oracle's Algorithm 1
+  * identical status
+"""
+import numpy as np
+import torch
+
+import oracle as O
+import xgcgen as X
+from paper_conf_ipps_kashinksla22_b200 import Solver
+
+FWD_TOL = 1e-8
+RES_TOL = 1e-10
+ITER_TOL = 2
+
+
+def to_dev(a, dtype=torch.float64):
+    return torch.as_tensor(np.ascontiguousarray(a)).to(device="cuda", dtype=dtype)
+
+
+def gpu_solve(row_ptr, col_idx, csr_values, b, x0=None, fmt="ell", placement="auto", tol=1e-10,
+              maxiter=1000, stop="rel_b", trc=True, block_threads=0):
+    batch = csr_values.shape[0]
+    S = Solver(row_ptr, col_idx, batch, format=fmt, placement=placement, stop=stop,
+               true_residual_check=trc, block_threads=block_threads)
+    vals = (X.csr_values_to_ell(csr_values, row_ptr, col_idx) if S.format == "ell"
+            else csr_values)
+    x, it, res, st = S.run(to_dev(vals), to_dev(b), None if x0 is None else to_dev(x0), tol=tol,
+                           maxiter=maxiter)
+    torch.cuda.synchronize()
+    out = dict(x=x.cpu().numpy(), iters=it.cpu().numpy(), resnorm=res.cpu().numpy(),
+               status=st.cpu().numpy().astype(np.int32), info=S.info)
+    S.close()
+    return out
+
+
+def compare(row_ptr, col_idx, csr_values, b, g, o=None, xd=None, res_tol=RES_TOL,
+            fwd_tol=FWD_TOL, iter_tol=ITER_TOL, x0=None, tol=1e-10, check_direct=True):
+    """Compare GPU outputs g against the oracle (computed here if o is None)."""
+    if o is None:
+        o = O.batch_bicgstab(row_ptr, col_idx, csr_values, b, x0=x0, tol=tol)
+    if xd is None and check_direct:
+        xd = O.batch_banded(row_ptr, col_idx, csr_values, b)
+    batch = csr_values.shape[0]
+    bn = np.linalg.norm(b, axis=1)
+    assert np.array_equal(g["status"], o["status"]), (g["status"], o["status"])
+    di = np.abs(g["iters"].astype(int) - o["iters"].astype(int))
+    assert di.max() <= iter_tol, f"iteration mismatch max {di.max()}"
+    conv = g["status"] == 0
+    ok_b = bn > 0
+    rel = np.where(ok_b, g["resnorm"] / np.where(ok_b, bn, 1), g["resnorm"])
+    assert np.all(rel[conv] <= res_tol), rel[conv].max()
+    # independent recomputation of the TRUE residual of the GPU x (oracle SpMV)
+    for i in range(batch):
+        rt = b[i] - O.spmv(row_ptr, col_idx, csr_values[i], g["x"][i])
+        rn = np.linalg.norm(rt)
+        assert abs(rn - g["resnorm"][i]) <= 1e-12 * max(bn[i], 1e-300) + 1e-300, (i, rn, g["resnorm"][i])
+    if check_direct:
+        for i in np.nonzero(conv)[0]:
+            nrm = np.linalg.norm(xd[i])
+            if nrm > 0:
+                assert np.linalg.norm(g["x"][i] - xd[i]) / nrm <= fwd_tol, i
+    return o, xd

@@ -1,0 +1,123 @@
+"""CPU-side checks of the C-ABI boundary (no GPU needed): the library loads,
+exports every symbol include/bsolve.h declares, and rejects bad arguments and
+bad patterns with the documented codes BEFORE any CUDA call."""
+import ctypes as C
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_kashinksla22_b200 as pkg
+from paper_conf_ipps_kashinksla22_b200 import bsolve as B
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "bsolve.h")
+
+
+def header_symbols():
+    txt = open(HEADER).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(bsolve_[a-z_]+)\s*\(", txt)))
+
+
+def test_header_declares_the_boundary():
+    syms = header_symbols()
+    for s in ("bsolve_create", "bsolve_run", "bsolve_destroy", "bsolve_last_error",
+              "bsolve_run_host", "bsolve_spmv", "bsolve_csr_to_ell", "bsolve_query"):
+        assert s in syms
+
+
+def test_library_exports_every_header_symbol():
+    L = C.CDLL(pkg.LIB_PATH)
+    for s in header_symbols():
+        assert hasattr(L, s), s
+
+
+def test_library_built_for_sm100a():
+    import subprocess
+    out = subprocess.run(["cuobjdump", "-lelf", pkg.LIB_PATH], capture_output=True, text=True)
+    assert "sm_100a" in out.stdout
+
+
+def _create(n, rp, ci, **kw):
+    L = B.lib()
+    opt = B.Options()
+    L.bsolve_default_options(C.byref(opt))
+    for k, v in kw.items():
+        setattr(opt, k, v)
+    h = C.c_void_p()
+    rpa = np.ascontiguousarray(rp, np.int32)
+    cia = np.ascontiguousarray(ci, np.int32)
+    rc = L.bsolve_create(C.byref(h), n, 4, rpa.ctypes.data, cia.ctypes.data, C.byref(opt))
+    return rc, L.bsolve_last_error().decode()
+
+
+def test_pattern_errors():
+    # missing diagonal
+    rc, msg = _create(2, [0, 1, 2], [1, 0])
+    assert rc == B.ERR_PATTERN and "diagonal" in msg
+    # column out of range
+    rc, msg = _create(2, [0, 1, 2], [0, 5])
+    assert rc == B.ERR_PATTERN and "range" in msg
+    # unsorted / duplicate
+    rc, _ = _create(2, [0, 2, 3], [1, 0, 1])
+    assert rc == B.ERR_PATTERN
+    rc, _ = _create(2, [0, 2, 3], [0, 0, 1])
+    assert rc == B.ERR_PATTERN
+    # row_ptr not starting at 0 / decreasing
+    rc, _ = _create(2, [1, 2, 3], [0, 1, 1])
+    assert rc == B.ERR_PATTERN
+    rc, _ = _create(2, [0, 2, 1], [0, 1])
+    assert rc == B.ERR_PATTERN
+
+
+def test_invalid_arguments():
+    L = B.lib()
+    h = C.c_void_p()
+    rp = np.array([0, 1], np.int32)
+    ci = np.array([0], np.int32)
+    assert L.bsolve_create(None, 1, 1, rp.ctypes.data, ci.ctypes.data, None) == B.ERR_INVALID
+    assert L.bsolve_create(C.byref(h), 0, 1, rp.ctypes.data, ci.ctypes.data, None) == B.ERR_INVALID
+    assert L.bsolve_create(C.byref(h), 1, -1, rp.ctypes.data, ci.ctypes.data, None) == B.ERR_INVALID
+    assert L.bsolve_create(C.byref(h), 1, 1, None, ci.ctypes.data, None) == B.ERR_INVALID
+    rc, _ = _create(1, rp, ci, format=7)
+    assert rc == B.ERR_INVALID
+    rc, _ = _create(1, rp, ci, placement=9)
+    assert rc == B.ERR_INVALID
+    rc, _ = _create(1, rp, ci, stop=3)
+    assert rc == B.ERR_INVALID
+    rc, _ = _create(1, rp, ci, block_threads=100)
+    assert rc == B.ERR_INVALID
+    # NULL handle on every entry point
+    assert L.bsolve_run(None, None, None, None, 1e-10, 10, None, None, None, None, None) == B.ERR_INVALID
+    assert L.bsolve_run_host(None, None, None, None, 1e-10, 10, None, None, None, None) == B.ERR_INVALID
+    assert L.bsolve_spmv(None, None, None, None, 1, None) == B.ERR_INVALID
+    assert L.bsolve_csr_to_ell(None, None, None, 1, None) == B.ERR_INVALID
+    assert L.bsolve_query(None, None) == B.ERR_INVALID
+    assert L.bsolve_destroy(None) == B.OK
+
+
+def test_unsupported_row_width():
+    n = 20
+    rp = np.arange(0, n * n + 1, n, dtype=np.int32)   # dense 20x20: 20 entries per row
+    ci = np.tile(np.arange(n, dtype=np.int32), n)
+    rc, msg = _create(n, rp, ci)
+    assert rc == B.ERR_UNSUPPORTED and "entries" in msg
+
+
+def test_fails_loudly_without_library(monkeypatch):
+    monkeypatch.setattr(B, "_lib", None)
+    monkeypatch.setattr(B, "LIB_PATH", "/nonexistent/libbsolve.so")
+    with pytest.raises(ImportError):
+        B.lib()
+
+
+def test_product_never_touches_oracle():
+    pkgdir = os.path.dirname(pkg.__file__)
+    for dp, _, fs in os.walk(pkgdir):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dp, f)).read()
+                assert not re.search(r"^\s*(import|from)\s+oracle\b", txt, re.M), f
+                assert "oracle.c" not in txt and "liboracle" not in txt, f

@@ -1,0 +1,290 @@
+"""GPU parity: the C-ABI CUDA path vs the CPU oracle on the same seeded inputs.
+
+Configs follow BASELINE.json (configs[0..2], [4]) and SURVEY.md 4 / 8(c):
+every test calls libbsolve.so through the binding (no torch compute on the
+solve path) and compares element by element with oracle/ results.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import xgcgen as X
+from gpu_common import compare, gpu_solve, to_dev
+from paper_conf_ipps_kashinksla22_b200 import BsolveError, Solver
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need a CUDA device")
+    torch.cuda.init()
+
+
+# ---------------------------------------------------------- configs[0] --
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_config0_ion_electron_pair(fmt):
+    """batch = 2 (g = 0 ion, g = 1 electron), 992 rows, tol 1e-10."""
+    B = X.make_batch(0, 2)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt)
+    assert g["info"]["placement"] == 1  # SMEM staged
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+
+
+# ---------------------------------------------------------- configs[1] --
+def test_config1_zero_and_picard_warm_start():
+    """batch = 1280 (640 mesh nodes x 2 species); Picard p = 0..4 with
+    x0 = previous solution (GPU chain vs oracle chain)."""
+    N = 1280
+    xg = xo = None
+    iters_e, iters_i = [], []
+    for pcd in range(5):
+        B = X.make_batch(0, N, picard=pcd)
+        p = B.pattern
+        g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=xg)
+        o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=xo)
+        compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+        xg, xo = g["x"], o["x"]
+        iters_i.append(g["iters"][0::2].mean())
+        iters_e.append(g["iters"][1::2].mean())
+    # warm start reduces iterations (Table III trend)
+    assert iters_e[-1] < iters_e[0] and iters_i[-1] <= iters_i[0]
+
+
+# ---------------------------------------------------- formats/placements --
+@pytest.mark.parametrize("fmt,placement", [("ell", "smem"), ("ell", "stream"),
+                                           ("csr", "smem"), ("csr", "stream")])
+def test_formats_and_placements(fmt, placement):
+    B = X.make_batch(100, 64)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt, placement=placement)
+    want = 1 if placement == "smem" else 2
+    assert g["info"]["placement"] == want
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+
+
+def test_block_512_variant():
+    B = X.make_batch(0, 8)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, block_threads=512)
+    assert g["info"]["block_threads"] == 512
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+
+
+# ------------------------------------------------------ awkward patterns --
+@pytest.mark.parametrize("nx,ny", [(1, 1), (3, 3), (5, 5), (31, 31), (31, 32), (40, 25),
+                                   (64, 32)])
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_stencil_sizes(nx, ny, fmt):
+    """n in {1, 9, 25, 961, 992 transposed, 1000, 2048}: several tiles and a
+    ragged tail of rows per thread; 31 as the fast dimension."""
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 6, pattern=pat)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, fmt=fmt)
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+
+
+@pytest.mark.parametrize("n,maxrow,seed", [(50, 9, 1), (333, 9, 2), (777, 12, 3), (1000, 16, 4)])
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_random_patterns(n, maxrow, seed, fmt):
+    """Non-stencil shared patterns (<= 16 entries per row, odd nnz possible:
+    exercises the non-TMA staging fallback for CSR)."""
+    rp, ci = X.random_pattern(n, maxrow, seed=seed)
+    vals = X.random_dd_values(rp, ci, 5, seed=seed, margin=1.0)
+    b = X.random_rhs(5, n, seed=seed)
+    g = gpu_solve(rp, ci, vals, b, fmt=fmt)
+    compare(rp, ci, vals, b, g)
+
+
+# ---------------------------------------------------------- edge cases --
+def test_x0_null_equals_zero_and_alias():
+    B = X.make_batch(0, 4)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 4)
+    v = to_dev(X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
+    b = to_dev(B.b)
+    x1, i1, r1, s1 = S.run(v, b)
+    z = torch.zeros_like(b)
+    x2, i2, r2, s2 = S.run(v, b, x0=z)
+    assert torch.equal(x1, x2) and torch.equal(i1, i2) and torch.equal(r1, r2)
+    # x aliasing x0 (in/out warm start)
+    xa = torch.zeros_like(b)
+    out = (xa, torch.empty_like(i1), torch.empty_like(r1), torch.empty_like(s1))
+    S.run(v, b, x0=xa, out=out)
+    assert torch.equal(xa, x1)
+
+
+def test_maxiter_zero_b_zero_huge_tol_nonconvergence():
+    B = X.make_batch(0, 4)
+    p = B.pattern
+    b = B.b.copy()
+    b[2] = 0.0
+    x0 = np.full_like(b, 0.5)
+    # maxiter = 0: x = x0, iters 0; b = 0 row: x = 0, converged
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, b, x0=x0, maxiter=0)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, b, x0=x0, maxiter=0)
+    assert np.array_equal(g["iters"], o["iters"]) and np.array_equal(g["status"], o["status"])
+    assert np.array_equal(g["x"][[0, 1, 3]], x0[[0, 1, 3]]) and not np.any(g["x"][2])
+    np.testing.assert_allclose(g["resnorm"], o["resnorm"], rtol=1e-12)
+    # huge tolerance: converged at iteration 0
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, tol=10.0)
+    assert np.all(g["iters"] == 0) and np.all(g["status"] == 0)
+    # forced non-convergence
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3)
+    assert np.all(g["iters"] == 3) and np.array_equal(g["status"], o["status"])
+    assert np.all(g["status"] == 1)
+
+
+def test_diagonal_exact_one_iteration():
+    """P3 on the GPU: off-diagonals zero -> exactly 1 iteration (stop test 2)."""
+    pat = X.stencil_pattern()
+    v = np.zeros((3, pat.nnz))
+    for i in range(pat.n):
+        for e in range(pat.row_ptr[i], pat.row_ptr[i + 1]):
+            if pat.col_idx[e] == i:
+                v[:, e] = [1.0 + i, 2.0 + 0.5 * i, -3.0 - i]
+    b = X.random_rhs(3, pat.n)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, v, b)
+    assert np.all(g["iters"] == 1) and np.all(g["status"] == 0)
+    dg = np.array([[1.0 + i, 2.0 + 0.5 * i, -3.0 - i] for i in range(pat.n)]).T
+    np.testing.assert_allclose(g["x"], b / dg, rtol=1e-15)
+
+
+def test_breakdown():
+    rp = np.array([0, 2, 4], np.int32)
+    ci = np.array([0, 1, 0, 1], np.int32)
+    v = np.array([[0.0, 1.0, 1.0, 0.0]])
+    g = gpu_solve(rp, ci, v, np.array([[1.0, 0.0]]))
+    assert g["status"][0] == 2 and g["iters"][0] == 1 and not np.any(g["x"])
+
+
+def test_abs_stop_mode():
+    B = X.make_batch(0, 8)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, stop="abs")
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, stop=O.STOP_ABS)
+    assert np.abs(g["iters"] - o["iters"]).max() <= 2
+    assert np.all(g["resnorm"] < 1e-10)
+
+
+def test_no_true_residual_check():
+    B = X.make_batch(0, 8)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, trc=False)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, true_res_check=False)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+
+
+def test_ill_conditioned_guard():
+    """configs[4] flavour: kappa ~ 1e5 electrons trigger the true-residual guard."""
+    ill = X.Species(X.ELECTRON_K, cross=0.0, margin=1e-3)
+    B = X.make_batch(1, 8, electron=ill)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, iter_tol=10)
+
+
+# ------------------------------------------------- invariants on the GPU --
+def test_power_of_two_scaling_bitwise_gpu():
+    """P5 holds for the kernel independently of its reduction order."""
+    B = X.make_batch(0, 6)
+    p = B.pattern
+    g1 = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    g2 = gpu_solve(p.row_ptr, p.col_idx, 8.0 * B.values, 8.0 * B.b)
+    assert np.array_equal(g1["x"], g2["x"]) and np.array_equal(g1["iters"], g2["iters"])
+
+
+def test_deterministic_and_partition_independent():
+    """Per-system outputs are bitwise identical across runs and batch slicing
+    (the multi-GPU bitwise claim of SURVEY 8(e) rests on this)."""
+    B = X.make_batch(0, 64)
+    p = B.pattern
+    g1 = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    g2 = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    g3 = gpu_solve(p.row_ptr, p.col_idx, B.values[40:], B.b[40:])
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(g1[k], g2[k])
+        assert np.array_equal(g1[k][40:], g3[k])
+
+
+def test_symmetric_permutation_gpu():
+    import scipy.sparse as sp
+    B = X.make_batch(0, 2)
+    p = B.pattern
+    perm = np.random.default_rng(3).permutation(p.n)
+    vals, rp = [], None
+    for j in range(2):
+        A = sp.csr_matrix((B.values[j], p.col_idx, p.row_ptr), shape=(p.n, p.n))
+        Ap = A[perm][:, perm].tocsr()
+        Ap.sort_indices()
+        rp, ci = Ap.indptr.astype(np.int32), Ap.indices.astype(np.int32)
+        vals.append(Ap.data)
+    vals = np.array(vals)
+    bp = B.b[:, perm]
+    g = gpu_solve(rp, ci, vals, bp)
+    compare(rp, ci, vals, bp, g)
+
+
+# ------------------------------------------------------- other entries --
+def test_csr_to_ell_bit_exact():
+    B = X.make_batch(0, 5)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 5)
+    ell = S.csr_to_ell(to_dev(B.values))
+    torch.cuda.synchronize()
+    assert np.array_equal(ell.cpu().numpy(), X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
+    assert np.array_equal(S.ell_cols(), X.ell_layout(p.row_ptr, p.col_idx)[0])
+
+
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_spmv_vs_oracle(fmt):
+    B = X.make_batch(0, 7)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 7, format=fmt)
+    vals = X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx) if fmt == "ell" else B.values
+    xs = X.random_rhs(7, p.n, seed=9)
+    y = S.spmv(to_dev(vals), to_dev(xs)).cpu().numpy()
+    for i in range(7):
+        ref = O.spmv(p.row_ptr, p.col_idx, B.values[i], xs[i])
+        np.testing.assert_allclose(y[i], ref, rtol=1e-13, atol=1e-13 * np.abs(ref).max())
+
+
+def test_run_host_matches_run():
+    B = X.make_batch(0, 300)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 300)
+    ell = X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx)
+    xh, ih, rh, sh = S.run_host(ell, B.b)
+    xd, idd, rd, sd = S.run(to_dev(ell), to_dev(B.b))
+    torch.cuda.synchronize()
+    assert np.array_equal(xh, xd.cpu().numpy()) and np.array_equal(ih, idd.cpu().numpy())
+    assert np.array_equal(rh, rd.cpu().numpy()) and np.array_equal(sh, sd.cpu().numpy())
+
+
+def test_run_arg_errors_on_gpu():
+    B = X.make_batch(0, 2)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 2)
+    v = to_dev(X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
+    b = to_dev(B.b)
+    with pytest.raises(BsolveError) as e:
+        S.run(v, b, tol=-1.0)
+    assert e.value.code == -1
+    with pytest.raises(BsolveError) as e:
+        S.run(v, b, maxiter=-5)
+    assert e.value.code == -1
+    with pytest.raises(BsolveError):
+        Solver(p.row_ptr, p.col_idx, 2, placement="smem",
+               format="ell").run(v, b, tol=float("nan"))
+
+
+def test_forced_smem_too_large_unsupported():
+    pat = X.stencil_pattern(64, 63)   # n = 4032: 290 KB of ELL values
+    with pytest.raises(BsolveError) as e:
+        Solver(pat.row_ptr, pat.col_idx, 1, placement="smem")
+    assert e.value.code in (-3,)
