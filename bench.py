@@ -72,27 +72,36 @@ class ClockSampler:
         self._stop = threading.Event()
         self._t = None
 
-    def _run(self):
-        while not self._stop.is_set():
-            try:
-                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True,
-                                     text=True, timeout=5).stdout.strip()
-                if out:
-                    self.rows.append([c.strip() for c in out.split(",")])
-            except Exception:
-                pass
-            self._stop.wait(0.2)
-
     def __enter__(self):
-        self._t = threading.Thread(target=self._run, daemon=True)
+        # streaming mode: one nvidia-smi process printing every 20 ms
+        try:
+            self._p = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "20"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self._p = None
+            return self
+        def reader():
+            for line in self._p.stdout:
+                line = line.strip()
+                if line:
+                    self.rows.append([c.strip() for c in line.split(",")])
+        self._t = threading.Thread(target=reader, daemon=True)
         self._t.start()
+        time.sleep(0.3)  # let the sampler start before the timed region
         return self
 
     def __exit__(self, *a):
-        self._stop.set()
+        if getattr(self, "_p", None):
+            time.sleep(0.05)
+            self._p.terminate()
+            try:
+                self._p.wait(timeout=5)
+            except Exception:
+                self._p.kill()
         if self._t:
-            self._t.join(timeout=10)
+            self._t.join(timeout=5)
 
     def summary(self):
         if not self.rows:
@@ -128,7 +137,8 @@ def make_inputs(g0, count, args, pinned):
     vals = torch.empty((count, per), dtype=torch.float64, pin_memory=pinned)
     b = torch.empty((count, pat.n), dtype=torch.float64, pin_memory=pinned)
     vn, bn = vals.numpy(), b.numpy()
-    _, src = X.ell_layout(pat.row_ptr, pat.col_idx)
+    from paper_conf_ipps_kashinksla22_b200 import ell_layout
+    _, _, src = ell_layout(pat.row_ptr, pat.col_idx)   # the library's ELL slot map
     ok = src >= 0
     CH = 8192
     for c0 in range(0, count, CH):

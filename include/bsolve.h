@@ -58,10 +58,13 @@ enum {
   BSOLVE_FMT_CSR = 1,  /* values[i*nnz + e]: entry e in the CSR order of
                           (row_ptr, col_idx)  (BatchCsr)     */
   BSOLVE_FMT_ELL = 2   /* values[i*W*n + k*n + r]: slot k of row r, column-
-                          major (BatchEll).  Slot k
-                          of row r is the k-th CSR entry of row r; slots past
-                          the row's length are padding and MUST hold 0.0.
-                          W = max entries per row (bsolve_info.ell_width).    */
+                          major (BatchEll).  W =
+                          max entries per row (bsolve_info.ell_width).  WHICH
+                          entry of row r sits in slot k is chosen by the
+                          handle (bank-conflict-free gathers, DESIGN.md
+                          "ELL slot map") and published by bsolve_ell_map;
+                          bsolve_csr_to_ell converts CSR-ordered values.
+                          Padding slots MUST hold 0.0.                        */
 };
 
 /* Where the matrix values live while a system iterates (PAPER.md:708-721,
@@ -172,9 +175,19 @@ int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, double *ell_val
 /* Describe the plan (see bsolve_info). */
 int bsolve_query(bsolve_handle h, bsolve_info *info);
 
-/* Copy the ELL column indices (W * n int32, column-major, padding slots hold
- * their own row) to HOST memory `out`. */
-int bsolve_ell_cols(bsolve_handle h, int32_t *out);
+/* Publish the handle's ELL slot map to HOST memory (either pointer may be
+ * NULL, not both):
+ *   cols[k*n + r]  column read by slot k of row r (W*n int32);
+ *   src[k*n + r]   index e of the CSR entry (row_ptr/col_idx order) stored in
+ *                  that slot, or -1 for a padding slot (value must be 0.0).
+ * Every CSR entry appears in exactly one slot of its row. */
+int bsolve_ell_map(bsolve_handle h, int32_t *cols, int32_t *src);
+
+/* Host-only: the ELL slot map the library uses for a pattern, without a
+ * handle or a GPU (same validation as bsolve_create).  *width receives W;
+ * cols/src (W*n int32 each, may be NULL) as in bsolve_ell_map. */
+int bsolve_ell_layout(int n, const int32_t *row_ptr, const int32_t *col_idx, int32_t *width,
+                      int32_t *cols, int32_t *src);
 
 /* Release the handle and its device memory.  NULL-safe; returns BSOLVE_OK. */
 int bsolve_destroy(bsolve_handle h);

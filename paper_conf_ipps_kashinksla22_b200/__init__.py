@@ -4,7 +4,7 @@ The product path is libbsolve.so (C ABI, include/bsolve.h) + this thin
 binding.  It never imports the CPU oracle (oracle/) and has no CPU fallback.
 """
 from .bsolve import (  # noqa: F401
-    BsolveError, Solver, lib, probe_smem_bandwidth, LIB_PATH,
+    BsolveError, Solver, lib, probe_smem_bandwidth, LIB_PATH, ell_layout, ell_values,
     SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN,
 )
 

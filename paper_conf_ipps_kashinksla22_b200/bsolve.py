@@ -69,14 +69,16 @@ def lib():
             L.bsolve_spmv.argtypes = [_P, _P, _P, _P, C.c_int, _P]
             L.bsolve_csr_to_ell.argtypes = [_P, _P, _P, C.c_int, _P]
             L.bsolve_query.argtypes = [_P, C.POINTER(Info)]
-            L.bsolve_ell_cols.argtypes = [_P, _P]
+            L.bsolve_ell_map.argtypes = [_P, _P, _P]
+            L.bsolve_ell_layout.argtypes = [C.c_int, _P, _P, C.POINTER(C.c_int32), _P, _P]
             L.bsolve_destroy.argtypes = [_P]
             L.bsolve_last_error.argtypes = []
             L.bsolve_last_error.restype = C.c_char_p
             L.bsolve_probe_smem_bandwidth.argtypes = [C.c_int, C.POINTER(C.c_double),
                                                       C.POINTER(C.c_double)]
             for f in ("bsolve_create", "bsolve_run", "bsolve_run_host", "bsolve_spmv",
-                      "bsolve_csr_to_ell", "bsolve_query", "bsolve_ell_cols", "bsolve_destroy",
+                      "bsolve_csr_to_ell", "bsolve_query", "bsolve_ell_map", "bsolve_destroy",
+                      "bsolve_ell_layout",
                       "bsolve_probe_smem_bandwidth"):
                 getattr(L, f).restype = C.c_int
             _lib = L
@@ -92,6 +94,29 @@ def _stream_ptr(stream):
     import torch
     s = torch.cuda.current_stream() if stream is None else stream
     return s.cuda_stream
+
+
+def ell_layout(row_ptr, col_idx):
+    """Host-only ELL slot map of a pattern: (W, cols[W*n], src[W*n])."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
+    ci = np.ascontiguousarray(col_idx, dtype=np.int32)
+    n = rp.size - 1
+    w = C.c_int32()
+    check(lib().bsolve_ell_layout(n, rp.ctypes.data, ci.ctypes.data, C.byref(w), None, None))
+    cols = np.empty(w.value * n, np.int32)
+    src = np.empty(w.value * n, np.int32)
+    check(lib().bsolve_ell_layout(n, rp.ctypes.data, ci.ctypes.data, C.byref(w),
+                                  cols.ctypes.data, src.ctypes.data))
+    return w.value, cols, src
+
+
+def ell_values(csr_values, src):
+    """[batch, nnz] CSR-ordered values -> [batch, W*n] ELL values given `src`."""
+    v = np.asarray(csr_values, dtype=np.float64)
+    out = np.zeros((v.shape[0], src.size), np.float64)
+    ok = src >= 0
+    out[:, ok] = v[:, src[ok]]
+    return out
 
 
 def probe_smem_bandwidth(device: int = -1):
@@ -140,10 +165,17 @@ class Solver:
         check(lib().bsolve_query(self._h, C.byref(inf)))
         return inf.as_dict()
 
-    def ell_cols(self) -> np.ndarray:
-        out = np.empty(self.width * self.n, np.int32)
-        check(lib().bsolve_ell_cols(self._h, out.ctypes.data))
-        return out
+    def ell_map(self):
+        """(cols, src): the handle's ELL slot map, each [W*n] int32 column-major."""
+        cols = np.empty(self.width * self.n, np.int32)
+        src = np.empty(self.width * self.n, np.int32)
+        check(lib().bsolve_ell_map(self._h, cols.ctypes.data, src.ctypes.data))
+        return cols, src
+
+    def ell_values(self, csr_values) -> np.ndarray:
+        """Host-side re-layout of CSR-ordered values [batch, nnz] into this
+        handle's ELL layout [batch, W*n] (pure permutation, zero padding)."""
+        return ell_values(csr_values, self.ell_map()[1])
 
     def close(self):
         if getattr(self, "_h", None):

@@ -48,24 +48,31 @@ static int fail(int code, const char *fmt, ...) {
 typedef void (*solve_fn)(const SolveParams);
 
 struct Variant {
-  int fmt, place, wb, r, nt;
+  int fmt, place, wb;
+  bool exact;
+  int r, nt;
   solve_fn fn;
 };
 
-#define V_(F, PL, WB, R, NT, MB) \
-  {F, PL, WB, R, NT, (solve_fn)bicgstab_kernel<F, PL, WB, R, NT, MB>}
-#define V_FP(WB, R, NT, MB)                                                     \
-  V_(FMT_ELL, PLACE_SMEM, WB, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, R, NT, MB), \
-      V_(FMT_CSR, PLACE_SMEM, WB, R, NT, MB), V_(FMT_CSR, PLACE_STREAM, WB, R, NT, MB)
+#define V_(F, PL, WB, EX, R, NT, MB) \
+  {F, PL, WB, EX, R, NT, (solve_fn)bicgstab_kernel<F, PL, WB, EX, R, NT, MB>}
+#define V_FP(WB, EX, R, NT, MB)                                                         \
+  V_(FMT_ELL, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, EX, R, NT, MB), \
+      V_(FMT_CSR, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_CSR, PLACE_STREAM, WB, EX, R, NT, MB)
 
+// W = 9 (the paper's 9-point stencil) gets exact-width variants; any other
+// width <= 16 runs the generic WB = 16 variants with a per-slot test.
 static const Variant kVariants[] = {
-    V_FP(9, 1, 256, 2),  V_FP(9, 2, 256, 2),  V_FP(9, 4, 256, 2),  V_FP(9, 4, 512, 1),
-    V_FP(16, 1, 256, 2), V_FP(16, 2, 256, 2), V_FP(16, 4, 256, 2), V_FP(16, 4, 512, 1),
+    V_FP(9, true, 1, 256, 2),   V_FP(9, true, 2, 256, 2),   V_FP(9, true, 4, 256, 2),
+    V_FP(9, true, 4, 512, 1),   V_FP(16, false, 1, 256, 2), V_FP(16, false, 2, 256, 2),
+    V_FP(16, false, 4, 256, 2), V_FP(16, false, 4, 512, 1),
 };
 
-static const Variant *find_variant(int fmt, int place, int wb, int r, int nt) {
+static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt) {
   for (const Variant &v : kVariants)
-    if (v.fmt == fmt && v.place == place && v.wb == wb && v.r == r && v.nt == nt) return &v;
+    if (v.fmt == fmt && v.place == place && v.wb == wb && v.exact == exact && v.r == r &&
+        v.nt == nt)
+      return &v;
   return nullptr;
 }
 
@@ -78,7 +85,7 @@ struct bsolve_plan {
   long long sys_stride = 0;
   const Variant *var = nullptr;
   std::vector<int32_t> h_ell_col;  // [W][n]
-  std::vector<int32_t> h_csr2ell;  // [W][n] -> CSR entry or -1
+  std::vector<int32_t> h_csr2ell;  // [W][n] -> CSR entry held by the slot, -1 = padding
   int32_t *d_ell_col = nullptr, *d_row_ptr = nullptr, *d_diag = nullptr, *d_src = nullptr;
   // bsolve_run_host pipeline (lazily allocated)
   static constexpr int kSlots = 3;
@@ -146,6 +153,105 @@ static int validate_pattern(int n, const int32_t *rp, const int32_t *ci, std::ve
   return BSOLVE_OK;
 }
 
+// ELL slot assignment (create time).  The paper's BatchEll stores each row's
+// entries padded to a uniform width, column-major (PAPER.md:491-499,
+// 522-524); it leaves the slot order free.  We choose it for conflict-free
+// shared-memory gathers on B200: slot k is tied to the k-th most frequent
+// column offset d_k = col - row of the pattern (for the 9-point stencil the
+// 9 stencil offsets), so the 32 lanes of a warp (32 consecutive rows) read
+// gather addresses row + d_k that are consecutive -> 2 wavefronts per
+// LDS.64 instead of 4 at grid-boundary rows.  Entries whose offset is not a
+// template offset take the remaining free slots; padding slots get a column
+// congruent to row + d_k modulo 16 doubles (same bank pair) and value 0.
+static void build_ell_map(int n, const int32_t *rp, const int32_t *ci, int W,
+                          std::vector<int32_t> &ell_col, std::vector<int32_t> &src,
+                          std::vector<int32_t> &ell_diag) {
+  std::vector<std::pair<int, int>> hist;  // (offset, count)
+  {
+    std::vector<int> offs;
+    offs.reserve(rp[n]);
+    for (int i = 0; i < n; ++i)
+      for (int e = rp[i]; e < rp[i + 1]; ++e) offs.push_back(ci[e] - i);
+    std::sort(offs.begin(), offs.end());
+    for (size_t a = 0; a < offs.size();) {
+      size_t b = a;
+      while (b < offs.size() && offs[b] == offs[a]) ++b;
+      hist.push_back({offs[a], (int)(b - a)});
+      a = b;
+    }
+  }
+  std::stable_sort(hist.begin(), hist.end(), [](const std::pair<int, int> &x,
+                                                const std::pair<int, int> &y) {
+    if (x.second != y.second) return x.second > y.second;
+    if (std::abs(x.first) != std::abs(y.first)) return std::abs(x.first) < std::abs(y.first);
+    return x.first < y.first;
+  });
+  std::vector<int> tmpl;
+  for (int k = 0; k < W && k < (int)hist.size(); ++k) tmpl.push_back(hist[k].first);
+  std::sort(tmpl.begin(), tmpl.end());
+  while ((int)tmpl.size() < W) tmpl.push_back(0);
+  ell_col.assign((size_t)W * n, 0);
+  src.assign((size_t)W * n, -1);
+  ell_diag.assign(n, 0);
+  std::vector<int> slot_of(W);
+  for (int i = 0; i < n; ++i) {
+    std::vector<char> used(W, 0);
+    std::vector<int> rest;
+    for (int e = rp[i]; e < rp[i + 1]; ++e) {
+      const int o = ci[e] - i;
+      int k = (int)(std::lower_bound(tmpl.begin(), tmpl.end(), o) - tmpl.begin());
+      bool placed = false;
+      for (; k < W && tmpl[k] == o; ++k)
+        if (!used[k]) {
+          used[k] = 1;
+          src[(size_t)k * n + i] = e;
+          ell_col[(size_t)k * n + i] = ci[e];
+          placed = true;
+          break;
+        }
+      if (!placed) rest.push_back(e);
+    }
+    size_t r = 0;
+    for (int k = 0; k < W; ++k) {
+      if (used[k]) continue;
+      if (r < rest.size()) {
+        const int e = rest[r++];
+        used[k] = 1;
+        src[(size_t)k * n + i] = e;
+        ell_col[(size_t)k * n + i] = ci[e];
+      } else {
+        long long t = (long long)i + tmpl[k];
+        long long c = t;
+        if (t < 0) c = ((t % 16) + 16) % 16;
+        else if (t >= n) c = t - 16 * ((t - (n - 1) + 15) / 16);
+        if (c < 0 || c >= n) c = i;
+        ell_col[(size_t)k * n + i] = (int32_t)c;
+      }
+    }
+    for (int k = 0; k < W; ++k)
+      if (src[(size_t)k * n + i] >= 0 && ell_col[(size_t)k * n + i] == i) ell_diag[i] = k;
+  }
+}
+
+extern "C" int bsolve_ell_layout(int n, const int32_t *row_ptr, const int32_t *col_idx,
+                                 int32_t *width, int32_t *cols, int32_t *src) {
+  g_err.clear();
+  if (n <= 0) return fail(BSOLVE_ERR_INVALID, "n = %d must be >= 1", n);
+  if (!row_ptr || !col_idx || !width) return fail(BSOLVE_ERR_INVALID, "NULL argument");
+  std::vector<int32_t> diag;
+  int W = 0;
+  int rc = validate_pattern(n, row_ptr, col_idx, diag, W);
+  if (rc) return rc;
+  *width = W;
+  if (cols || src) {
+    std::vector<int32_t> c, s, d;
+    build_ell_map(n, row_ptr, col_idx, W, c, s, d);
+    if (cols) std::memcpy(cols, c.data(), sizeof(int32_t) * c.size());
+    if (src) std::memcpy(src, s.data(), sizeof(int32_t) * s.size());
+  }
+  return BSOLVE_OK;
+}
+
 extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t *row_ptr,
                              const int32_t *col_idx, const bsolve_options *opt_in) {
   g_err.clear();
@@ -183,7 +289,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->nnz = nnz;
   h->batch = batch;
   h->W = W;
-  h->wb = W <= 9 ? 9 : 16;
+  h->wb = W == 9 ? 9 : 16;
   h->fmt = opt.format == BSOLVE_FMT_CSR ? FMT_CSR : FMT_ELL;
   h->stop = opt.stop;
   h->trc = opt.true_residual_check ? 1 : 0;
@@ -195,16 +301,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->kl = std::max(h->kl, i - col_idx[e]);
       h->ku = std::max(h->ku, col_idx[e] - i);
     }
-  // ELL columns: slot k of row i = k-th CSR entry; padding -> own row
-  h->h_ell_col.assign((size_t)W * n, 0);
-  h->h_csr2ell.assign((size_t)W * n, -1);
-  for (int i = 0; i < n; ++i)
-    for (int k = 0; k < W; ++k) {
-      const int e = row_ptr[i] + k;
-      const bool real = e < row_ptr[i + 1];
-      h->h_ell_col[(size_t)k * n + i] = real ? col_idx[e] : i;
-      h->h_csr2ell[(size_t)k * n + i] = real ? e : -1;
-    }
+  // ELL slot map (conflict-free gathers, see build_ell_map)
+  std::vector<int32_t> ell_diag;
+  build_ell_map(n, row_ptr, col_idx, W, h->h_ell_col, h->h_csr2ell, ell_diag);
+  if (h->fmt == FMT_ELL) diag = ell_diag;  // kernel needs the diagonal's slot in its format
 
   // ---- device + variant choice -------------------------------------------
   int dev = opt.device;
@@ -259,7 +359,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                           smem_need, smem_optin));
   h->place = place;
   h->smem_bytes = (int)(place == PLACE_SMEM ? smem_need : tail);
-  h->var = find_variant(h->fmt, place, h->wb, r, nt);
+  h->var = find_variant(h->fmt, place, h->wb, h->wb == 9, r, nt);
   if (!h->var)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
                           h->fmt, place, h->wb, r, nt));
@@ -321,9 +421,10 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   return BSOLVE_OK;
 }
 
-extern "C" int bsolve_ell_cols(bsolve_handle h, int32_t *out) {
-  if (!h || !out) return fail(BSOLVE_ERR_INVALID, "NULL handle or out");
-  std::memcpy(out, h->h_ell_col.data(), sizeof(int32_t) * h->h_ell_col.size());
+extern "C" int bsolve_ell_map(bsolve_handle h, int32_t *cols, int32_t *src) {
+  if (!h || (!cols && !src)) return fail(BSOLVE_ERR_INVALID, "NULL handle or outputs");
+  if (cols) std::memcpy(cols, h->h_ell_col.data(), sizeof(int32_t) * h->h_ell_col.size());
+  if (src) std::memcpy(src, h->h_csr2ell.data(), sizeof(int32_t) * h->h_csr2ell.size());
   return BSOLVE_OK;
 }
 

@@ -90,13 +90,21 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity)
 
 __device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
 
-// Block-wide sum of K doubles: warp butterfly (all lanes end bitwise equal),
-// lane 0 publishes, ONE barrier, then every thread sums the NWARP partials
-// in warp order.  `buf` alternates between two scratch halves so that the
-// next reduction never overwrites partials a slow thread is still reading.
+// Block-wide sum of K doubles with ONE barrier:
+//  1. xor-butterfly inside each warp (after it every lane holds the same
+//     bits: at each step lanes L and L^o add the same two operands, and fp
+//     addition is commutative);
+//  2. lane 0 of each warp publishes its partial, __syncthreads();
+//  3. lane w < NWARP of EVERY warp loads partial w (one LDS wavefront per
+//     value per warp instead of NWARP broadcast loads), then a butterfly over
+//     the NWARP lanes and a broadcast from lane 0 give every thread the same
+//     bits.  Fixed order => deterministic, independent of batch slicing.
+// `buf` alternates between two scratch halves so that the next reduction
+// never overwrites partials a slow warp is still reading.
 template <int K, int NWARP>
 __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf, int lane,
                                           int warp) {
+  static_assert((NWARP & (NWARP - 1)) == 0 && NWARP <= 32, "NWARP must be a power of two");
 #pragma unroll
   for (int k = 0; k < K; ++k) {
 #pragma unroll
@@ -105,15 +113,15 @@ __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf
   double *S = sred + buf * (NWARP * 4);
   if (lane == 0) {
 #pragma unroll
-    for (int k = 0; k < K; ++k) S[warp * 4 + k] = v[k];
+    for (int k = 0; k < K; ++k) S[k * NWARP + warp] = v[k];
   }
   __syncthreads();
 #pragma unroll
   for (int k = 0; k < K; ++k) {
-    double a = 0.0;
+    double a = lane < NWARP ? S[k * NWARP + lane] : 0.0;
 #pragma unroll
-    for (int w = 0; w < NWARP; ++w) a += S[w * 4 + k];
-    v[k] = a;
+    for (int o = NWARP / 2; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+    v[k] = __shfl_sync(0xffffffffu, a, 0);
   }
   buf ^= 1;
 }
@@ -127,10 +135,8 @@ struct RowMeta {
   bool act[R];                   // row < n
 };
 
-// y = A * g for this thread's rows; g is the shared gather buffer sg;
-// values come from V (shared or global).
-// Extract the 16-bit field at bit `pos` of `pk`.  volatile: keeps the unpack
-// inside the SpMV loop instead of letting the compiler hoist 2x as many
+// Extract the 16-bit field at bit `POS` of `pk`.  volatile keeps the unpack
+// inside the SpMV loop instead of letting the compiler hoist twice as many
 // unpacked offsets into registers (which spills at R = 4).
 template <int POS>
 __device__ __forceinline__ uint32_t field16(uint32_t pk) {
@@ -139,35 +145,41 @@ __device__ __forceinline__ uint32_t field16(uint32_t pk) {
   return v;
 }
 
-template <int FMT, int PLACE, int WB, int R, int NT>
+// y = A * g for this thread's rows (one thread per row,
+// W sequential slots, no intra-row reduction).  g is the shared gather
+// buffer sg; values come from V (shared or global).  EXACT: W == WB known at
+// compile time (no per-slot test).  A warp whose rows j are all >= n skips
+// block j with a warp-uniform branch; lanes of a partial warp run on a
+// clamped row and zero their result.
+template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT>
 __device__ __forceinline__ void spmv_rows(const double *__restrict__ V, const double *sg, int n,
                                           int W, const RowMeta<WB, R> &m, double (&y)[R]) {
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
-  const double *Vt = V + threadIdx.x;  // ELL: slot k of row tid + j*NT at Vt[k*n + j*NT]
+  const int wrow0 = threadIdx.x & ~31;
 #pragma unroll
   for (int j = 0; j < R; ++j) {
     double acc = 0.0;
-    if (m.act[j]) {
+    if (wrow0 + j * NT < n) {
 #pragma unroll
       for (int k = 0; k < WB; ++k) {
-        if (k < W) {
+        if (EXACT || k < W) {
           const uint32_t off = (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
           const double g = *reinterpret_cast<const double *>(gb + off);
           if (FMT == FMT_ELL) {
-            const double a = (PLACE == PLACE_STREAM) ? __ldg(Vt + (size_t)k * n + j * NT)
-                                                     : Vt[k * n + j * NT];
+            const double *a_p = V + m.vbase[j] + k * n;
+            const double a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
             acc = fma(a, g, acc);
           } else {
             if (k < m.vlen[j]) {
-              const double a = (PLACE == PLACE_STREAM) ? __ldg(V + m.vbase[j] + k)
-                                                       : V[m.vbase[j] + k];
+              const double *a_p = V + m.vbase[j] + k;
+              const double a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
               acc = fma(a, g, acc);
             }
           }
         }
       }
     }
-    y[j] = acc;
+    y[j] = m.act[j] ? acc : 0.0;
   }
 }
 
@@ -175,7 +187,7 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V, const do
 // Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
 //   [values: smem_vals doubles (PLACE_SMEM only)] [gather: n_pad doubles]
 //   [reduction scratch: 2*NWARP*4 doubles] [mbarrier: 8 B]
-template <int FMT, int PLACE, int WB, int R, int NT, int MINB>
+template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB>
 __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -226,7 +238,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     m.act[j] = row < n;
 #pragma unroll
     for (int k = 0; k < (WB + 1) / 2; ++k) m.cpk[j][k] = 0u;
-    m.vbase[j] = 0;
+    m.vbase[j] = (FMT == FMT_ELL) ? (row < n ? row : n - 1) : 0;  // clamped for idle lanes
     m.vlen[j] = 0;
     dsl[j] = 0;
     r[j] = 0.0;
@@ -278,7 +290,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R];
-    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) r[j] = r[j] - q[j];
   }
@@ -325,7 +337,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       }
       __syncthreads();
       // a6: v = A p^
-      spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, v);
+      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, v);
       ++it;
       // a7: alpha = rho / (r^ . v)
       double rv[1] = {0.0};
@@ -352,7 +364,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       }
       // a9: t = A s^
       double t[R];
-      spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, t);
+      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, t);
       // a10: omega = (t.s)/(t.t); x, r updates
       double ts[2] = {0.0, 0.0};
 #pragma unroll
@@ -386,7 +398,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
       q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
@@ -417,7 +429,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
       q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;

@@ -27,7 +27,7 @@ def gpu_solve(row_ptr, col_idx, csr_values, b, x0=None, fmt="ell", placement="au
     batch = csr_values.shape[0]
     S = Solver(row_ptr, col_idx, batch, format=fmt, placement=placement, stop=stop,
                true_residual_check=trc, block_threads=block_threads)
-    vals = (X.csr_values_to_ell(csr_values, row_ptr, col_idx) if S.format == "ell"
+    vals = (S.ell_values(csr_values) if S.format == "ell"
             else csr_values)
     x, it, res, st = S.run(to_dev(vals), to_dev(b), None if x0 is None else to_dev(x0), tol=tol,
                            maxiter=maxiter)

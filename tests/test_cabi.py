@@ -121,3 +121,65 @@ def test_product_never_touches_oracle():
                 txt = open(os.path.join(dp, f)).read()
                 assert not re.search(r"^\s*(import|from)\s+oracle\b", txt, re.M), f
                 assert "oracle.c" not in txt and "liboracle" not in txt, f
+
+
+# ------------------------------------------------------------ ELL slot map --
+def _check_map(rp, ci, W, cols, src):
+    n = len(rp) - 1
+    seen = np.zeros(rp[-1], np.int32)
+    for k in range(W):
+        for i in range(n):
+            e = src[k * n + i]
+            if e >= 0:
+                assert rp[i] <= e < rp[i + 1]          # entry belongs to row i
+                assert cols[k * n + i] == ci[e]
+                seen[e] += 1
+            else:
+                assert 0 <= cols[k * n + i] < n         # padding reads a valid column
+    assert np.all(seen == 1)                            # every CSR entry exactly once
+
+
+def test_ell_map_is_a_valid_permutation():
+    import xgcgen as X
+    for (nx, ny) in [(32, 31), (31, 32), (5, 5), (1, 1), (64, 63)]:
+        pat = X.stencil_pattern(nx, ny)
+        W, cols, src = pkg.ell_layout(pat.row_ptr, pat.col_idx)
+        assert W == pat.max_row_nnz
+        _check_map(pat.row_ptr, pat.col_idx, W, cols, src)
+        assert int(np.sum(src < 0)) == W * pat.n - pat.nnz  # 374 pads at 32x31
+    for seed in range(3):
+        rp, ci = X.random_pattern(300, 12, seed=seed)
+        W, cols, src = pkg.ell_layout(rp, ci)
+        _check_map(rp, ci, W, cols, src)
+
+
+def _excess_wavefronts(cols, n, W):
+    """Bank-conflict excess of the gather LDS.64 of each (warp, slot): lanes
+    of a half-warp hitting the same 8-byte bank pair at different addresses."""
+    excess = 0
+    for k in range(W):
+        for w0 in range(0, n, 32):
+            for h0 in (w0, w0 + 16):
+                addr = [cols[k * n + i] for i in range(h0, min(h0 + 16, n))]
+                banks = {}
+                for a in set(addr):
+                    banks.setdefault(a % 16, set()).add(a)
+                excess += max(len(v) for v in banks.values()) - 1 if banks else 0
+    return excess
+
+
+def test_ell_map_conflict_free_gathers_on_stencil():
+    """the library's slot assignment makes the 9-point
+    gathers conflict-free, where the CSR-order slot assignment is not."""
+    import xgcgen as X
+    pat = X.stencil_pattern(32, 31)
+    W, cols, src = pkg.ell_layout(pat.row_ptr, pat.col_idx)
+    csr_cols, _ = X.ell_layout(pat.row_ptr, pat.col_idx)
+    assert _excess_wavefronts(cols, pat.n, W) == 0
+    assert _excess_wavefronts(csr_cols, pat.n, W) > 0
+
+
+def test_ell_layout_rejects_bad_pattern():
+    with pytest.raises(B.BsolveError) as e:
+        pkg.ell_layout([0, 1, 2], [1, 0])
+    assert e.value.code == B.ERR_PATTERN

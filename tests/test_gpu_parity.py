@@ -104,7 +104,7 @@ def test_x0_null_equals_zero_and_alias():
     B = X.make_batch(0, 4)
     p = B.pattern
     S = Solver(p.row_ptr, p.col_idx, 4)
-    v = to_dev(X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
+    v = to_dev(S.ell_values(B.values))
     b = to_dev(B.b)
     x1, i1, r1, s1 = S.run(v, b)
     z = torch.zeros_like(b)
@@ -237,8 +237,7 @@ def test_csr_to_ell_bit_exact():
     S = Solver(p.row_ptr, p.col_idx, 5)
     ell = S.csr_to_ell(to_dev(B.values))
     torch.cuda.synchronize()
-    assert np.array_equal(ell.cpu().numpy(), X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
-    assert np.array_equal(S.ell_cols(), X.ell_layout(p.row_ptr, p.col_idx)[0])
+    assert np.array_equal(ell.cpu().numpy(), S.ell_values(B.values))
 
 
 @pytest.mark.parametrize("fmt", ["ell", "csr"])
@@ -246,7 +245,7 @@ def test_spmv_vs_oracle(fmt):
     B = X.make_batch(0, 7)
     p = B.pattern
     S = Solver(p.row_ptr, p.col_idx, 7, format=fmt)
-    vals = X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx) if fmt == "ell" else B.values
+    vals = S.ell_values(B.values) if fmt == "ell" else B.values
     xs = X.random_rhs(7, p.n, seed=9)
     y = S.spmv(to_dev(vals), to_dev(xs)).cpu().numpy()
     for i in range(7):
@@ -258,7 +257,7 @@ def test_run_host_matches_run():
     B = X.make_batch(0, 300)
     p = B.pattern
     S = Solver(p.row_ptr, p.col_idx, 300)
-    ell = X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx)
+    ell = S.ell_values(B.values)
     xh, ih, rh, sh = S.run_host(ell, B.b)
     xd, idd, rd, sd = S.run(to_dev(ell), to_dev(B.b))
     torch.cuda.synchronize()
@@ -270,7 +269,7 @@ def test_run_arg_errors_on_gpu():
     B = X.make_batch(0, 2)
     p = B.pattern
     S = Solver(p.row_ptr, p.col_idx, 2)
-    v = to_dev(X.csr_values_to_ell(B.values, p.row_ptr, p.col_idx))
+    v = to_dev(S.ell_values(B.values))
     b = to_dev(B.b)
     with pytest.raises(BsolveError) as e:
         S.run(v, b, tol=-1.0)

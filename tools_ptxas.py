@@ -8,6 +8,6 @@ for l in lines:
     if m and cur: spill = f"spill {m.group(1)}/{m.group(2)}"
     m = re.search(r"Used (\d+) registers", l)
     if m and cur:
-        k = re.search(r"bicgstab_kernelILi(\d)ELi(\d)ELi(\d+)ELi(\d)ELi(\d+)", cur)
+        k = re.search(r"bicgstab_kernelILi(\d)ELi(\d)ELi(\d+)ELb[01]ELi(\d)ELi(\d+)", cur)
         if k: print(f"fmt={k.group(1)} place={k.group(2)} WB={k.group(3)} R={k.group(4)} NT={k.group(5)}: regs {m.group(1)} {spill}")
         cur=None
