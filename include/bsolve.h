@@ -113,6 +113,9 @@ typedef struct bsolve_info {
   int grid;                /* CTAs launched per bsolve_run                    */
   int kl, ku;              /* lower / upper bandwidth of the pattern          */
   int device;
+  int kernel_mode;         /* 1 CSR column table, 2 ELL column table, 3 DIA:
+                              ELL values whose slot k is column row + d_k in
+                              every row (stencils; uniform gather offsets)    */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

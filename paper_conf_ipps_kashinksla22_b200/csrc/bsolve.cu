@@ -10,6 +10,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -58,6 +59,7 @@ struct Variant {
   {F, PL, WB, EX, R, NT, (solve_fn)bicgstab_kernel<F, PL, WB, EX, R, NT, MB>}
 #define V_FP(WB, EX, R, NT, MB)                                                         \
   V_(FMT_ELL, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, EX, R, NT, MB), \
+      V_(FMT_DIA, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_DIA, PLACE_STREAM, WB, EX, R, NT, MB), \
       V_(FMT_CSR, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_CSR, PLACE_STREAM, WB, EX, R, NT, MB)
 
 // W = 9 (the paper's 9-point stencil) gets exact-width variants; any other
@@ -82,6 +84,9 @@ struct bsolve_plan {
   int fmt = 0, place = 0, stop = 0, trc = 1, device = 0;
   int nt = 0, r = 0, smem_bytes = 0, smem_vals = 0, n_pad = 0, ctas_per_sm = 0, num_sms = 0;
   int kl = 0, ku = 0;
+  int kfmt = 0;            // kernel storage mode: FMT_CSR / FMT_ELL / FMT_DIA
+  int guard = 0;           // DIA: zero doubles around the gather body
+  int doff[kMaxW] = {};    // DIA: byte offset of slot k
   long long sys_stride = 0;
   const Variant *var = nullptr;
   std::vector<int32_t> h_ell_col;  // [W][n]
@@ -189,6 +194,10 @@ static void build_ell_map(int n, const int32_t *rp, const int32_t *ci, int W,
   std::vector<int> tmpl;
   for (int k = 0; k < W && k < (int)hist.size(); ++k) tmpl.push_back(hist[k].first);
   std::sort(tmpl.begin(), tmpl.end());
+  // the diagonal (offset 0, present in every row, hence in the template) goes
+  // to slot 0: the kernels keep its value and its gather operand in registers
+  tmpl.erase(std::find(tmpl.begin(), tmpl.end(), 0));
+  tmpl.insert(tmpl.begin(), 0);
   while ((int)tmpl.size() < W) tmpl.push_back(0);
   ell_col.assign((size_t)W * n, 0);
   src.assign((size_t)W * n, -1);
@@ -305,6 +314,30 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   std::vector<int32_t> ell_diag;
   build_ell_map(n, row_ptr, col_idx, W, h->h_ell_col, h->h_csr2ell, ell_diag);
   if (h->fmt == FMT_ELL) diag = ell_diag;  // kernel needs the diagonal's slot in its format
+  h->kfmt = h->fmt;
+  if (h->fmt == FMT_ELL) {
+    // DIA (uniform-offset) addressing if every real entry of slot k sits at
+    // column row + d_k for one d_k per slot: true for stencil patterns
+    std::vector<long long> dk(W, LLONG_MIN);
+    bool uniform = true;
+    for (int k = 0; k < W && uniform; ++k)
+      for (int i = 0; i < n; ++i) {
+        if (h->h_csr2ell[(size_t)k * n + i] < 0) continue;
+        const long long o = (long long)h->h_ell_col[(size_t)k * n + i] - i;
+        if (dk[k] == LLONG_MIN) dk[k] = o;
+        else if (dk[k] != o) { uniform = false; break; }
+      }
+    if (uniform && dk[0] == 0) {
+      long long g = 0;
+      for (int k = 0; k < W; ++k) {
+        if (dk[k] == LLONG_MIN) dk[k] = 0;
+        g = std::max<long long>(g, dk[k] < 0 ? -dk[k] : dk[k]);
+        h->doff[k] = (int)(dk[k] * 8);
+      }
+      h->guard = (int)((g + 1) & ~1LL);
+      h->kfmt = FMT_DIA;
+    }
+  }
 
   // ---- device + variant choice -------------------------------------------
   int dev = opt.device;
@@ -348,7 +381,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->n_pad = (n + 1) & ~1;
   h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
   const int nwarp = nt / 32;
-  const int tail = h->n_pad * 8 + 2 * nwarp * 4 * 8 + 16;
+  const int tail = (h->n_pad + 2 * h->guard) * 8 + 4 * nwarp * 8 + 16;
   const long long smem_need = (long long)h->smem_vals * 8 + tail;
   int place = opt.placement;
   if (place == BSOLVE_PLACE_AUTO) place = smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM;
@@ -359,7 +392,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                           smem_need, smem_optin));
   h->place = place;
   h->smem_bytes = (int)(place == PLACE_SMEM ? smem_need : tail);
-  h->var = find_variant(h->fmt, place, h->wb, h->wb == 9, r, nt);
+  h->var = find_variant(h->kfmt, place, h->wb, h->wb == 9, r, nt);
   if (!h->var)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
                           h->fmt, place, h->wb, r, nt));
@@ -378,12 +411,21 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   // ---- device copy of the pattern ------------------------------------------
   std::vector<int32_t> rp(row_ptr, row_ptr + n + 1);
   const size_t ell_b = sizeof(int32_t) * (size_t)W * n;
+  // Column table the kernels read, [W][n]: ELL -> the slot map; CSR -> the
+  // k-th CSR entry of each row (padding: own row, never multiplied).
+  std::vector<int32_t> kcols = h->h_ell_col;
+  if (h->fmt == FMT_CSR)
+    for (int i = 0; i < n; ++i)
+      for (int k = 0; k < W; ++k) {
+        const int e = row_ptr[i] + k;
+        kcols[(size_t)k * n + i] = e < row_ptr[i + 1] ? col_idx[e] : i;
+      }
   if (cudaMalloc(&h->d_ell_col, ell_b) != cudaSuccess ||
       cudaMalloc(&h->d_src, ell_b) != cudaSuccess ||
       cudaMalloc(&h->d_row_ptr, sizeof(int32_t) * (n + 1)) != cudaSuccess ||
       cudaMalloc(&h->d_diag, sizeof(int32_t) * n) != cudaSuccess)
     return fail_free(fail(BSOLVE_ERR_NOMEM, "device allocation of the pattern failed"));
-  if (cudaMemcpy(h->d_ell_col, h->h_ell_col.data(), ell_b, cudaMemcpyHostToDevice) != cudaSuccess ||
+  if (cudaMemcpy(h->d_ell_col, kcols.data(), ell_b, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(h->d_src, h->h_csr2ell.data(), ell_b, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(h->d_row_ptr, rp.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice) !=
           cudaSuccess ||
@@ -418,6 +460,7 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->kl = h->kl;
   info->ku = h->ku;
   info->device = h->device;
+  info->kernel_mode = h->kfmt;
   return BSOLVE_OK;
 }
 
@@ -466,6 +509,8 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   P.trc = h->trc;
   P.smem_vals = h->smem_vals;
   P.n_pad = h->n_pad;
+  P.guard = h->guard;
+  for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
   h->var->fn<<<count, h->nt, h->smem_bytes, stream>>>(P);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));

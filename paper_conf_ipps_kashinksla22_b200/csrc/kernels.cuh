@@ -14,23 +14,26 @@
 //  * every BiCGSTAB vector lives in REGISTERS: thread t owns rows t + j*NT,
 //    j < R.  Only the vector being multiplied (p^ or s^) is published to a
 //    shared "gather" buffer for the SpMV.
-//  * column indices are held in registers as packed 16-bit byte offsets into
-//    the gather buffer (read once per CTA from the shared pattern in L2).
-//  * dot products and norms are fused into the vector updates and reduced
-//    warp-shuffle -> one __syncthreads -> redundant per-thread final sum over
-//    the NT/32 warp partials, so every reduction costs exactly one barrier
-//    and all threads hold bitwise-identical scalars (uniform control flow,
-//    deterministic results independent of batch partitioning).
+//  * the shared-memory data pipe (LDS wavefronts + SHFL) is the bound, so the
+//    kernel minimises wavefronts: conflict-free ELL slot map, diagonal in
+//    slot 0 (its value and its gather operand stay in registers), offset
+//    ("DIA") addressing for stencil patterns (no column registers, no index
+//    arithmetic), and reductions that spend as few shuffles as possible.
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
 
 namespace bsolve {
 
-enum { FMT_CSR = 1, FMT_ELL = 2 };
+// Kernel-level storage modes.  CSR and ELL are the paper's BatchCsr and
+// BatchEll.  DIA is BatchEll values whose slot k holds,
+// in every row r, the entry of column r + d_k (the host detects this for
+// stencil patterns): the gather address is row + d_k with d_k uniform.
+enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
 enum { PLACE_SMEM = 1, PLACE_STREAM = 2 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
+constexpr int kMaxW = 16;
 
 struct SolveParams {
   const double *values;     // [batch][sys_stride]
@@ -40,14 +43,16 @@ struct SolveParams {
   int32_t *iters;           // [batch]
   double *resnorm;          // [batch]
   int8_t *status;           // [batch] or nullptr
-  const int32_t *ell_col;   // [W][n] shared pattern, column-major
+  const int32_t *ell_col;   // [W][n] column table, column-major
   const int32_t *row_ptr;   // [n+1]
-  const int32_t *diag_slot; // [n] slot of the diagonal entry in its row
+  const int32_t *diag_slot; // [n] CSR position of the diagonal in its row
   long long sys_stride;     // doubles per system in `values`
   double tol;
   int n, W, batch, maxiter, stop, trc;
   int smem_vals;            // doubles of SMEM reserved for values (even)
-  int n_pad;                // doubles of the gather buffer (even)
+  int n_pad;                // doubles of the gather buffer body (even)
+  int guard;                // zero doubles before and after the gather body (DIA)
+  int doff[kMaxW];          // DIA: byte offset d_k * 8 of slot k
 };
 
 // ------------------------------------------------------------ PTX helpers --
@@ -60,9 +65,6 @@ __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
 }
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void fence_proxy_async_smem() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
@@ -90,50 +92,53 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity)
 
 __device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
 
-// Block-wide sum of K doubles with ONE barrier:
-//  1. xor-butterfly inside each warp (after it every lane holds the same
-//     bits: at each step lanes L and L^o add the same two operands, and fp
-//     addition is commutative);
-//  2. lane 0 of each warp publishes its partial, __syncthreads();
-//  3. lane w < NWARP of EVERY warp loads partial w (one LDS wavefront per
-//     value per warp instead of NWARP broadcast loads), then a butterfly over
-//     the NWARP lanes and a broadcast from lane 0 give every thread the same
-//     bits.  Fixed order => deterministic, independent of batch slicing.
-// `buf` alternates between two scratch halves so that the next reduction
-// never overwrites partials a slow warp is still reading.
+// Block-wide sum of K in {1, 2} doubles with ONE barrier.  Every SHFL costs
+// one data-pipe wavefront on B200, like an LDS, so:
+//  * inside a warp: xor butterfly; for K = 2 the first step is a recursive
+//    halving exchange (lanes with bit 4 clear keep value 0, the others value
+//    1), so two sums cost the shuffles of one plus one step;
+//  * lane 0 (value 0) / lane 16 (value 1) publish the warp partial;
+//  * after the barrier every thread reads the NWARP partials of each value
+//    with broadcast 16-byte loads and adds them in warp order.
+// All threads obtain bitwise-identical sums in a fixed order (uniform control
+// flow, results independent of batch slicing).  `buf` alternates between
+// two scratch halves so the next reduction never overwrites partials that a
+// slow warp is still reading.
 template <int K, int NWARP>
 __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf, int lane,
                                           int warp) {
-  static_assert((NWARP & (NWARP - 1)) == 0 && NWARP <= 32, "NWARP must be a power of two");
+  static_assert(K == 1 || K == 2, "block_sum supports 1 or 2 values");
+  static_assert(NWARP % 2 == 0, "NWARP must be even");
+  double keep;
+  if (K == 2) {
+    const bool hi = lane & 16;
+    const double send = hi ? v[0] : v[K - 1];
+    keep = hi ? v[K - 1] : v[0];
+    keep += __shfl_xor_sync(0xffffffffu, send, 16);
 #pragma unroll
-  for (int k = 0; k < K; ++k) {
+    for (int o = 8; o > 0; o >>= 1) keep += __shfl_xor_sync(0xffffffffu, keep, o);
+  } else {
+    keep = v[0];
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v[k] += __shfl_xor_sync(0xffffffffu, v[k], o);
+    for (int o = 16; o > 0; o >>= 1) keep += __shfl_xor_sync(0xffffffffu, keep, o);
   }
-  double *S = sred + buf * (NWARP * 4);
-  if (lane == 0) {
-#pragma unroll
-    for (int k = 0; k < K; ++k) S[k * NWARP + warp] = v[k];
-  }
+  double *S = sred + buf * (2 * NWARP);
+  if ((lane & 15) == 0 && (K == 2 || lane == 0)) S[(lane >> 4) * NWARP + warp] = keep;
   __syncthreads();
 #pragma unroll
   for (int k = 0; k < K; ++k) {
-    double a = lane < NWARP ? S[k * NWARP + lane] : 0.0;
+    const double2 *S2 = reinterpret_cast<const double2 *>(S + k * NWARP);
+    double a = 0.0;
 #pragma unroll
-    for (int o = NWARP / 2; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-    v[k] = __shfl_sync(0xffffffffu, a, 0);
+    for (int w = 0; w < NWARP / 2; ++w) {
+      const double2 q = S2[w];
+      a += q.x;
+      a += q.y;
+    }
+    v[k] = a;
   }
   buf ^= 1;
 }
-
-// Per-thread view of its rows of the shared pattern.
-template <int WB, int R>
-struct RowMeta {
-  uint32_t cpk[R][(WB + 1) / 2]; // packed 16-bit byte offsets (col*8) into the gather buffer
-  int vbase[R];                  // ELL: row; CSR: row_ptr[row]
-  int vlen[R];                   // CSR row length
-  bool act[R];                   // row < n
-};
 
 // Extract the 16-bit field at bit `POS` of `pk`.  volatile keeps the unpack
 // inside the SpMV loop instead of letting the compiler hoist twice as many
@@ -145,36 +150,62 @@ __device__ __forceinline__ uint32_t field16(uint32_t pk) {
   return v;
 }
 
+// Per-thread view of its rows of the shared pattern.
+template <int FMT, int WB, int R>
+struct RowMeta {
+  uint32_t cpk[R][(WB + 1) / 2]; // CSR/ELL: packed 16-bit byte offsets (col*8) into the gather body
+  int vbase[R];                  // ELL/DIA: row (clamped for idle lanes); CSR: row_ptr[row]
+  int vlen[R];                   // CSR row length
+  double a0[R];                  // ELL/DIA: the diagonal value (slot 0)
+  bool act[R];                   // row < n
+};
+
 // y = A * g for this thread's rows (one thread per row,
-// W sequential slots, no intra-row reduction).  g is the shared gather
-// buffer sg; values come from V (shared or global).  EXACT: W == WB known at
-// compile time (no per-slot test).  A warp whose rows j are all >= n skips
-// block j with a warp-uniform branch; lanes of a partial warp run on a
-// clamped row and zero their result.
+// W sequential slots, no intra-row reduction).  `gb` points at the gather
+// body (byte address), `own[j]` is this thread's own gather entry g[row]
+// (ELL/DIA: slot 0 is the diagonal, so its operand never leaves registers).
+// Values come from V (shared or global).  EXACT: W == WB at compile time.
+// A warp whose row block j lies entirely at or beyond n skips it with a
+// warp-uniform branch; idle lanes of a partial warp run on a clamped row and
+// zero their result.
 template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT>
-__device__ __forceinline__ void spmv_rows(const double *__restrict__ V, const double *sg, int n,
-                                          int W, const RowMeta<WB, R> &m, double (&y)[R]) {
-  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+__device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
+                                          const unsigned char *gb, const SolveParams &P,
+                                          const RowMeta<FMT, WB, R> &m, const double (&own)[R],
+                                          double (&y)[R]) {
+  const int n = P.n;
   const int wrow0 = threadIdx.x & ~31;
 #pragma unroll
   for (int j = 0; j < R; ++j) {
     double acc = 0.0;
     if (wrow0 + j * NT < n) {
+      if (FMT == FMT_CSR) {
 #pragma unroll
-      for (int k = 0; k < WB; ++k) {
-        if (EXACT || k < W) {
-          const uint32_t off = (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
-          const double g = *reinterpret_cast<const double *>(gb + off);
-          if (FMT == FMT_ELL) {
-            const double *a_p = V + m.vbase[j] + k * n;
-            const double a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
-            acc = fma(a, g, acc);
-          } else {
-            if (k < m.vlen[j]) {
-              const double *a_p = V + m.vbase[j] + k;
-              const double a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
-              acc = fma(a, g, acc);
+        for (int k = 0; k < WB; ++k) {
+          if ((EXACT || k < P.W) && k < m.vlen[j]) {
+            const uint32_t off =
+                (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+            const double g = *reinterpret_cast<const double *>(gb + off);
+            const double *a_p = V + m.vbase[j] + k;
+            acc = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p, g, acc);
+          }
+        }
+      } else {
+        acc = m.a0[j] * own[j];  // slot 0: diagonal, operand = own entry
+        const unsigned char *grow = gb + m.vbase[j] * 8;
+#pragma unroll
+        for (int k = 1; k < WB; ++k) {
+          if (EXACT || k < P.W) {
+            double g;
+            if (FMT == FMT_DIA) {
+              g = *reinterpret_cast<const double *>(grow + P.doff[k]);
+            } else {
+              const uint32_t off =
+                  (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+              g = *reinterpret_cast<const double *>(gb + off);
             }
+            const double *a_p = V + m.vbase[j] + k * n;
+            acc = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p, g, acc);
           }
         }
       }
@@ -185,19 +216,22 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V, const do
 
 // ------------------------------------------------------------ the solver --
 // Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
-//   [values: smem_vals doubles (PLACE_SMEM only)] [gather: n_pad doubles]
-//   [reduction scratch: 2*NWARP*4 doubles] [mbarrier: 8 B]
+//   [values: smem_vals doubles (PLACE_SMEM only)]
+//   [gather: guard | n_pad body | guard doubles]
+//   [reduction scratch: 2 * 2 * NWARP doubles] [mbarrier: 8 B]
 template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB>
 __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double *sval = reinterpret_cast<double *>(smem_raw);
-  double *sg = sval + (PLACE == PLACE_SMEM ? P.smem_vals : 0);
-  double *sred = sg + P.n_pad;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 2 * NWARP * 4);
+  double *sgf = sval + (PLACE == PLACE_SMEM ? P.smem_vals : 0);  // gather incl. guards
+  double *sg = sgf + P.guard;                                     // gather body
+  double *sred = sgf + P.n_pad + 2 * P.guard;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 4 * NWARP);
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int n = P.n, W = P.W;
+  const int n = P.n;
   const long long sys = blockIdx.x;
   const double *gval = P.values + sys * P.sys_stride;
 
@@ -226,9 +260,15 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     }
   }
   const double *V = (PLACE == PLACE_SMEM) ? sval : gval;
+  // zero the gather guards (read, times a zero value, by DIA padding slots);
+  // the first gather happens after at least one __syncthreads
+  for (int i = tid; i < P.guard; i += NT) {
+    sgf[i] = 0.0;
+    sg[P.n_pad + i] = 0.0;
+  }
 
   // ---- pattern + right-hand side + initial guess into registers ----------
-  RowMeta<WB, R> m;
+  RowMeta<FMT, WB, R> m;
   double x[R], r[R], rh[R], p[R], v[R], d[R];
   const double *bsys = P.b + sys * n;
   int dsl[R];
@@ -238,27 +278,28 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     m.act[j] = row < n;
 #pragma unroll
     for (int k = 0; k < (WB + 1) / 2; ++k) m.cpk[j][k] = 0u;
-    m.vbase[j] = (FMT == FMT_ELL) ? (row < n ? row : n - 1) : 0;  // clamped for idle lanes
+    m.vbase[j] = (FMT == FMT_CSR) ? 0 : (row < n ? row : n - 1);
     m.vlen[j] = 0;
+    m.a0[j] = 0.0;
     dsl[j] = 0;
     r[j] = 0.0;
     x[j] = 0.0;
     if (m.act[j]) {
+      if (FMT != FMT_DIA) {
 #pragma unroll
-      for (int k = 0; k < WB; ++k) {
-        if (k < W) {
-          const uint32_t off = static_cast<uint32_t>(__ldg(P.ell_col + (size_t)k * n + row)) * 8u;
-          m.cpk[j][k >> 1] |= (k & 1) ? (off << 16) : off;
+        for (int k = 0; k < WB; ++k) {
+          if (EXACT || k < P.W) {
+            const uint32_t off =
+                static_cast<uint32_t>(__ldg(P.ell_col + (size_t)k * n + row)) * 8u;
+            m.cpk[j][k >> 1] |= (k & 1) ? (off << 16) : off;
+          }
         }
       }
-      if (FMT == FMT_ELL) {
-        m.vbase[j] = row;
-        m.vlen[j] = W;
-      } else {
+      if (FMT == FMT_CSR) {
         m.vbase[j] = __ldg(P.row_ptr + row);
         m.vlen[j] = __ldg(P.row_ptr + row + 1) - m.vbase[j];
+        dsl[j] = __ldg(P.diag_slot + row);
       }
-      dsl[j] = __ldg(P.diag_slot + row);
       r[j] = __ldg(bsys + row);  // r holds b until the initial residual is formed
       if (P.x0) x[j] = __ldg(P.x0 + sys * n + row);
     }
@@ -271,12 +312,10 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   // ---- a2: scalar Jacobi d = 1/a_rr (zero diagonal -> 1, DESIGN R11) -----
 #pragma unroll
   for (int j = 0; j < R; ++j) {
-    d[j] = 1.0;
-    if (m.act[j]) {
-      const int pos = (FMT == FMT_ELL) ? dsl[j] * n + m.vbase[j] : m.vbase[j] + dsl[j];
-      const double a = (PLACE == PLACE_STREAM) ? __ldg(V + pos) : V[pos];
-      d[j] = (a != 0.0) ? 1.0 / a : 1.0;
-    }
+    const int pos = (FMT == FMT_CSR) ? m.vbase[j] + dsl[j] : m.vbase[j];  // ELL/DIA: slot 0
+    const double a = m.act[j] ? ((PLACE == PLACE_STREAM) ? __ldg(V + pos) : V[pos]) : 0.0;
+    if (FMT != FMT_CSR) m.a0[j] = a;
+    d[j] = (a != 0.0) ? 1.0 / a : 1.0;
   }
 
   int buf = 0;
@@ -290,7 +329,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R];
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) r[j] = r[j] - q[j];
   }
@@ -330,14 +369,16 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (bad(rho)) { st = SYS_BREAKDOWN; break; }
       const double beta = (rho / rho_old) * (alpha / omega);  // R2
       // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
+      double ph[R];
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         p[j] = r[j] + beta * (p[j] - omega * v[j]);
-        if (m.act[j]) sg[tid + j * NT] = d[j] * p[j];
+        ph[j] = d[j] * p[j];
+        if (m.act[j]) sg[tid + j * NT] = ph[j];
       }
       __syncthreads();
       // a6: v = A p^
-      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, v);
+      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, ph, v);
       ++it;
       // a7: alpha = rho / (r^ . v)
       double rv[1] = {0.0};
@@ -348,12 +389,13 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       alpha = rho / rv[0];                                 // R3
       // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
       // barrier in the reduction above separates them)
-      double s[R], ss[1] = {0.0};
+      double s[R], sh[R], ss[1] = {0.0};
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         s[j] = r[j] - alpha * v[j];
         ss[0] += s[j] * s[j];
-        if (m.act[j]) sg[tid + j * NT] = d[j] * s[j];
+        sh[j] = d[j] * s[j];
+        if (m.act[j]) sg[tid + j * NT] = sh[j];
       }
       block_sum<1, NWARP>(ss, sred, buf, lane, warp);      // also publishes s^
       if (sqrt(ss[0]) < tau) {                             // stop test 2
@@ -364,7 +406,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       }
       // a9: t = A s^
       double t[R];
-      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, t);
+      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, sh, t);
       // a10: omega = (t.s)/(t.t); x, r updates
       double ts[2] = {0.0, 0.0};
 #pragma unroll
@@ -398,7 +440,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
       q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
@@ -429,7 +471,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
       if (m.act[j]) sg[tid + j * NT] = x[j];
     __syncthreads();
     double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, sg, n, W, m, q);
+    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
       q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
@@ -455,12 +497,13 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
 // -------------------------------------------------- standalone batched SpMV --
 // y_i = A_i x_i (Fig. 7).  One CTA per system; x_i is
 // staged into SMEM for the gather, values stream from global (coalesced for
-// ELL: consecutive rows of one slot are contiguous).
+// ELL: consecutive rows of one slot are contiguous).  `cols` is the column
+// table of the handle's format ([W][n]; CSR: k-th entry of the row).
 template <int FMT, int NT>
 __global__ void __launch_bounds__(NT) spmv_kernel(const double *__restrict__ values,
                                                   const double *__restrict__ xin,
                                                   double *__restrict__ y,
-                                                  const int32_t *__restrict__ ell_col,
+                                                  const int32_t *__restrict__ cols,
                                                   const int32_t *__restrict__ row_ptr, int n,
                                                   int W, long long sys_stride) {
   extern __shared__ __align__(16) double sx[];
@@ -470,13 +513,13 @@ __global__ void __launch_bounds__(NT) spmv_kernel(const double *__restrict__ val
   __syncthreads();
   for (int row = threadIdx.x; row < n; row += NT) {
     double acc = 0.0;
-    if (FMT == FMT_ELL) {
-      for (int k = 0; k < W; ++k)
-        acc = fma(__ldg(V + (size_t)k * n + row), sx[__ldg(ell_col + (size_t)k * n + row)], acc);
-    } else {
+    if (FMT == FMT_CSR) {
       const int a = __ldg(row_ptr + row), e = __ldg(row_ptr + row + 1);
       for (int q = a; q < e; ++q)
-        acc = fma(__ldg(V + q), sx[__ldg(ell_col + (size_t)(q - a) * n + row)], acc);
+        acc = fma(__ldg(V + q), sx[__ldg(cols + (size_t)(q - a) * n + row)], acc);
+    } else {
+      for (int k = 0; k < W; ++k)
+        acc = fma(__ldg(V + (size_t)k * n + row), sx[__ldg(cols + (size_t)k * n + row)], acc);
     }
     y[sys * n + row] = acc;
   }
@@ -495,8 +538,8 @@ __global__ void csr_to_ell_kernel(const double *__restrict__ csr, double *__rest
 }
 
 // -------------------------------------------------- SMEM bandwidth probe --
-// Every thread streams conflict-free 16-byte shared loads; the sum is kept
-// live through a conditional store.  bytes = grid * NT * ITERS * 4 * 16.
+// Every thread streams conflict-free 32-byte shared loads; the sum is kept
+// live through a conditional store.  bytes = grid * NT * iters * 4 * 32.
 template <int NT>
 __global__ void __launch_bounds__(NT) smem_probe_kernel(int iters, double *sink,
                                                         long long *cycles) {
