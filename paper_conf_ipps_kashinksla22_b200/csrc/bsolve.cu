@@ -208,10 +208,9 @@ static void build_ell_map(int n, const int32_t *rp, const int32_t *ci, int W,
     std::vector<int> rest;
     for (int e = rp[i]; e < rp[i + 1]; ++e) {
       const int o = ci[e] - i;
-      int k = (int)(std::lower_bound(tmpl.begin(), tmpl.end(), o) - tmpl.begin());
       bool placed = false;
-      for (; k < W && tmpl[k] == o; ++k)
-        if (!used[k]) {
+      for (int k = 0; k < W; ++k)  // tmpl is not sorted (offset 0 first)
+        if (tmpl[k] == o && !used[k]) {
           used[k] = 1;
           src[(size_t)k * n + i] = e;
           ell_col[(size_t)k * n + i] = ci[e];

@@ -183,3 +183,20 @@ def test_ell_layout_rejects_bad_pattern():
     with pytest.raises(B.BsolveError) as e:
         pkg.ell_layout([0, 1, 2], [1, 0])
     assert e.value.code == B.ERR_PATTERN
+
+
+def test_ell_map_slot0_diagonal_and_stencil_offsets():
+    """Slot 0 holds the diagonal in every row (any pattern); for stencils each
+    slot has one column offset (the kernel's DIA addressing)."""
+    import xgcgen as X
+    pats = [X.stencil_pattern(32, 31), X.stencil_pattern(5, 5), X.stencil_pattern(64, 32)]
+    for pat in pats:
+        W, cols, src = pkg.ell_layout(pat.row_ptr, pat.col_idx)
+        n = pat.n
+        assert np.all(cols[:n] == np.arange(n)) and np.all(src[:n] >= 0)
+        for k in range(W):
+            offs = {int(cols[k * n + i]) - i for i in range(n) if src[k * n + i] >= 0}
+            assert len(offs) == 1
+    rp, ci = X.random_pattern(200, 9, seed=7)
+    W, cols, src = pkg.ell_layout(rp, ci)
+    assert np.all(cols[:200] == np.arange(200)) and np.all(src[:200] >= 0)
