@@ -218,7 +218,7 @@ def run_reference(args, rank, world):
     """--impl reference: the oracle (as it stands) on the host cores."""
     if rank != 0:
         return
-    per_rank = args.batch if args.scaling == "weak" else args.batch // world
+    per_rank = rank_slice_count(args, world)
     cal = oracle_sample_rate(0, per_rank, args, target_s=min(5.0, args.cpu_seconds))
     count = cal["_count"]
     import oracle as O
@@ -248,12 +248,18 @@ def run_reference(args, rank, world):
     emit(line, args)
 
 
+def rank_slice_count(args, world):
+    from paper_conf_ipps_kashinksla22_b200.parallel import rank_slice
+    return rank_slice(args.batch, 0, world, args.scaling).count
+
+
 def config_dict(args, world, per_rank):
     n = args.nx * args.ny
     return {"workload": f"xgc{n}_9pt_mix_zero_guess",
             "description": "BASELINE configs[3]: 10^5-system batch of XGC-shaped 9-point "
                            "stencil systems per GPU, 50/50 ion/electron, x0 = 0",
-            "batch_per_gpu": per_rank, "global_batch": per_rank * world, "n": n,
+            "batch_per_gpu": per_rank,
+            "global_batch": args.batch * world if args.scaling == "weak" else args.batch, "n": n,
             "grid": f"{args.nx}x{args.ny}", "format": args.format, "placement": args.placement,
             "tol": args.tol, "stop": "rel_b", "maxiter": args.maxiter, "x0": "zero",
             "parallelism": f"batch-partitioned x{world} (one process per GPU, no solve-path "
@@ -274,11 +280,13 @@ def run_ours(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_kashinksla22_b200 import Solver, probe_smem_bandwidth
+    from paper_conf_ipps_kashinksla22_b200.parallel import (gather_stats, max_over_ranks,
+                                                            rank_slice)
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    per_rank = args.batch if args.scaling == "weak" else args.batch // world
-    g0 = rank * per_rank
+    sl = rank_slice(args.batch, rank, world, args.scaling)
+    per_rank, g0 = sl.count, sl.g0
     pat, vals_h, b_h = make_inputs(g0, per_rank, args, pinned=True)
     n, nnz, W = pat.n, pat.nnz, pat.max_row_nnz
     S = Solver(pat.row_ptr, pat.col_idx, per_rank, format=args.format,
@@ -315,26 +323,15 @@ def run_ours(args, rank, world, local_rank):
         barrier()
     total_ms = ev0.elapsed_time(ev1)
     kern_ms = [a.elapsed_time(bb) for a, bb in launch_ms]
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms = float(t.item())
+    total_ms = max_over_ranks(total_ms, device=dev)
     ms_per_step = total_ms / args.steps
-    value = per_rank * world * args.steps / (total_ms * 1e-3)
+    value = sl.total * args.steps / (total_ms * 1e-3)
 
     # ---- stats of the last step (outside the timed region) ------------------
     it_h = it.cpu().numpy()
     st_h = st.cpu().numpy()
     res_h = res.cpu().numpy()
-    if world > 1:
-        its = [torch.empty_like(it) for _ in range(world)]
-        dist.all_gather(its, it)
-        sts = [torch.empty_like(st) for _ in range(world)]
-        dist.all_gather(sts, st)
-        it_all = torch.cat(its).cpu().numpy()
-        st_all = torch.cat(sts).cpu().numpy()
-    else:
-        it_all, st_all = it_h, st_h
+    it_all, _, st_all = (t.numpy() for t in gather_stats(it, res, st))
     sum_iters_rank = int(it_h.astype(np.int64).sum())
 
     # ---- roofline (dominant kernel = the one solve kernel per step) ---------
@@ -399,13 +396,10 @@ def run_ours(args, rank, world, local_rank):
             S.run_host(vn, bn, None, args.tol, args.maxiter, out=outs)
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
-        tt = torch.tensor([dt], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        dt = float(tt.item())
+        dt = max_over_ranks(dt, device=dev)
         h2d = int(vn.nbytes + bn.nbytes)
         d2h = int(x_h.nbytes + i_h.nbytes + r_h.nbytes + s_h.nbytes)
-        e2e = {"value": per_rank * world * e2e_steps / dt, "unit": UNIT,
+        e2e = {"value": sl.total * e2e_steps / dt, "unit": UNIT,
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps,
                "api": "bsolve_run_host (C ABI, chunked H2D/solve/D2H pipeline)",
                "bitwise_equal_to_device_path": bool(np.array_equal(i_h, it_h) and
