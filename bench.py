@@ -375,6 +375,22 @@ def run_ours(args, rank, world, local_rank):
                 "frac": hbm_achieved / hbm_peak, "bytes_per_system": hbm_bytes_sys,
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
     }
+    # traffic from the committed ncu --set full capture of this kernel on this
+    # workload (profiles/ncu_traffic.json), scaled to this launch's systems
+    try:
+        tr = _json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        scale = per_rank / tr["systems_per_launch"]
+        roofline["traffic"] = tr["smem_data_pipe_bytes_per_launch"] * scale
+        roofline["traffic_unit"] = ("bytes per launch through the SMEM/L1 data pipe "
+                                    "(ncu l1tex__data_pipe_lsu_wavefronts_mem_shared x 128 B)")
+        roofline["traffic_over_algorithmic"] = (roofline["traffic"] / smem_bytes_launch
+                                                if smem_bytes_launch else None)
+        roofline["hbm"]["traffic"] = tr["dram_bytes_per_launch"] * scale
+        roofline["hbm"]["traffic_over_algorithmic"] = (tr["dram_bytes_per_launch"] * scale /
+                                                       (hbm_bytes_sys * per_rank))
+        roofline["traffic_source"] = tr["source"]
+    except Exception:  # noqa: BLE001 - no capture committed for this build
+        pass
     if clocks.get("sm_mhz"):
         roofline["frac_at_observed_clock"] = smem_achieved / (128.0 * num_sms *
                                                               clocks["sm_mhz"] * 1e6)
