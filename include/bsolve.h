@@ -70,9 +70,14 @@ enum {
 /* Where the matrix values live while a system iterates (PAPER.md:708-721,
  * 738-813: the paper's automatic shared-memory configuration). */
 enum {
-  BSOLVE_PLACE_AUTO = 0,   /* SMEM if one system's values fit, else STREAM   */
+  BSOLVE_PLACE_AUTO = 0,   /* REGS if eligible, else SMEM if one system's
+                              values fit, else STREAM                         */
   BSOLVE_PLACE_SMEM = 1,   /* staged once into shared memory by TMA bulk copy */
-  BSOLVE_PLACE_STREAM = 2  /* re-read from global memory (L2/L1) every SpMV   */
+  BSOLVE_PLACE_STREAM = 2, /* re-read from global memory (L2/L1) every SpMV   */
+  BSOLVE_PLACE_REGS = 3    /* persistent kernel, one CTA per SM: values staged by
+                              TMA, then held in REGISTERS for the whole solve;
+                              the next system's TMA overlaps the current one
+                              (ELL, 9 entries per row, even n <= 1024)        */
 };
 
 /* Stopping criterion (R5). */
@@ -110,7 +115,7 @@ typedef struct bsolve_info {
   int smem_bytes;          /* dynamic shared memory per CTA                   */
   int ctas_per_sm;         /* resident CTAs per SM (occupancy calculator)     */
   int num_sms;             /* SMs on the device                               */
-  int grid;                /* CTAs launched per bsolve_run                    */
+  int grid;                /* CTAs launched per bsolve_run (REGS: persistent) */
   int kl, ku;              /* lower / upper bandwidth of the pattern          */
   int device;
   int kernel_mode;         /* 1 CSR column table, 2 ELL column table, 3 DIA:

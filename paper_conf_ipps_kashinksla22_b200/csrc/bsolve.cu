@@ -11,6 +11,7 @@
 
 #include <algorithm>
 #include <climits>
+#include <cstdint>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -70,6 +71,21 @@ static const Variant kVariants[] = {
     V_FP(16, false, 4, 256, 2), V_FP(16, false, 4, 512, 1),
 };
 
+// Persistent register-resident variants (PLACE_REGS): ELL/DIA, W = 9.
+typedef void (*persist_fn)(const SolveParams, unsigned long long *);
+struct PVariant {
+  int fmt, r;
+  persist_fn fn;
+};
+#define PV_(F, R) {F, R, (persist_fn)bicgstab_persist_kernel<F, 9, true, R, 256>}
+static const PVariant kPVariants[] = {PV_(FMT_DIA, 1), PV_(FMT_DIA, 2), PV_(FMT_DIA, 4),
+                                      PV_(FMT_ELL, 1), PV_(FMT_ELL, 2), PV_(FMT_ELL, 4)};
+static const PVariant *find_pvariant(int fmt, int r) {
+  for (const PVariant &v : kPVariants)
+    if (v.fmt == fmt && v.r == r) return &v;
+  return nullptr;
+}
+
 static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt) {
   for (const Variant &v : kVariants)
     if (v.fmt == fmt && v.place == place && v.wb == wb && v.exact == exact && v.r == r &&
@@ -88,7 +104,10 @@ struct bsolve_plan {
   int guard = 0;           // DIA: zero doubles around the gather body
   int doff[kMaxW] = {};    // DIA: byte offset of slot k
   long long sys_stride = 0;
-  const Variant *var = nullptr;
+  const Variant *var = nullptr;      // per-system-CTA kernel (also the REGS fallback)
+  const PVariant *pvar = nullptr;    // persistent kernel when place == PLACE_REGS
+  int smem_bytes_fallback = 0, grid_persist = 0;
+  unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
   std::vector<int32_t> h_ell_col;  // [W][n]
   std::vector<int32_t> h_csr2ell;  // [W][n] -> CSR entry held by the slot, -1 = padding
   int32_t *d_ell_col = nullptr, *d_row_ptr = nullptr, *d_diag = nullptr, *d_src = nullptr;
@@ -121,6 +140,7 @@ static void free_plan(bsolve_plan *h) {
   cudaFree(h->d_row_ptr);
   cudaFree(h->d_diag);
   cudaFree(h->d_src);
+  cudaFree(h->d_ctr);
   for (int s = 0; s < bsolve_plan::kSlots; ++s) {
     if (h->hs[s]) cudaStreamDestroy(h->hs[s]);
     cudaFree(h->h_val[s]);
@@ -382,30 +402,65 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   const int nwarp = nt / 32;
   const int tail = (h->n_pad + 2 * h->guard) * 8 + 4 * nwarp * 8 + 16;
   const long long smem_need = (long long)h->smem_vals * 8 + tail;
+  // PLACE_REGS: persistent kernel, values in registers, staging buffers for
+  // values + b + x0 in SMEM (DESIGN.md "Kernels" 7)
+  const long long smem_regs = (long long)h->smem_vals * 8 + 2LL * h->n_pad * 8 + tail + 16;
+  const bool regs_ok = (h->kfmt == FMT_ELL || h->kfmt == FMT_DIA) && W == 9 && nt == 256 &&
+                       n % 2 == 0 && (h->sys_stride * 8) % 16 == 0 && smem_regs <= smem_optin &&
+                       find_pvariant(h->kfmt, r) != nullptr;
   int place = opt.placement;
-  if (place == BSOLVE_PLACE_AUTO) place = smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM;
-  else place = place == BSOLVE_PLACE_SMEM ? PLACE_SMEM : PLACE_STREAM;
+  if (place == BSOLVE_PLACE_AUTO)
+    place = regs_ok ? PLACE_REGS : (smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM);
+  else if (place == BSOLVE_PLACE_REGS) {
+    if (!regs_ok)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                            "register-resident placement needs ELL, 9 entries per row, even "
+                            "n <= 1024 and %lld B of shared memory",
+                            smem_regs));
+    place = PLACE_REGS;
+  } else
+    place = place == BSOLVE_PLACE_SMEM ? PLACE_SMEM : PLACE_STREAM;
   if (place == PLACE_SMEM && smem_need > smem_optin)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "SMEM placement needs %lld B of shared memory, device allows %d",
                           smem_need, smem_optin));
   h->place = place;
-  h->smem_bytes = (int)(place == PLACE_SMEM ? smem_need : tail);
-  h->var = find_variant(h->kfmt, place, h->wb, h->wb == 9, r, nt);
+  // the per-system-CTA kernel: the plan itself (SMEM/STREAM) or the fallback
+  // of PLACE_REGS for buffers that are not 16-byte aligned
+  const int fb_place = (place == PLACE_STREAM || smem_need > smem_optin) ? PLACE_STREAM : PLACE_SMEM;
+  h->smem_bytes_fallback = (int)(fb_place == PLACE_SMEM ? smem_need : tail);
+  h->var = find_variant(h->kfmt, fb_place, h->wb, h->wb == 9, r, nt);
   if (!h->var)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
-                          h->fmt, place, h->wb, r, nt));
+                          h->fmt, fb_place, h->wb, r, nt));
   ce = cudaFuncSetAttribute((const void *)h->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            h->smem_bytes);
+                            h->smem_bytes_fallback);
   if (ce != cudaSuccess)
     return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
   cudaFuncSetAttribute((const void *)h->var->fn, cudaFuncAttributePreferredSharedMemoryCarveout,
                        cudaSharedmemCarveoutMaxShared);
-  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var->fn, nt, h->smem_bytes);
+  if (place == PLACE_REGS) {
+    h->pvar = find_pvariant(h->kfmt, r);
+    h->smem_bytes = (int)smem_regs;
+    ce = cudaFuncSetAttribute((const void *)h->pvar->fn,
+                              cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
+    if (ce != cudaSuccess)
+      return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->pvar->fn, nt,
+                                                       h->smem_bytes);
+    if (cudaMalloc(&h->d_ctr, 2 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(h->d_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
+      return fail_free(fail(BSOLVE_ERR_NOMEM, "work counter allocation failed"));
+  } else {
+    h->smem_bytes = h->smem_bytes_fallback;
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var->fn, nt,
+                                                       h->smem_bytes);
+  }
   if (ce != cudaSuccess)
     return fail_free(fail(BSOLVE_ERR_CUDA, "occupancy query: %s", cudaGetErrorString(ce)));
   if (h->ctas_per_sm < 1)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "kernel variant cannot be resident on an SM"));
+  h->grid_persist = h->num_sms * h->ctas_per_sm;
 
   // ---- device copy of the pattern ------------------------------------------
   std::vector<int32_t> rp(row_ptr, row_ptr + n + 1);
@@ -449,13 +504,15 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->batch = h->batch;
   info->ell_width = h->W;
   info->format = h->fmt == FMT_ELL ? BSOLVE_FMT_ELL : BSOLVE_FMT_CSR;
-  info->placement = h->place == PLACE_SMEM ? BSOLVE_PLACE_SMEM : BSOLVE_PLACE_STREAM;
+  info->placement = h->place == PLACE_SMEM ? BSOLVE_PLACE_SMEM
+                    : h->place == PLACE_REGS ? BSOLVE_PLACE_REGS : BSOLVE_PLACE_STREAM;
   info->block_threads = h->nt;
   info->rows_per_thread = h->r;
   info->smem_bytes = h->smem_bytes;
   info->ctas_per_sm = h->ctas_per_sm;
   info->num_sms = h->num_sms;
-  info->grid = h->batch;
+  info->grid = h->place == PLACE_REGS ? (int)std::min<long long>(h->grid_persist, h->batch)
+                                      : h->batch;
   info->kl = h->kl;
   info->ku = h->ku;
   info->device = h->device;
@@ -510,7 +567,14 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   P.n_pad = h->n_pad;
   P.guard = h->guard;
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
-  h->var->fn<<<count, h->nt, h->smem_bytes, stream>>>(P);
+  const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
+                         reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
+  if (h->place == PLACE_REGS && aligned) {
+    const int grid = (int)std::min<long long>(h->grid_persist, count);
+    h->pvar->fn<<<grid, h->nt, h->smem_bytes, stream>>>(P, h->d_ctr);
+  } else {
+    h->var->fn<<<count, h->nt, h->smem_bytes_fallback, stream>>>(P);
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));
   return BSOLVE_OK;

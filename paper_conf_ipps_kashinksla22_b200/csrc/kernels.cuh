@@ -30,7 +30,7 @@ namespace bsolve {
 // in every row r, the entry of column r + d_k (the host detects this for
 // stencil patterns): the gather address is row + d_k with d_k uniform.
 enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
-enum { PLACE_SMEM = 1, PLACE_STREAM = 2 };
+enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
 constexpr int kMaxW = 16;
@@ -65,6 +65,9 @@ __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
 }
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
@@ -215,6 +218,196 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
 }
 
 // ------------------------------------------------------------ the solver --
+// Algorithm 1 for ONE system, shared by both kernels.
+//   on entry: x = x0 (or 0), r = b, d = Jacobi diagonal, act = row < n;
+//   spmv(own, y): y = A g for this thread's rows, where g was published to
+//                 the gather body sg (and a barrier passed); own[j] = g[row].
+//   bv: b in registers (B_IN_REGS) for the true residual, else re-read bsys.
+// Writes x, iters, resnorm, status of system `sys`.  Every path executes at
+// least one block_sum (one barrier) after entry.
+template <int R, int NT, bool B_IN_REGS, class SpMV>
+__device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sys, double (&x)[R],
+                                              double (&r)[R], const double (&d)[R],
+                                              const bool (&act)[R], const double (&bv)[R],
+                                              double *sg, double *sred, int &buf, SpMV &&spmv) {
+  constexpr int NWARP = NT / 32;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int n = P.n;
+  const double *bsys = P.b + sys * n;
+  double rh[R], p[R], v[R];
+
+  // ---- a3: r = b - A x0 ; r^ = r ; ||b|| --------------------------------
+  double red3[2] = {0.0, 0.0};
+#pragma unroll
+  for (int j = 0; j < R; ++j) red3[0] += r[j] * r[j];  // b.b
+  if (P.x0) {
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (act[j]) sg[tid + j * NT] = x[j];
+    __syncthreads();
+    double q[R];
+    spmv(x, q);
+#pragma unroll
+    for (int j = 0; j < R; ++j) r[j] = r[j] - q[j];
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    rh[j] = r[j];
+    p[j] = 0.0;
+    v[j] = 0.0;
+    red3[1] += r[j] * r[j];
+  }
+  block_sum<2, NWARP>(red3, sred, buf, lane, warp);
+  const double bnorm = sqrt(red3[0]);
+  const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
+  double rnorm = sqrt(red3[1]);
+  double rho = red3[1];  // r^ . r with r^ = r
+
+  double *xout = P.x + sys * n;
+  if (P.stop == STOP_REL_B && bnorm == 0.0) {
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (act[j]) xout[tid + j * NT] = 0.0;
+    if (tid == 0) {
+      P.iters[sys] = 0;
+      P.resnorm[sys] = 0.0;
+      if (P.status) P.status[sys] = SYS_CONVERGED;
+    }
+    return;
+  }
+
+  auto true_residual = [&](double (&q)[R]) -> double {
+    // publish x, q = b - A x, returns ||q||_2 (one more barrier)
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (act[j]) sg[tid + j * NT] = x[j];
+    __syncthreads();
+    double tr[1] = {0.0};
+    spmv(x, q);
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const double bj = B_IN_REGS ? bv[j] : (act[j] ? __ldg(bsys + tid + j * NT) : 0.0);
+      q[j] = act[j] ? bj - q[j] : 0.0;
+      tr[0] += q[j] * q[j];
+    }
+    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
+    return tr[0];
+  };
+
+  int it = 0, st = -1, exit_kind = 0;
+  double rho_old = 1.0, alpha = 1.0, omega = 1.0;
+  double final_res = -1.0;
+  for (;;) {
+    exit_kind = 0;
+    while (it < P.maxiter) {
+      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1 (P:767)
+      if (bad(rho)) { st = SYS_BREAKDOWN; break; }
+      const double beta = (rho / rho_old) * (alpha / omega);  // R2
+      // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
+      double ph[R];
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        p[j] = r[j] + beta * (p[j] - omega * v[j]);
+        ph[j] = d[j] * p[j];
+        if (act[j]) sg[tid + j * NT] = ph[j];
+      }
+      __syncthreads();
+      // a6: v = A p^
+      spmv(ph, v);
+      ++it;
+      // a7: alpha = rho / (r^ . v)
+      double rv[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
+      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
+      if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
+      alpha = rho / rv[0];                                 // R3
+      // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
+      // barrier in the reduction above separates them)
+      double s[R], sh[R], ss[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        s[j] = r[j] - alpha * v[j];
+        ss[0] += s[j] * s[j];
+        sh[j] = d[j] * s[j];
+        if (act[j]) sg[tid + j * NT] = sh[j];
+      }
+      block_sum<1, NWARP>(ss, sred, buf, lane, warp);      // also publishes s^
+      if (sqrt(ss[0]) < tau) {                             // stop test 2 (P:782-786)
+#pragma unroll
+        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
+        exit_kind = 2;
+        break;
+      }
+      // a9: t = A s^
+      double t[R];
+      spmv(sh, t);
+      // a10: omega = (t.s)/(t.t); x, r updates
+      double ts[2] = {0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        ts[0] += t[j] * s[j];
+        ts[1] += t[j] * t[j];
+      }
+      block_sum<2, NWARP>(ts, sred, buf, lane, warp);
+      if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
+      omega = ts[0] / ts[1];
+      if (bad(omega)) { st = SYS_BREAKDOWN; break; }
+      double rr[2] = {0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
+        r[j] = s[j] - omega * t[j];
+        rr[0] += r[j] * r[j];
+        rr[1] += rh[j] * r[j];
+      }
+      rho_old = rho;
+      // next iteration's ||r|| and rho = r^ . r in the same single barrier
+      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
+      rnorm = sqrt(rr[0]);
+      rho = rr[1];
+    }
+    if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
+    // ---- a11: true-residual guard (DESIGN R4) -----------------------------
+    // (gather buffer is free: its last readers passed a barrier already)
+    double q[R];
+    const double tr2 = true_residual(q);
+    final_res = sqrt(tr2);
+    if (final_res < tau || it >= P.maxiter) break;
+    // restart from the true residual, keep counting iterations
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      r[j] = q[j];
+      rh[j] = q[j];
+      p[j] = 0.0;
+      v[j] = 0.0;
+    }
+    rho_old = alpha = omega = 1.0;
+    rnorm = final_res;
+    rho = tr2;
+    final_res = -1.0;
+  }
+
+  if (final_res < 0.0) {
+    // final TRUE residual ||b - A x|| (always reported, R4)
+    __syncthreads();  // previous gather readers done before overwriting
+    double q[R];
+    final_res = sqrt(true_residual(q));
+  }
+  if (st != SYS_BREAKDOWN) {
+    if (P.trc) st = final_res < tau ? SYS_CONVERGED : SYS_MAXITER;
+    else st = exit_kind != 0 ? SYS_CONVERGED : SYS_MAXITER;
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j)
+    if (act[j]) xout[tid + j * NT] = x[j];
+  if (tid == 0) {
+    P.iters[sys] = it;
+    P.resnorm[sys] = final_res;
+    if (P.status) P.status[sys] = static_cast<int8_t>(st);
+  }
+}
+
 // Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
 //   [values: smem_vals doubles (PLACE_SMEM only)]
 //   [gather: guard | n_pad body | guard doubles]
@@ -230,7 +423,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 4 * NWARP);
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x;
   const int n = P.n;
   const long long sys = blockIdx.x;
   const double *gval = P.values + sys * P.sys_stride;
@@ -269,7 +462,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
 
   // ---- pattern + right-hand side + initial guess into registers ----------
   RowMeta<FMT, WB, R> m;
-  double x[R], r[R], rh[R], p[R], v[R], d[R];
+  double x[R], r[R], d[R];
   const double *bsys = P.b + sys * n;
   int dsl[R];
 #pragma unroll
@@ -319,178 +512,159 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   }
 
   int buf = 0;
-  // ---- a3: r = b - A x0 ; r^ = r ; ||b|| --------------------------------
-  double red3[2] = {0.0, 0.0};
-#pragma unroll
-  for (int j = 0; j < R; ++j) red3[0] += r[j] * r[j];  // b.b
-  if (P.x0) {
-#pragma unroll
-    for (int j = 0; j < R; ++j)
-      if (m.act[j]) sg[tid + j * NT] = x[j];
-    __syncthreads();
-    double q[R];
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
-#pragma unroll
-    for (int j = 0; j < R; ++j) r[j] = r[j] - q[j];
-  }
+  bicgstab_core<R, NT, false>(
+      P, sys, x, r, d, m.act, r, sg, sred, buf, [&](const double(&own)[R], double(&y)[R]) {
+        spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, own, y);
+      });
+}
+
+// ------------------------------------- persistent, register-resident values --
+// PLACE_REGS (DESIGN.md "Kernels" 7): one CTA per SM (up to 255 registers per
+// thread) loops over systems claimed from a device work counter.  The
+// system's values, b and x0 arrive in SMEM by TMA; each thread moves ITS rows'
+// values (all W slots) and b into registers, then thread 0 immediately
+// claims the next system and re-arms the same SMEM buffers with TMA, so the
+// HBM load of system k+1 overlaps the iterations of system k.  Every SpMV
+// then reads only the gathered operands from SMEM: the matrix never touches
+// the shared-memory data pipe again.
+//   SMEM: [values: smem_vals][b: n_pad][x0: n_pad][gather: guard|n_pad|guard]
+//         [reduction scratch: 4*NWARP][mbarrier][next-system slot]
+// The counter (ctr[0]) and the finished-CTA count (ctr[1]) reset themselves
+// when the last CTA leaves, so consecutive launches on one stream need no
+// host-side reset.
+template <int FMT, int WB, bool EXACT, int R, int NT>
+__global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolveParams P,
+                                                                 unsigned long long *ctr) {
+  static_assert(FMT == FMT_ELL || FMT == FMT_DIA, "register-resident values need ELL/DIA");
+  constexpr int NWARP = NT / 32;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sb = sval + P.smem_vals;
+  double *sx0 = sb + P.n_pad;
+  double *sgf = sx0 + P.n_pad;
+  double *sg = sgf + P.guard;
+  double *sred = sgf + P.n_pad + 2 * P.guard;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 4 * NWARP);
+  volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+
+  const int tid = threadIdx.x;
+  const int n = P.n;
+  const long long batch = P.batch;
+  const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
+  const uint32_t nbytes = static_cast<uint32_t>(n * 8);
+
+  auto issue = [&](long long s) {  // thread 0: TMA of system s into the staging buffers
+    mbar_arrive_expect_tx(mbar, vbytes + nbytes + (P.x0 ? nbytes : 0u));
+    const unsigned char *src = reinterpret_cast<const unsigned char *>(P.values + s * P.sys_stride);
+    constexpr uint32_t CH = 32768;
+    for (uint32_t off = 0; off < vbytes; off += CH)
+      tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off, src + off,
+                   vbytes - off < CH ? vbytes - off : CH, mbar);
+    tma_bulk_g2s(sb, P.b + s * n, nbytes, mbar);
+    if (P.x0) tma_bulk_g2s(sx0, P.x0 + s * n, nbytes, mbar);
+  };
+
+  // pattern registers (once per CTA) and gather guards
+  RowMeta<FMT, WB, R> m;
 #pragma unroll
   for (int j = 0; j < R; ++j) {
-    rh[j] = r[j];
-    p[j] = 0.0;
-    v[j] = 0.0;
-    red3[1] += r[j] * r[j];
-  }
-  block_sum<2, NWARP>(red3, sred, buf, lane, warp);
-  const double bnorm = sqrt(red3[0]);
-  const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
-  double rnorm = sqrt(red3[1]);
-  double rho = red3[1];  // r^ . r with r^ = r
-
-  double *xout = P.x + sys * n;
-  if (P.stop == STOP_REL_B && bnorm == 0.0) {
+    const int row = tid + j * NT;
+    m.act[j] = row < n;
+    m.vbase[j] = row < n ? row : n - 1;
+    m.vlen[j] = 0;
+    m.a0[j] = 0.0;
 #pragma unroll
-    for (int j = 0; j < R; ++j)
-      if (m.act[j]) xout[tid + j * NT] = 0.0;
-    if (tid == 0) {
-      P.iters[sys] = 0;
-      P.resnorm[sys] = 0.0;
-      if (P.status) P.status[sys] = SYS_CONVERGED;
-    }
-    return;
-  }
-
-  int it = 0, st = -1, exit_kind = 0;
-  double rho_old = 1.0, alpha = 1.0, omega = 1.0;
-  double final_res = -1.0;
-  for (;;) {
-    exit_kind = 0;
-    while (it < P.maxiter) {
-      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1 (P:767)
-      if (bad(rho)) { st = SYS_BREAKDOWN; break; }
-      const double beta = (rho / rho_old) * (alpha / omega);  // R2
-      // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
-      double ph[R];
+    for (int k = 0; k < (WB + 1) / 2; ++k) m.cpk[j][k] = 0u;
+    if (FMT == FMT_ELL && m.act[j]) {
 #pragma unroll
-      for (int j = 0; j < R; ++j) {
-        p[j] = r[j] + beta * (p[j] - omega * v[j]);
-        ph[j] = d[j] * p[j];
-        if (m.act[j]) sg[tid + j * NT] = ph[j];
+      for (int k = 0; k < WB; ++k) {
+        if (EXACT || k < P.W) {
+          const uint32_t off = static_cast<uint32_t>(__ldg(P.ell_col + (size_t)k * n + row)) * 8u;
+          m.cpk[j][k >> 1] |= (k & 1) ? (off << 16) : off;
+        }
       }
-      __syncthreads();
-      // a6: v = A p^
-      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, ph, v);
-      ++it;
-      // a7: alpha = rho / (r^ . v)
-      double rv[1] = {0.0};
-#pragma unroll
-      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
-      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
-      if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
-      alpha = rho / rv[0];                                 // R3
-      // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
-      // barrier in the reduction above separates them)
-      double s[R], sh[R], ss[1] = {0.0};
-#pragma unroll
-      for (int j = 0; j < R; ++j) {
-        s[j] = r[j] - alpha * v[j];
-        ss[0] += s[j] * s[j];
-        sh[j] = d[j] * s[j];
-        if (m.act[j]) sg[tid + j * NT] = sh[j];
-      }
-      block_sum<1, NWARP>(ss, sred, buf, lane, warp);      // also publishes s^
-      if (sqrt(ss[0]) < tau) {                             // stop test 2 (P:782-786)
-#pragma unroll
-        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
-        exit_kind = 2;
-        break;
-      }
-      // a9: t = A s^
-      double t[R];
-      spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, sh, t);
-      // a10: omega = (t.s)/(t.t); x, r updates
-      double ts[2] = {0.0, 0.0};
-#pragma unroll
-      for (int j = 0; j < R; ++j) {
-        ts[0] += t[j] * s[j];
-        ts[1] += t[j] * t[j];
-      }
-      block_sum<2, NWARP>(ts, sred, buf, lane, warp);
-      if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
-      omega = ts[0] / ts[1];
-      if (bad(omega)) { st = SYS_BREAKDOWN; break; }
-      double rr[2] = {0.0, 0.0};
-#pragma unroll
-      for (int j = 0; j < R; ++j) {
-        x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
-        r[j] = s[j] - omega * t[j];
-        rr[0] += r[j] * r[j];
-        rr[1] += rh[j] * r[j];
-      }
-      rho_old = rho;
-      // next iteration's ||r|| and rho = r^ . r in the same single barrier
-      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
-      rnorm = sqrt(rr[0]);
-      rho = rr[1];
     }
-    if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
-    // ---- a11: true-residual guard (DESIGN R4) -----------------------------
-    // (gather buffer is free: its last readers passed a barrier already)
-#pragma unroll
-    for (int j = 0; j < R; ++j)
-      if (m.act[j]) sg[tid + j * NT] = x[j];
-    __syncthreads();
-    double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
-      tr[0] += q[j] * q[j];
-    }
-    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
-    final_res = sqrt(tr[0]);
-    if (final_res < tau || it >= P.maxiter) break;
-    // restart from the true residual, keep counting iterations
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      r[j] = q[j];
-      rh[j] = q[j];
-      p[j] = 0.0;
-      v[j] = 0.0;
-    }
-    rho_old = alpha = omega = 1.0;
-    rnorm = final_res;
-    rho = tr[0];
-    final_res = -1.0;
   }
-
-  if (final_res < 0.0) {
-    // final TRUE residual ||b - A x|| (always reported, R4)
-    __syncthreads();  // previous gather readers done before overwriting
-#pragma unroll
-    for (int j = 0; j < R; ++j)
-      if (m.act[j]) sg[tid + j * NT] = x[j];
-    __syncthreads();
-    double q[R], tr[1] = {0.0};
-    spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, x, q);
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      q[j] = m.act[j] ? __ldg(bsys + tid + j * NT) - q[j] : 0.0;
-      tr[0] += q[j] * q[j];
-    }
-    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
-    final_res = sqrt(tr[0]);
+  for (int i = tid; i < P.guard; i += NT) {
+    sgf[i] = 0.0;
+    sg[P.n_pad + i] = 0.0;
   }
-  if (st != SYS_BREAKDOWN) {
-    if (P.trc) st = final_res < tau ? SYS_CONVERGED : SYS_MAXITER;
-    else st = exit_kind != 0 ? SYS_CONVERGED : SYS_MAXITER;
-  }
-#pragma unroll
-  for (int j = 0; j < R; ++j)
-    if (m.act[j]) xout[tid + j * NT] = x[j];
   if (tid == 0) {
-    P.iters[sys] = it;
-    P.resnorm[sys] = final_res;
-    if (P.status) P.status[sys] = static_cast<int8_t>(st);
+    mbar_init(mbar, 1);
+    fence_mbar_init();
+    const long long first = static_cast<long long>(atomicAdd(ctr, 1ull));
+    *s_next = first;
+    if (first < batch) issue(first);
+  }
+  __syncthreads();
+  long long cur = *s_next;
+  uint32_t phase = 0;
+  int buf = 0;
+  while (cur < batch) {
+    mbar_wait_parity(mbar, phase);
+    phase ^= 1u;
+    // ---- registers <- staging buffers -------------------------------------
+    double val[R][WB], x[R], r[R], d[R], bv[R];
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+#pragma unroll
+      for (int k = 0; k < WB; ++k)
+        val[j][k] = (EXACT || k < P.W) ? sval[k * n + m.vbase[j]] : 0.0;
+      const double a = m.act[j] ? val[j][0] : 0.0;  // slot 0 = diagonal
+      d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+      bv[j] = m.act[j] ? sb[m.vbase[j]] : 0.0;
+      r[j] = bv[j];
+      x[j] = (P.x0 && m.act[j]) ? sx0[m.vbase[j]] : 0.0;
+    }
+    __syncthreads();  // every thread is done with the staging buffers
+    if (tid == 0) {
+      const long long nxt = static_cast<long long>(atomicAdd(ctr, 1ull));
+      *s_next = nxt;
+      if (nxt < batch) {
+        fence_proxy_async_smem();  // generic reads above before the async-proxy writes
+        issue(nxt);
+      }
+    }
+    const int wrow0 = tid & ~31;
+    bicgstab_core<R, NT, true>(
+        P, cur, x, r, d, m.act, bv, sg, sred, buf,
+        [&](const double(&own)[R], double(&y)[R]) {
+#pragma unroll
+          for (int j = 0; j < R; ++j) {
+            double acc = 0.0;
+            if (wrow0 + j * NT < n) {
+              acc = val[j][0] * own[j];
+              const unsigned char *grow = gb + m.vbase[j] * 8;
+#pragma unroll
+              for (int k = 1; k < WB; ++k) {
+                if (EXACT || k < P.W) {
+                  double g;
+                  if (FMT == FMT_DIA) {
+                    g = *reinterpret_cast<const double *>(grow + P.doff[k]);
+                  } else {
+                    const uint32_t off = (k & 1) ? field16<16>(m.cpk[j][k >> 1])
+                                                 : field16<0>(m.cpk[j][k >> 1]);
+                    g = *reinterpret_cast<const double *>(gb + off);
+                  }
+                  acc = fma(val[j][k], g, acc);
+                }
+              }
+            }
+            y[j] = m.act[j] ? acc : 0.0;
+          }
+        });
+    cur = *s_next;  // written before the core's first barrier
+  }
+  // ---- self-resetting work counter ------------------------------------------
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    const unsigned long long done = atomicAdd(ctr + 1, 1ull);
+    if (done == gridDim.x - 1) {
+      atomicExch(ctr, 0ull);
+      atomicExch(ctr + 1, 0ull);
+    }
   }
 }
 

@@ -30,7 +30,8 @@ def test_config0_ion_electron_pair(fmt):
     B = X.make_batch(0, 2)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt)
-    assert g["info"]["placement"] == 1  # SMEM staged
+    # ELL auto-plans the persistent register-resident kernel, CSR the SMEM one
+    assert g["info"]["placement"] == (3 if fmt == "ell" else 1)
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
 
 
@@ -55,13 +56,13 @@ def test_config1_zero_and_picard_warm_start():
 
 
 # ---------------------------------------------------- formats/placements --
-@pytest.mark.parametrize("fmt,placement", [("ell", "smem"), ("ell", "stream"),
+@pytest.mark.parametrize("fmt,placement", [("ell", "smem"), ("ell", "stream"), ("ell", "regs"),
                                            ("csr", "smem"), ("csr", "stream")])
 def test_formats_and_placements(fmt, placement):
     B = X.make_batch(100, 64)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt, placement=placement)
-    want = 1 if placement == "smem" else 2
+    want = {"smem": 1, "stream": 2, "regs": 3}[placement]
     assert g["info"]["placement"] == want
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
 
@@ -287,3 +288,50 @@ def test_forced_smem_too_large_unsupported():
     with pytest.raises(BsolveError) as e:
         Solver(pat.row_ptr, pat.col_idx, 1, placement="smem")
     assert e.value.code in (-3,)
+
+
+# ------------------------------------------- persistent register kernel --
+def test_regs_repeated_launches_counter_reset_and_fallback():
+    """PLACE_REGS: the self-resetting work counter makes back-to-back launches
+    on one handle identical; batches smaller and larger than the persistent
+    grid; misaligned buffers take the per-system-CTA fallback, same results."""
+    for batch in (3, 148, 1000):
+        B = X.make_batch(0, batch)
+        p = B.pattern
+        S = Solver(p.row_ptr, p.col_idx, batch, placement="regs")
+        assert S.info["placement"] == 3
+        v = to_dev(S.ell_values(B.values))
+        b = to_dev(B.b)
+        outs = [S.run(v, b) for _ in range(3)]
+        torch.cuda.synchronize()
+        for o in outs[1:]:
+            for a, c in zip(outs[0], o):
+                assert torch.equal(a, c)
+        g = dict(x=outs[0][0].cpu().numpy(), iters=outs[0][1].cpu().numpy(),
+                 resnorm=outs[0][2].cpu().numpy(), status=outs[0][3].cpu().numpy().astype(np.int32))
+        compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+    # misaligned values/b (8-byte offset): fallback kernel, same per-system results
+    vbig = torch.empty(v.numel() + 1, dtype=torch.float64, device="cuda")
+    vbig[1:] = v.reshape(-1)
+    bbig = torch.empty(b.numel() + 1, dtype=torch.float64, device="cuda")
+    bbig[1:] = b.reshape(-1)
+    xf, itf, rf, sf = S.run(vbig[1:].view_as(v), bbig[1:].view_as(b))
+    torch.cuda.synchronize()
+    assert np.array_equal(itf.cpu().numpy(), g["iters"])
+    np.testing.assert_allclose(xf.cpu().numpy(), g["x"], rtol=0, atol=1e-12)
+
+
+def test_regs_warm_start_x0_alias():
+    """x0 staged by TMA in the persistent kernel; x may alias x0."""
+    B = X.make_batch(0, 300, picard=1)
+    p = B.pattern
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-6)
+    S = Solver(p.row_ptr, p.col_idx, 300)
+    v = to_dev(S.ell_values(B.values))
+    xa = to_dev(x0)
+    x, it, res, st = S.run(v, to_dev(B.b), x0=xa, out=(xa, *S.alloc_outputs()[1:]))
+    torch.cuda.synchronize()
+    g = dict(x=xa.cpu().numpy(), iters=it.cpu().numpy(), resnorm=res.cpu().numpy(),
+             status=st.cpu().numpy().astype(np.int32))
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
