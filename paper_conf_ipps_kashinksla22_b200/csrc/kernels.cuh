@@ -95,51 +95,84 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity)
 
 __device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
 
-// Block-wide sum of K in {1, 2} doubles with ONE barrier.  Every SHFL costs
-// one data-pipe wavefront on B200, like an LDS, so:
-//  * inside a warp: xor butterfly; for K = 2 the first step is a recursive
-//    halving exchange (lanes with bit 4 clear keep value 0, the others value
-//    1), so two sums cost the shuffles of one plus one step;
-//  * lane 0 (value 0) / lane 16 (value 1) publish the warp partial;
-//  * after the barrier every thread reads the NWARP partials of each value
-//    with broadcast 16-byte loads and adds them in warp order.
-// All threads obtain bitwise-identical sums in a fixed order (uniform control
-// flow, results independent of batch slicing).  `buf` alternates between
-// two scratch halves so the next reduction never overwrites partials that a
-// slow warp is still reading.
+// Pairwise (tree) sum of N doubles, fixed order: latency log2(N) adds.
+template <int N>
+__device__ __forceinline__ double tree_sum(const double *a) {
+  if constexpr (N == 1) {
+    return a[0];
+  } else {
+    return tree_sum<N / 2>(a) + tree_sum<N - N / 2>(a + N / 2);
+  }
+}
+
+// Block-wide sum of K <= 4 doubles with ONE barrier.  On B200 every SHFL.32
+// costs one shared-memory data-pipe wavefront (like an LDS) and ~20+ cycles
+// of latency, so:
+//  * inside a warp, recursive halving: with K > 1 the first steps exchange
+//    only the half of the values a lane is NOT responsible for (lane bit 4,
+//    then bit 3, select the value), the remaining steps are an xor butterfly
+//    on one value; K values cost about the shuffles of one;
+//  * lane 8q publishes the warp partial of value q (K = 1: lane 0);
+//  * after the barrier every thread loads the NWARP partials of each value
+//    (broadcast 16-byte loads, all values in flight together) and adds them
+//    as a pairwise tree.
+// After the butterfly all lanes that hold a value hold the same bits (each
+// step adds the same two operands in both partner lanes; fp addition is
+// commutative), and the tree has a fixed order, so every thread obtains
+// bitwise-identical sums: uniform control flow, results independent of the
+// batch slicing.  `buf` alternates between two scratch halves so the next
+// reduction never overwrites partials that a slow warp is still reading.
 template <int K, int NWARP>
 __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf, int lane,
                                           int warp) {
-  static_assert(K == 1 || K == 2, "block_sum supports 1 or 2 values");
-  static_assert(NWARP % 2 == 0, "NWARP must be even");
+  static_assert(K >= 1 && K <= 4, "block_sum supports 1..4 values");
+  static_assert(NWARP % 2 == 0 && NWARP <= 32, "NWARP must be even");
   double keep;
-  if (K == 2) {
-    const bool hi = lane & 16;
-    const double send = hi ? v[0] : v[K - 1];
-    keep = hi ? v[K - 1] : v[0];
-    keep += __shfl_xor_sync(0xffffffffu, send, 16);
-#pragma unroll
-    for (int o = 8; o > 0; o >>= 1) keep += __shfl_xor_sync(0xffffffffu, keep, o);
-  } else {
+  int first_step;
+  if constexpr (K == 1) {
     keep = v[0];
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) keep += __shfl_xor_sync(0xffffffffu, keep, o);
+    first_step = 16;
+  } else if constexpr (K == 2) {
+    const bool hi = lane & 16;
+    keep = (hi ? v[1] : v[0]) + __shfl_xor_sync(0xffffffffu, hi ? v[0] : v[1], 16);
+    first_step = 8;
+  } else {
+    // K = 3 or 4: pairs (v0, v1) and (v2, v3) by lane bit 4, then by bit 3
+    const double v3 = (K == 4) ? v[K - 1] : 0.0;
+    const bool hi4 = lane & 16, hi3 = lane & 8;
+    const double k0 = (hi4 ? v[2] : v[0]) + __shfl_xor_sync(0xffffffffu, hi4 ? v[0] : v[2], 16);
+    const double k1 = (hi4 ? v3 : v[1]) + __shfl_xor_sync(0xffffffffu, hi4 ? v[1] : v3, 16);
+    keep = (hi3 ? k1 : k0) + __shfl_xor_sync(0xffffffffu, hi3 ? k0 : k1, 8);
+    first_step = 4;
   }
-  double *S = sred + buf * (2 * NWARP);
-  if ((lane & 15) == 0 && (K == 2 || lane == 0)) S[(lane >> 4) * NWARP + warp] = keep;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1)
+    if (o <= first_step) keep += __shfl_xor_sync(0xffffffffu, keep, o);
+  // value index held by this lane: K = 1: all lanes value 0; K = 2: bit 4;
+  // K >= 3: bit 4 selects the pair (v0,v1) / (v2,v3), bit 3 the member
+  double *S = sred + buf * (4 * NWARP);
+  if constexpr (K == 1) {
+    if (lane == 0) S[warp] = keep;
+  } else if constexpr (K == 2) {
+    if ((lane & 15) == 0) S[(lane >> 4) * NWARP + warp] = keep;
+  } else {
+    const int q = ((lane >> 4) & 1) * 2 + ((lane >> 3) & 1);  // 0: v0, 1: v1, 2: v2, 3: v3
+    if ((lane & 7) == 0 && q < K) S[q * NWARP + warp] = keep;
+  }
   __syncthreads();
+  double part[K][NWARP];
 #pragma unroll
   for (int k = 0; k < K; ++k) {
     const double2 *S2 = reinterpret_cast<const double2 *>(S + k * NWARP);
-    double a = 0.0;
 #pragma unroll
     for (int w = 0; w < NWARP / 2; ++w) {
       const double2 q = S2[w];
-      a += q.x;
-      a += q.y;
+      part[k][2 * w] = q.x;
+      part[k][2 * w + 1] = q.y;
     }
-    v[k] = a;
   }
+#pragma unroll
+  for (int k = 0; k < K; ++k) v[k] = tree_sum<NWARP>(part[k]);
   buf ^= 1;
 }
 
@@ -324,32 +357,34 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       alpha = rho / rv[0];                                 // R3
       // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
       // barrier in the reduction above separates them)
-      double s[R], sh[R], ss[1] = {0.0};
+      double s[R], sh[R];
+      double ts[3] = {0.0, 0.0, 0.0};  // t.s, t.t, s.s
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         s[j] = r[j] - alpha * v[j];
-        ss[0] += s[j] * s[j];
+        ts[2] += s[j] * s[j];
         sh[j] = d[j] * s[j];
         if (act[j]) sg[tid + j * NT] = sh[j];
       }
-      block_sum<1, NWARP>(ss, sred, buf, lane, warp);      // also publishes s^
-      if (sqrt(ss[0]) < tau) {                             // stop test 2
-#pragma unroll
-        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
-        exit_kind = 2;
-        break;
-      }
-      // a9: t = A s^
+      __syncthreads();  // publish s^
+      // a9: t = A s^.  ||s|| for stop test 2 is reduced together with t.s and
+      // t.t (one reduction round fewer per iteration); when stop test 2 fires
+      // this SpMV was speculative and t is discarded -- x, iteration count and
+      // exit are exactly those of Alg. 1
       double t[R];
       spmv(sh, t);
-      // a10: omega = (t.s)/(t.t); x, r updates
-      double ts[2] = {0.0, 0.0};
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         ts[0] += t[j] * s[j];
         ts[1] += t[j] * t[j];
       }
-      block_sum<2, NWARP>(ts, sred, buf, lane, warp);
+      block_sum<3, NWARP>(ts, sred, buf, lane, warp);
+      if (sqrt(ts[2]) < tau) {                             // stop test 2
+#pragma unroll
+        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
+        exit_kind = 2;
+        break;
+      }
       if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
       omega = ts[0] / ts[1];
       if (bad(omega)) { st = SYS_BREAKDOWN; break; }
@@ -411,7 +446,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
 // Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
 //   [values: smem_vals doubles (PLACE_SMEM only)]
 //   [gather: guard | n_pad body | guard doubles]
-//   [reduction scratch: 2 * 2 * NWARP doubles] [mbarrier: 8 B]
+//   [reduction scratch: 2 * 4 * NWARP doubles] [mbarrier: 8 B]
 template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB>
 __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
@@ -420,7 +455,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   double *sgf = sval + (PLACE == PLACE_SMEM ? P.smem_vals : 0);  // gather incl. guards
   double *sg = sgf + P.guard;                                     // gather body
   double *sred = sgf + P.n_pad + 2 * P.guard;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 4 * NWARP);
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 8 * NWARP);
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
   const int tid = threadIdx.x;
@@ -528,7 +563,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
 // then reads only the gathered operands from SMEM: the matrix never touches
 // the shared-memory data pipe again.
 //   SMEM: [values: smem_vals][b: n_pad][x0: n_pad][gather: guard|n_pad|guard]
-//         [reduction scratch: 4*NWARP][mbarrier][next-system slot]
+//         [reduction scratch: 8*NWARP][mbarrier][next-system slot]
 // The counter (ctr[0]) and the finished-CTA count (ctr[1]) reset themselves
 // when the last CTA leaves, so consecutive launches on one stream need no
 // host-side reset.
@@ -544,7 +579,7 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
   double *sgf = sx0 + P.n_pad;
   double *sg = sgf + P.guard;
   double *sred = sgf + P.n_pad + 2 * P.guard;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 4 * NWARP);
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 8 * NWARP);
   volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
