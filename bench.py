@@ -47,7 +47,9 @@ def parse():
     ap.add_argument("--nx", type=int, default=32)
     ap.add_argument("--ny", type=int, default=31)
     ap.add_argument("--format", choices=["ell", "csr"], default="ell")
-    ap.add_argument("--placement", choices=["auto", "smem", "stream"], default="auto")
+    ap.add_argument("--placement", choices=["auto", "smem", "stream", "regs"], default="auto")
+    ap.add_argument("--block-threads", type=int, default=0)
+    ap.add_argument("--reg-slots", type=int, default=0)
     ap.add_argument("--tol", type=float, default=1e-10)
     ap.add_argument("--maxiter", type=int, default=1000)
     ap.add_argument("--seed", type=int, default=20220530)
@@ -290,7 +292,8 @@ def run_ours(args, rank, world, local_rank):
     pat, vals_h, b_h = make_inputs(g0, per_rank, args, pinned=True)
     n, nnz, W = pat.n, pat.nnz, pat.max_row_nnz
     S = Solver(pat.row_ptr, pat.col_idx, per_rank, format=args.format,
-               placement=args.placement, device=local_rank)
+               placement=args.placement, device=local_rank, block_threads=args.block_threads,
+               reg_slots=args.reg_slots)
     vals = vals_h.to(dev, non_blocking=False)
     b = b_h.to(dev)
     out = S.alloc_outputs()

@@ -70,8 +70,7 @@ enum {
 /* Where the matrix values live while a system iterates (PAPER.md:708-721,
  * 738-813: the paper's automatic shared-memory configuration). */
 enum {
-  BSOLVE_PLACE_AUTO = 0,   /* REGS if eligible, else SMEM if one system's
-                              values fit, else STREAM                         */
+  BSOLVE_PLACE_AUTO = 0,   /* SMEM if one system's values fit, else STREAM   */
   BSOLVE_PLACE_SMEM = 1,   /* staged once into shared memory by TMA bulk copy */
   BSOLVE_PLACE_STREAM = 2, /* re-read from global memory (L2/L1) every SpMV   */
   BSOLVE_PLACE_REGS = 3    /* persistent kernel, one CTA per SM: values staged by
@@ -103,7 +102,11 @@ typedef struct bsolve_options {
                               it is >= tau (R4); 0: trust the
                               recursive residual of Alg. 1  (default 1)       */
   int device;              /* CUDA device ordinal, -1 = current (default -1)  */
-  int block_threads;       /* threads per CTA, 0 = auto (default 0)          */
+  int block_threads;       /* threads per CTA: 0 = auto, 128, 256 or 512
+                              (default 0); 128 = 8 rows per thread (ELL) */
+  int reg_slots;           /* with block_threads = 128: off-diagonal ELL slots
+                              held in registers instead of SMEM, 0, 2 or 4
+                              (default 0)                                     */
 } bsolve_options;
 
 typedef struct bsolve_info {

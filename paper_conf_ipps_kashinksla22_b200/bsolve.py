@@ -36,7 +36,7 @@ class BsolveError(RuntimeError):
 class Options(C.Structure):
     _fields_ = [("format", C.c_int), ("placement", C.c_int), ("stop", C.c_int),
                 ("true_residual_check", C.c_int), ("device", C.c_int),
-                ("block_threads", C.c_int)]
+                ("block_threads", C.c_int), ("reg_slots", C.c_int)]
 
 
 class Info(C.Structure):
@@ -136,7 +136,7 @@ class Solver:
 
     def __init__(self, row_ptr, col_idx, batch: int, *, format: str = "ell",
                  placement: str = "auto", stop: str = "rel_b", true_residual_check: bool = True,
-                 device: int | None = None, block_threads: int = 0):
+                 device: int | None = None, block_threads: int = 0, reg_slots: int = 0):
         L = lib()
         rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
         ci = np.ascontiguousarray(col_idx, dtype=np.int32)
@@ -150,6 +150,7 @@ class Solver:
         opt.true_residual_check = int(bool(true_residual_check))
         opt.device = -1 if device is None else int(device)
         opt.block_threads = int(block_threads)
+        opt.reg_slots = int(reg_slots)
         h = _P()
         check(L.bsolve_create(C.byref(h), self.n, self.batch, rp.ctypes.data, ci.ctypes.data,
                               C.byref(opt)))

@@ -53,11 +53,14 @@ struct Variant {
   int fmt, place, wb;
   bool exact;
   int r, nt;
+  int kreg;  // off-diagonal ELL slots held in registers (hybrid variants)
   solve_fn fn;
 };
 
 #define V_(F, PL, WB, EX, R, NT, MB) \
-  {F, PL, WB, EX, R, NT, (solve_fn)bicgstab_kernel<F, PL, WB, EX, R, NT, MB>}
+  {F, PL, WB, EX, R, NT, 0, (solve_fn)bicgstab_kernel<F, PL, WB, EX, R, NT, MB>}
+#define VK_(F, R, NT, MB, KR) \
+  {F, PLACE_SMEM, 9, true, R, NT, KR, (solve_fn)bicgstab_kernel<F, PLACE_SMEM, 9, true, R, NT, MB, KR>}
 #define V_FP(WB, EX, R, NT, MB)                                                         \
   V_(FMT_ELL, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, EX, R, NT, MB), \
       V_(FMT_DIA, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_DIA, PLACE_STREAM, WB, EX, R, NT, MB), \
@@ -69,6 +72,8 @@ static const Variant kVariants[] = {
     V_FP(9, true, 1, 256, 2),   V_FP(9, true, 2, 256, 2),   V_FP(9, true, 4, 256, 2),
     V_FP(9, true, 4, 512, 1),   V_FP(16, false, 1, 256, 2), V_FP(16, false, 2, 256, 2),
     V_FP(16, false, 4, 256, 2), V_FP(16, false, 4, 512, 1),
+    // experimental hybrid: 128 threads x 8 rows, 2 CTAs/SM, slots 1..KREG in registers
+    VK_(FMT_DIA, 8, 128, 2, 0), VK_(FMT_DIA, 8, 128, 2, 2), VK_(FMT_DIA, 8, 128, 2, 4),
 };
 
 // Persistent register-resident variants (PLACE_REGS): ELL/DIA, W = 9.
@@ -86,10 +91,11 @@ static const PVariant *find_pvariant(int fmt, int r) {
   return nullptr;
 }
 
-static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt) {
+static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt,
+                                   int kreg = 0) {
   for (const Variant &v : kVariants)
     if (v.fmt == fmt && v.place == place && v.wb == wb && v.exact == exact && v.r == r &&
-        v.nt == nt)
+        v.nt == nt && v.kreg == kreg)
       return &v;
   return nullptr;
 }
@@ -129,6 +135,7 @@ extern "C" void bsolve_default_options(bsolve_options *o) {
   o->true_residual_check = 1;
   o->device = -1;
   o->block_threads = 0;
+  o->reg_slots = 0;
 }
 
 static void free_plan(bsolve_plan *h) {
@@ -297,9 +304,12 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     return fail(BSOLVE_ERR_INVALID, "bad placement %d", opt.placement);
   if (opt.stop != BSOLVE_STOP_REL_B && opt.stop != BSOLVE_STOP_ABS)
     return fail(BSOLVE_ERR_INVALID, "bad stop mode %d", opt.stop);
-  if (opt.block_threads != 0 && opt.block_threads != 256 && opt.block_threads != 512)
-    return fail(BSOLVE_ERR_INVALID, "block_threads must be 0, 256 or 512 (got %d)",
+  if (opt.block_threads != 0 && opt.block_threads != 128 && opt.block_threads != 256 &&
+      opt.block_threads != 512)
+    return fail(BSOLVE_ERR_INVALID, "block_threads must be 0, 128, 256 or 512 (got %d)",
                 opt.block_threads);
+  if (opt.reg_slots != 0 && opt.reg_slots != 2 && opt.reg_slots != 4)
+    return fail(BSOLVE_ERR_INVALID, "reg_slots must be 0, 2 or 4 (got %d)", opt.reg_slots);
 
   std::vector<int32_t> diag;
   int W = 0;
@@ -392,7 +402,15 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   int r = (n + nt - 1) / nt;
   if (r == 3) r = 4;
   if (nt == 512) r = 4;  // the 512-thread variants own 4 rows per thread
-  if (r > 4)
+  if (nt == 128) {       // hybrid: 8 rows per thread, DIA + SMEM only
+    if (n > 1024 || h->kfmt != FMT_DIA || W != 9)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                            "block_threads = 128 needs a 9-slot stencil (DIA) pattern, n <= 1024"));
+    r = 8;
+  } else if (opt.reg_slots != 0) {
+    return fail_free(fail(BSOLVE_ERR_INVALID, "reg_slots needs block_threads = 128"));
+  }
+  if (r > 4 && nt != 128)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "n = %d needs more than 4 rows per thread at %d threads", n, nt));
   h->nt = nt;
@@ -409,8 +427,9 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                        n % 2 == 0 && (h->sys_stride * 8) % 16 == 0 && smem_regs <= smem_optin &&
                        find_pvariant(h->kfmt, r) != nullptr;
   int place = opt.placement;
-  if (place == BSOLVE_PLACE_AUTO)
-    place = regs_ok ? PLACE_REGS : (smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM);
+  // AUTO: SMEM-staged values with 2 CTAs per SM measured fastest on B200 for
+  // the 992-row workload (DESIGN.md perf log); REGS is opt-in
+  if (place == BSOLVE_PLACE_AUTO) place = smem_need <= smem_optin ? PLACE_SMEM : PLACE_STREAM;
   else if (place == BSOLVE_PLACE_REGS) {
     if (!regs_ok)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
@@ -429,7 +448,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   // of PLACE_REGS for buffers that are not 16-byte aligned
   const int fb_place = (place == PLACE_STREAM || smem_need > smem_optin) ? PLACE_STREAM : PLACE_SMEM;
   h->smem_bytes_fallback = (int)(fb_place == PLACE_SMEM ? smem_need : tail);
-  h->var = find_variant(h->kfmt, fb_place, h->wb, h->wb == 9, r, nt);
+  h->var = find_variant(h->kfmt, fb_place, h->wb, h->wb == 9, r, nt, opt.reg_slots);
   if (!h->var)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
                           h->fmt, fb_place, h->wb, r, nt));

@@ -187,12 +187,13 @@ __device__ __forceinline__ uint32_t field16(uint32_t pk) {
 }
 
 // Per-thread view of its rows of the shared pattern.
-template <int FMT, int WB, int R>
+template <int FMT, int WB, int R, int KREG = 0>
 struct RowMeta {
   uint32_t cpk[R][(WB + 1) / 2]; // CSR/ELL: packed 16-bit byte offsets (col*8) into the gather body
   int vbase[R];                  // ELL/DIA: row (clamped for idle lanes); CSR: row_ptr[row]
   int vlen[R];                   // CSR row length
   double a0[R];                  // ELL/DIA: the diagonal value (slot 0)
+  double vreg[R][KREG > 0 ? KREG : 1];  // ELL/DIA: values of slots 1..KREG in registers
   bool act[R];                   // row < n
 };
 
@@ -204,11 +205,11 @@ struct RowMeta {
 // A warp whose row block j lies entirely at or beyond n skips it with a
 // warp-uniform branch; idle lanes of a partial warp run on a clamped row and
 // zero their result.
-template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT>
+template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int KREG>
 __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
                                           const unsigned char *gb, const SolveParams &P,
-                                          const RowMeta<FMT, WB, R> &m, const double (&own)[R],
-                                          double (&y)[R]) {
+                                          const RowMeta<FMT, WB, R, KREG> &m,
+                                          const double (&own)[R], double (&y)[R]) {
   const int n = P.n;
   const int wrow0 = threadIdx.x & ~31;
 #pragma unroll
@@ -240,8 +241,14 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
                   (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
               g = *reinterpret_cast<const double *>(gb + off);
             }
-            const double *a_p = V + m.vbase[j] + k * n;
-            acc = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p, g, acc);
+            double a;
+            if (k <= KREG) {
+              a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];  // slots 1..KREG: registers
+            } else {
+              const double *a_p = V + m.vbase[j] + k * n;
+              a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
+            }
+            acc = fma(a, g, acc);
           }
         }
       }
@@ -447,7 +454,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
 //   [values: smem_vals doubles (PLACE_SMEM only)]
 //   [gather: guard | n_pad body | guard doubles]
 //   [reduction scratch: 2 * 4 * NWARP doubles] [mbarrier: 8 B]
-template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB>
+template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB, int KREG = 0>
 __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -496,7 +503,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   }
 
   // ---- pattern + right-hand side + initial guess into registers ----------
-  RowMeta<FMT, WB, R> m;
+  RowMeta<FMT, WB, R, KREG> m;
   double x[R], r[R], d[R];
   const double *bsys = P.b + sys * n;
   int dsl[R];
@@ -543,13 +550,17 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     const int pos = (FMT == FMT_CSR) ? m.vbase[j] + dsl[j] : m.vbase[j];  // ELL/DIA: slot 0
     const double a = m.act[j] ? ((PLACE == PLACE_STREAM) ? __ldg(V + pos) : V[pos]) : 0.0;
     if (FMT != FMT_CSR) m.a0[j] = a;
+#pragma unroll
+    for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k)  // hybrid: slots 1..KREG -> registers
+      m.vreg[j][k] = (PLACE == PLACE_STREAM) ? __ldg(V + m.vbase[j] + (k + 1) * n)
+                                             : V[m.vbase[j] + (k + 1) * n];
     d[j] = (a != 0.0) ? 1.0 / a : 1.0;
   }
 
   int buf = 0;
   bicgstab_core<R, NT, false>(
       P, sys, x, r, d, m.act, r, sg, sred, buf, [&](const double(&own)[R], double(&y)[R]) {
-        spmv_rows<FMT, PLACE, WB, EXACT, R, NT>(V, gb, P, m, own, y);
+        spmv_rows<FMT, PLACE, WB, EXACT, R, NT, KREG>(V, gb, P, m, own, y);
       });
 }
 

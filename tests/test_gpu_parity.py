@@ -30,8 +30,7 @@ def test_config0_ion_electron_pair(fmt):
     B = X.make_batch(0, 2)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt)
-    # ELL auto-plans the persistent register-resident kernel, CSR the SMEM one
-    assert g["info"]["placement"] == (3 if fmt == "ell" else 1)
+    assert g["info"]["placement"] == 1  # SMEM staged (AUTO)
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
 
 
@@ -180,14 +179,20 @@ def test_no_true_residual_check():
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
 
 
-def test_ill_conditioned_guard():
-    """configs[4] flavour: kappa ~ 1e5 electrons trigger the true-residual guard."""
-    ill = X.Species(X.ELECTRON_K, cross=0.0, margin=1e-3)
-    B = X.make_batch(1, 8, electron=ill)
-    p = B.pattern
-    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
-    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, iter_tol=10)
+@pytest.mark.parametrize("placement", ["smem", "regs"])
+def test_ill_conditioned_guard(placement):
+    """configs[4] flavour: kappa ~ 1e3..1e5 electrons (R18): the
+    iteration count is chaotic in the summation order at this conditioning,
+    so parity is x vs the direct solve (1e-8), the TRUE residual (<= tau) and
+    the status; iterations agree within 50% of the oracle's."""
+    for margin in (1e-1, 1e-2, 1e-3):
+        ill = X.Species(X.ELECTRON_K, cross=0.0, margin=margin)
+        B = X.make_batch(1, 8, electron=ill)
+        p = B.pattern
+        g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000, placement=placement)
+        o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
+        compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o,
+                iter_tol=max(10, int(0.5 * o["iters"].max())))
 
 
 # ------------------------------------------------- invariants on the GPU --
@@ -335,3 +340,17 @@ def test_regs_warm_start_x0_alias():
              status=st.cpu().numpy().astype(np.int32))
     o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+
+
+@pytest.mark.parametrize("reg_slots", [0, 2, 4])
+def test_hybrid_128_threads(reg_slots):
+    """block_threads = 128 (8 rows per thread) with slots 1..reg_slots in registers."""
+    B = X.make_batch(0, 200)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 200, block_threads=128, reg_slots=reg_slots)
+    assert S.info["block_threads"] == 128 and S.info["rows_per_thread"] == 8
+    x, it, res, st = S.run(to_dev(S.ell_values(B.values)), to_dev(B.b))
+    torch.cuda.synchronize()
+    g = dict(x=x.cpu().numpy(), iters=it.cpu().numpy(), resnorm=res.cpu().numpy(),
+             status=st.cpu().numpy().astype(np.int32))
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
