@@ -74,6 +74,7 @@ static const Variant kVariants[] = {
     V_FP(16, false, 4, 256, 2), V_FP(16, false, 4, 512, 1),
     // experimental hybrid: 128 threads x 8 rows, 2 CTAs/SM, slots 1..KREG in registers
     VK_(FMT_DIA, 8, 128, 2, 0), VK_(FMT_DIA, 8, 128, 2, 2), VK_(FMT_DIA, 8, 128, 2, 4),
+    VK_(FMT_DIA, 8, 128, 2, 6), VK_(FMT_DIA, 8, 128, 2, 8),
 };
 
 // Persistent register-resident variants (PLACE_REGS): ELL/DIA, W = 9.
@@ -308,8 +309,8 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       opt.block_threads != 512)
     return fail(BSOLVE_ERR_INVALID, "block_threads must be 0, 128, 256 or 512 (got %d)",
                 opt.block_threads);
-  if (opt.reg_slots != 0 && opt.reg_slots != 2 && opt.reg_slots != 4)
-    return fail(BSOLVE_ERR_INVALID, "reg_slots must be 0, 2 or 4 (got %d)", opt.reg_slots);
+  if (opt.reg_slots < 0 || opt.reg_slots > 8 || (opt.reg_slots & 1))
+    return fail(BSOLVE_ERR_INVALID, "reg_slots must be 0, 2, 4, 6 or 8 (got %d)", opt.reg_slots);
 
   std::vector<int32_t> diag;
   int W = 0;
