@@ -202,40 +202,88 @@ struct RowMeta {
 // body (byte address), `own[j]` is this thread's own gather entry g[row]
 // (ELL/DIA: slot 0 is the diagonal, so its operand never leaves registers).
 // Values come from V (shared or global).  EXACT: W == WB at compile time.
-// A warp whose row block j lies entirely at or beyond n skips it with a
-// warp-uniform branch; idle lanes of a partial warp run on a clamped row and
-// zero their result.
+// Row blocks: a warp whose row block j lies entirely at or beyond n skips it.
+// The common cases -- all R blocks of the warp active, or all but the last --
+// run branch-free so the compiler interleaves the loads and FMA chains of
+// all rows (per-row branches serialised them: DFMA latency was exposed).
+// Idle lanes of a partial warp run on a clamped row and zero their result.
+template <int FMT, int PLACE, int WB, bool EXACT, int R, int KREG, int NB>
+__device__ __forceinline__ void spmv_block(const double *__restrict__ V,
+                                           const unsigned char *gb, const SolveParams &P,
+                                           const RowMeta<FMT, WB, R, KREG> &m,
+                                           const double (&own)[R], double (&y)[R]) {
+  const int n = P.n;
+  double acc[R];
+#pragma unroll
+  for (int j = 0; j < NB; ++j) acc[j] = (FMT == FMT_CSR) ? 0.0 : m.a0[j] * own[j];  // slot 0
+#pragma unroll
+  for (int k = (FMT == FMT_CSR) ? 0 : 1; k < WB; ++k) {
+#pragma unroll
+    for (int j = 0; j < NB; ++j) {
+      if (FMT == FMT_CSR) {
+        if ((EXACT || k < P.W) && k < m.vlen[j]) {
+          const uint32_t off =
+              (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+          const double g = *reinterpret_cast<const double *>(gb + off);
+          const double *a_p = V + m.vbase[j] + k;
+          acc[j] = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p, g, acc[j]);
+        }
+      } else if (EXACT || k < P.W) {
+        double g;
+        if (FMT == FMT_DIA) {
+          g = *reinterpret_cast<const double *>(gb + m.vbase[j] * 8 + P.doff[k]);
+        } else {
+          const uint32_t off =
+              (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+          g = *reinterpret_cast<const double *>(gb + off);
+        }
+        double a;
+        if (k <= KREG) {
+          a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];  // slots 1..KREG: registers
+        } else {
+          const double *a_p = V + m.vbase[j] + k * n;
+          a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
+        }
+        acc[j] = fma(a, g, acc[j]);
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j) y[j] = (j < NB && m.act[j]) ? acc[j] : 0.0;
+}
+
 template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int KREG>
 __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
                                           const unsigned char *gb, const SolveParams &P,
                                           const RowMeta<FMT, WB, R, KREG> &m,
                                           const double (&own)[R], double (&y)[R]) {
-  const int n = P.n;
   const int wrow0 = threadIdx.x & ~31;
+  const int n = P.n;
+  if (wrow0 + (R - 1) * NT < n) {
+    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, R>(V, gb, P, m, own, y);
+  } else if (R > 1 && wrow0 + (R - 2) * NT < n) {
+    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, (R > 1 ? R - 1 : 1)>(V, gb, P, m, own, y);
+  } else {
+    // generic tail (small n: several idle row blocks): one block at a time
 #pragma unroll
-  for (int j = 0; j < R; ++j) {
-    double acc = 0.0;
-    if (wrow0 + j * NT < n) {
-      if (FMT == FMT_CSR) {
+    for (int j = 0; j < R; ++j) {
+      double acc = 0.0;
+      if (wrow0 + j * NT < n) {
+        if (FMT != FMT_CSR) acc = m.a0[j] * own[j];  // slot 0, same order as spmv_block
 #pragma unroll
-        for (int k = 0; k < WB; ++k) {
-          if ((EXACT || k < P.W) && k < m.vlen[j]) {
-            const uint32_t off =
-                (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
-            const double g = *reinterpret_cast<const double *>(gb + off);
-            const double *a_p = V + m.vbase[j] + k;
-            acc = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p, g, acc);
-          }
-        }
-      } else {
-        acc = m.a0[j] * own[j];  // slot 0: diagonal, operand = own entry
-        const unsigned char *grow = gb + m.vbase[j] * 8;
-#pragma unroll
-        for (int k = 1; k < WB; ++k) {
-          if (EXACT || k < P.W) {
+        for (int k = (FMT == FMT_CSR) ? 0 : 1; k < WB; ++k) {
+          if (FMT == FMT_CSR) {
+            if ((EXACT || k < P.W) && k < m.vlen[j]) {
+              const uint32_t off =
+                  (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
+              const double *a_p = V + m.vbase[j] + k;
+              acc = fma((PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p,
+                        *reinterpret_cast<const double *>(gb + off), acc);
+            }
+          } else if (EXACT || k < P.W) {
             double g;
             if (FMT == FMT_DIA) {
-              g = *reinterpret_cast<const double *>(grow + P.doff[k]);
+              g = *reinterpret_cast<const double *>(gb + m.vbase[j] * 8 + P.doff[k]);
             } else {
               const uint32_t off =
                   (k & 1) ? field16<16>(m.cpk[j][k >> 1]) : field16<0>(m.cpk[j][k >> 1]);
@@ -243,7 +291,7 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
             }
             double a;
             if (k <= KREG) {
-              a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];  // slots 1..KREG: registers
+              a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];
             } else {
               const double *a_p = V + m.vbase[j] + k * n;
               a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
@@ -252,8 +300,8 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
           }
         }
       }
+      y[j] = m.act[j] ? acc : 0.0;
     }
-    y[j] = m.act[j] ? acc : 0.0;
   }
 }
 
