@@ -659,8 +659,10 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
     if (P.x0) tma_bulk_g2s(sx0, P.x0 + s * n, nbytes, mbar);
   };
 
-  // pattern registers (once per CTA) and gather guards
-  RowMeta<FMT, WB, R> m;
+  // pattern registers (once per CTA) and gather guards.  All W - 1 off-
+  // diagonal slots are "register slots" (KREG = WB - 1), so the shared SpMV
+  // never dereferences the values buffer.
+  RowMeta<FMT, WB, R, WB - 1> m;
 #pragma unroll
   for (int j = 0; j < R; ++j) {
     const int row = tid + j * NT;
@@ -699,13 +701,14 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
     mbar_wait_parity(mbar, phase);
     phase ^= 1u;
     // ---- registers <- staging buffers -------------------------------------
-    double val[R][WB], x[R], r[R], d[R], bv[R];
+    double x[R], r[R], d[R], bv[R];
 #pragma unroll
     for (int j = 0; j < R; ++j) {
+      m.a0[j] = sval[m.vbase[j]];  // slot 0 = diagonal
 #pragma unroll
-      for (int k = 0; k < WB; ++k)
-        val[j][k] = (EXACT || k < P.W) ? sval[k * n + m.vbase[j]] : 0.0;
-      const double a = m.act[j] ? val[j][0] : 0.0;  // slot 0 = diagonal
+      for (int k = 1; k < WB; ++k)
+        m.vreg[j][k - 1] = (EXACT || k < P.W) ? sval[k * n + m.vbase[j]] : 0.0;
+      const double a = m.act[j] ? m.a0[j] : 0.0;
       d[j] = (a != 0.0) ? 1.0 / a : 1.0;
       bv[j] = m.act[j] ? sb[m.vbase[j]] : 0.0;
       r[j] = bv[j];
@@ -720,33 +723,10 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
         issue(nxt);
       }
     }
-    const int wrow0 = tid & ~31;
     bicgstab_core<R, NT, true>(
         P, cur, x, r, d, m.act, bv, sg, sred, buf,
         [&](const double(&own)[R], double(&y)[R]) {
-#pragma unroll
-          for (int j = 0; j < R; ++j) {
-            double acc = 0.0;
-            if (wrow0 + j * NT < n) {
-              acc = val[j][0] * own[j];
-              const unsigned char *grow = gb + m.vbase[j] * 8;
-#pragma unroll
-              for (int k = 1; k < WB; ++k) {
-                if (EXACT || k < P.W) {
-                  double g;
-                  if (FMT == FMT_DIA) {
-                    g = *reinterpret_cast<const double *>(grow + P.doff[k]);
-                  } else {
-                    const uint32_t off = (k & 1) ? field16<16>(m.cpk[j][k >> 1])
-                                                 : field16<0>(m.cpk[j][k >> 1]);
-                    g = *reinterpret_cast<const double *>(gb + off);
-                  }
-                  acc = fma(val[j][k], g, acc);
-                }
-              }
-            }
-            y[j] = m.act[j] ? acc : 0.0;
-          }
+          spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, WB - 1>(sval, gb, P, m, own, y);
         });
     cur = *s_next;  // written before the core's first barrier
   }
