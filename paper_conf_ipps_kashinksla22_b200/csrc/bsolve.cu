@@ -419,7 +419,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->n_pad = (n + 1) & ~1;
   h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
   const int nwarp = nt / 32;
-  const int tail = (h->n_pad + 2 * h->guard) * 8 + 8 * nwarp * 8 + 16;
+  const int tail = (h->n_pad + 2 * h->guard) * 8 + 16 * nwarp * 8 + 16;
   const long long smem_need = (long long)h->smem_vals * 8 + tail;
   // PLACE_REGS: persistent kernel, values in registers, staging buffers for
   // values + b + x0 in SMEM (DESIGN.md "Kernels" 7)

@@ -105,7 +105,7 @@ __device__ __forceinline__ double tree_sum(const double *a) {
   }
 }
 
-// Block-wide sum of K <= 4 doubles with ONE barrier.  On B200 every SHFL.32
+// Block-wide sum of K <= 8 doubles with ONE barrier.  On B200 every SHFL.32
 // costs one shared-memory data-pipe wavefront (like an LDS) and ~20+ cycles
 // of latency, so:
 //  * inside a warp, recursive halving: with K > 1 the first steps exchange
@@ -125,40 +125,31 @@ __device__ __forceinline__ double tree_sum(const double *a) {
 template <int K, int NWARP>
 __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf, int lane,
                                           int warp) {
-  static_assert(K >= 1 && K <= 4, "block_sum supports 1..4 values");
+  static_assert(K >= 1 && K <= 8, "block_sum supports 1..8 values");
   static_assert(NWARP % 2 == 0 && NWARP <= 32, "NWARP must be even");
-  double keep;
-  int first_step;
-  if constexpr (K == 1) {
-    keep = v[0];
-    first_step = 16;
-  } else if constexpr (K == 2) {
-    const bool hi = lane & 16;
-    keep = (hi ? v[1] : v[0]) + __shfl_xor_sync(0xffffffffu, hi ? v[0] : v[1], 16);
-    first_step = 8;
-  } else {
-    // K = 3 or 4: pairs (v0, v1) and (v2, v3) by lane bit 4, then by bit 3
-    const double v3 = (K == 4) ? v[K - 1] : 0.0;
-    const bool hi4 = lane & 16, hi3 = lane & 8;
-    const double k0 = (hi4 ? v[2] : v[0]) + __shfl_xor_sync(0xffffffffu, hi4 ? v[0] : v[2], 16);
-    const double k1 = (hi4 ? v3 : v[1]) + __shfl_xor_sync(0xffffffffu, hi4 ? v[1] : v3, 16);
-    keep = (hi3 ? k1 : k0) + __shfl_xor_sync(0xffffffffu, hi3 ? k0 : k1, 8);
-    first_step = 4;
-  }
+  constexpr int KP = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;  // padded value count
+  constexpr int SPAN = 32 / KP;  // lanes sharing one value after the halving steps
+  double a[KP];
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1)
-    if (o <= first_step) keep += __shfl_xor_sync(0xffffffffu, keep, o);
-  // value index held by this lane: K = 1: all lanes value 0; K = 2: bit 4;
-  // K >= 3: bit 4 selects the pair (v0,v1) / (v2,v3), bit 3 the member
-  double *S = sred + buf * (4 * NWARP);
-  if constexpr (K == 1) {
-    if (lane == 0) S[warp] = keep;
-  } else if constexpr (K == 2) {
-    if ((lane & 15) == 0) S[(lane >> 4) * NWARP + warp] = keep;
-  } else {
-    const int q = ((lane >> 4) & 1) * 2 + ((lane >> 3) & 1);  // 0: v0, 1: v1, 2: v2, 3: v3
-    if ((lane & 7) == 0 && q < K) S[q * NWARP + warp] = keep;
+  for (int i = 0; i < KP; ++i) a[i] = i < K ? v[i] : 0.0;
+  // recursive halving: at offset o a lane keeps the upper half of its values
+  // if lane bit o is set, the lower half otherwise, and adds its partner's copy
+#pragma unroll
+  for (int cnt = KP, o = 16; cnt > 1; cnt >>= 1, o >>= 1) {
+    const bool hi = lane & o;
+#pragma unroll
+    for (int i = 0; i < cnt / 2; ++i) {
+      const double send = hi ? a[i] : a[i + cnt / 2];
+      const double keep = hi ? a[i + cnt / 2] : a[i];
+      a[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+    }
   }
+  // xor butterfly over the SPAN lanes that hold the same value
+#pragma unroll
+  for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
+  double *S = sred + buf * (8 * NWARP);
+  const int q = lane / SPAN;  // value index held by this lane
+  if ((lane % SPAN) == 0 && q < K) S[q * NWARP + warp] = a[0];
   __syncthreads();
   double part[K][NWARP];
 #pragma unroll
@@ -166,9 +157,9 @@ __device__ __forceinline__ void block_sum(double (&v)[K], double *sred, int &buf
     const double2 *S2 = reinterpret_cast<const double2 *>(S + k * NWARP);
 #pragma unroll
     for (int w = 0; w < NWARP / 2; ++w) {
-      const double2 q = S2[w];
-      part[k][2 * w] = q.x;
-      part[k][2 * w + 1] = q.y;
+      const double2 qq = S2[w];
+      part[k][2 * w] = qq.x;
+      part[k][2 * w + 1] = qq.y;
     }
   }
 #pragma unroll
@@ -382,14 +373,42 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
     return tr[0];
   };
 
+  // Iteration schedule (DESIGN.md "Kernels" 5): two reduction rounds per
+  // iteration instead of four.
+  //  * ||s|| (stop test 2) is reduced together with t.s and t.t after the
+  //    second SpMV; when it fires, that SpMV was speculative and t is
+  //    discarded;
+  //  * rho_{i+1} = r^.r_{i+1} = r^.s - omega r^.t (exact algebra for
+  //    r_{i+1} = s - omega t) comes from the same round;
+  //  * ||r_{i+1}|| (stop test 1) is reduced together with r^.v after the next
+  //    first SpMV; when it fires, that SpMV was speculative and the exit is
+  //    reported at loop index i+1 with x untouched, as in Alg. 1.
+  // x, the iteration count and the exit test are those of Alg. 1; only the
+  // rounding of rho differs (fp sums in another order).
   int it = 0, st = -1, exit_kind = 0;
   double rho_old = 1.0, alpha = 1.0, omega = 1.0;
   double final_res = -1.0;
+  bool have_rnorm = true;  // rnorm holds ||r|| of the current r
   for (;;) {
     exit_kind = 0;
-    while (it < P.maxiter) {
-      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1
-      if (bad(rho)) { st = SYS_BREAKDOWN; break; }
+    while (true) {
+      if (have_rnorm && rnorm < tau) { exit_kind = 1; break; }  // stop test 1
+      if (it >= P.maxiter) break;
+      if (bad(rho)) {
+        if (!have_rnorm) {  // rare: settle stop test 1 before declaring breakdown
+          double rr[1];
+          double pr[R];
+#pragma unroll
+          for (int j = 0; j < R; ++j) pr[j] = r[j] * r[j];
+          rr[0] = tree_sum<R>(pr);
+          block_sum<1, NWARP>(rr, sred, buf, lane, warp);
+          rnorm = sqrt(rr[0]);
+          have_rnorm = true;
+          continue;
+        }
+        st = SYS_BREAKDOWN;
+        break;
+      }
       const double beta = (rho / rho_old) * (alpha / omega);  // R2
       // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
       double ph[R];
@@ -402,38 +421,55 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       __syncthreads();
       // a6: v = A p^
       spmv(ph, v);
-      ++it;
-      // a7: alpha = rho / (r^ . v)
-      double rv[1] = {0.0};
+      // a7: r^.v, and ||r|| of the current r for the deferred stop test 1
+      double red[2], pa[R], pb[R];
 #pragma unroll
-      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
-      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
-      if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
-      alpha = rho / rv[0];                                 // R3
+      for (int j = 0; j < R; ++j) {
+        pa[j] = rh[j] * v[j];
+        pb[j] = r[j] * r[j];
+      }
+      red[0] = tree_sum<R>(pa);
+      red[1] = tree_sum<R>(pb);
+      block_sum<2, NWARP>(red, sred, buf, lane, warp);
+      if (!have_rnorm) {
+        rnorm = sqrt(red[1]);
+        if (rnorm < tau) { exit_kind = 1; break; }         // stop test 1, deferred
+      }
+      have_rnorm = false;
+      ++it;
+      if (bad(red[0])) { st = SYS_BREAKDOWN; break; }
+      alpha = rho / red[0];                                // R3
       // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
       // barrier in the reduction above separates them)
       double s[R], sh[R];
-      double ts[3] = {0.0, 0.0, 0.0};  // t.s, t.t, s.s
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         s[j] = r[j] - alpha * v[j];
-        ts[2] += s[j] * s[j];
         sh[j] = d[j] * s[j];
         if (act[j]) sg[tid + j * NT] = sh[j];
       }
       __syncthreads();  // publish s^
-      // a9: t = A s^.  ||s|| for stop test 2 is reduced together with t.s and
-      // t.t (one reduction round fewer per iteration); when stop test 2 fires
-      // this SpMV was speculative and t is discarded -- x, iteration count and
-      // exit are exactly those of Alg. 1
+      // a9: t = A s^ (speculative when stop test 2 fires)
       double t[R];
       spmv(sh, t);
+      double ts[5];  // t.s, t.t, s.s, r^.s, r^.t
+      {
+        double q0[R], q1[R], q2[R], q3[R], q4[R];
 #pragma unroll
-      for (int j = 0; j < R; ++j) {
-        ts[0] += t[j] * s[j];
-        ts[1] += t[j] * t[j];
+        for (int j = 0; j < R; ++j) {
+          q0[j] = t[j] * s[j];
+          q1[j] = t[j] * t[j];
+          q2[j] = s[j] * s[j];
+          q3[j] = rh[j] * s[j];
+          q4[j] = rh[j] * t[j];
+        }
+        ts[0] = tree_sum<R>(q0);
+        ts[1] = tree_sum<R>(q1);
+        ts[2] = tree_sum<R>(q2);
+        ts[3] = tree_sum<R>(q3);
+        ts[4] = tree_sum<R>(q4);
       }
-      block_sum<3, NWARP>(ts, sred, buf, lane, warp);
+      block_sum<5, NWARP>(ts, sred, buf, lane, warp);
       if (sqrt(ts[2]) < tau) {                             // stop test 2
 #pragma unroll
         for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
@@ -443,19 +479,13 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
       omega = ts[0] / ts[1];
       if (bad(omega)) { st = SYS_BREAKDOWN; break; }
-      double rr[2] = {0.0, 0.0};
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
         r[j] = s[j] - omega * t[j];
-        rr[0] += r[j] * r[j];
-        rr[1] += rh[j] * r[j];
       }
       rho_old = rho;
-      // next iteration's ||r|| and rho = r^ . r in the same single barrier
-      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
-      rnorm = sqrt(rr[0]);
-      rho = rr[1];
+      rho = ts[3] - omega * ts[4];  // r^ . (s - omega t)
     }
     if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
     // ---- a11: true-residual guard (DESIGN R4) -----------------------------
@@ -474,6 +504,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
     }
     rho_old = alpha = omega = 1.0;
     rnorm = final_res;
+    have_rnorm = true;
     rho = tr2;
     final_res = -1.0;
   }
@@ -501,7 +532,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
 // Grid: one CTA per system (blockIdx.x = system).  Dynamic SMEM layout:
 //   [values: smem_vals doubles (PLACE_SMEM only)]
 //   [gather: guard | n_pad body | guard doubles]
-//   [reduction scratch: 2 * 4 * NWARP doubles] [mbarrier: 8 B]
+//   [reduction scratch: 2 * 8 * NWARP doubles] [mbarrier: 8 B]
 template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int MINB, int KREG = 0>
 __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
@@ -510,7 +541,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   double *sgf = sval + (PLACE == PLACE_SMEM ? P.smem_vals : 0);  // gather incl. guards
   double *sg = sgf + P.guard;                                     // gather body
   double *sred = sgf + P.n_pad + 2 * P.guard;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 8 * NWARP);
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
   const int tid = threadIdx.x;
@@ -622,7 +653,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
 // then reads only the gathered operands from SMEM: the matrix never touches
 // the shared-memory data pipe again.
 //   SMEM: [values: smem_vals][b: n_pad][x0: n_pad][gather: guard|n_pad|guard]
-//         [reduction scratch: 8*NWARP][mbarrier][next-system slot]
+//         [reduction scratch: 16*NWARP][mbarrier][next-system slot]
 // The counter (ctr[0]) and the finished-CTA count (ctr[1]) reset themselves
 // when the last CTA leaves, so consecutive launches on one stream need no
 // host-side reset.
@@ -638,7 +669,7 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
   double *sgf = sx0 + P.n_pad;
   double *sg = sgf + P.guard;
   double *sred = sgf + P.n_pad + 2 * P.guard;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 8 * NWARP);
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
   volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
   const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
 
