@@ -396,10 +396,21 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->num_sms = prop.multiProcessorCount;
   const int smem_optin = (int)prop.sharedMemPerBlockOptin;
 
-  // rows per thread / CTA size: prefer 256 threads (2 CTAs per SM fit the
-  // register file at <= 128 regs/thread), 512 threads for 1025..2048 rows.
+  // rows per thread / CTA size.  Auto: 9-point stencils (DIA) up to 1024 rows
+  // take the hybrid 128 threads x 8 rows with 4 off-diagonal slots in
+  // registers (measured fastest on B200, DESIGN.md perf log); otherwise 256
+  // threads (2 CTAs per SM at <= 128 regs/thread), 512 for 1025..2048 rows.
   int nt = opt.block_threads;
-  if (nt == 0) nt = n <= 1024 ? 256 : 512;
+  int kreg = opt.reg_slots;
+  const bool stencil9 = h->kfmt == FMT_DIA && W == 9 && n <= 1024;
+  if (nt == 0) {
+    if (stencil9 && (opt.placement == BSOLVE_PLACE_AUTO || opt.placement == BSOLVE_PLACE_SMEM)) {
+      nt = 128;
+      kreg = 4;
+    } else {
+      nt = n <= 1024 ? 256 : 512;
+    }
+  }
   int r = (n + nt - 1) / nt;
   if (r == 3) r = 4;
   if (nt == 512) r = 4;  // the 512-thread variants own 4 rows per thread
@@ -408,7 +419,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                             "block_threads = 128 needs a 9-slot stencil (DIA) pattern, n <= 1024"));
     r = 8;
-  } else if (opt.reg_slots != 0) {
+  } else if (kreg != 0) {
     return fail_free(fail(BSOLVE_ERR_INVALID, "reg_slots needs block_threads = 128"));
   }
   if (r > 4 && nt != 128)
@@ -449,7 +460,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   // of PLACE_REGS for buffers that are not 16-byte aligned
   const int fb_place = (place == PLACE_STREAM || smem_need > smem_optin) ? PLACE_STREAM : PLACE_SMEM;
   h->smem_bytes_fallback = (int)(fb_place == PLACE_SMEM ? smem_need : tail);
-  h->var = find_variant(h->kfmt, fb_place, h->wb, h->wb == 9, r, nt, opt.reg_slots);
+  h->var = find_variant(h->kfmt, fb_place, h->wb, h->wb == 9, r, nt, kreg);
   if (!h->var)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no kernel variant for fmt=%d place=%d W=%d R=%d NT=%d",
                           h->fmt, fb_place, h->wb, r, nt));

@@ -95,6 +95,20 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity)
 
 __device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
 
+// Sum over this thread's R rows of f(j) with two interleaved accumulators
+// (even / odd rows): half the dependent-add latency of one chain at the
+// register cost of two.  Fixed order.
+template <int R, class F>
+__device__ __forceinline__ double rows_sum(F &&f) {
+  double e = 0.0, o = 0.0;
+#pragma unroll
+  for (int j = 0; j < R; j += 2) {
+    e += f(j);
+    if (j + 1 < R) o += f(j + 1);
+  }
+  return e + o;
+}
+
 // Pairwise (tree) sum of N doubles, fixed order: latency log2(N) adds.
 template <int N>
 __device__ __forceinline__ double tree_sum(const double *a) {
@@ -304,7 +318,7 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
 //   bv: b in registers (B_IN_REGS) for the true residual, else re-read bsys.
 // Writes x, iters, resnorm, status of system `sys`.  Every path executes at
 // least one block_sum (one barrier) after entry.
-template <int R, int NT, bool B_IN_REGS, class SpMV>
+template <int R, int NT, bool B_IN_REGS, int ROUNDS, class SpMV>
 __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sys, double (&x)[R],
                                               double (&r)[R], const double (&d)[R],
                                               const bool (&act)[R], const double (&bv)[R],
@@ -373,8 +387,11 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
     return tr[0];
   };
 
-  // Iteration schedule (DESIGN.md "Kernels" 5): two reduction rounds per
-  // iteration instead of four.
+  // Iteration schedules (DESIGN.md "Kernels" 5).  ROUNDS == 3 (register-
+  // limited 2-CTA/SM kernels): r^.v | t.s, t.t, ||s|| | ||r||, r^.r -- ||s||
+  // for stop test 2 is reduced with t.s and t.t after the second SpMV, which
+  // is discarded (speculative) when the test fires.  ROUNDS == 2 (latency-
+  // limited persistent kernel): two reduction rounds per iteration.
   //  * ||s|| (stop test 2) is reduced together with t.s and t.t after the
   //    second SpMV; when it fires, that SpMV was speculative and t is
   //    discarded;
@@ -391,16 +408,83 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   bool have_rnorm = true;  // rnorm holds ||r|| of the current r
   for (;;) {
     exit_kind = 0;
+    if constexpr (ROUNDS == 3) {
+    while (true) {
+      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1
+      if (it >= P.maxiter) break;
+      if (bad(rho)) { st = SYS_BREAKDOWN; break; }
+      const double beta = (rho / rho_old) * (alpha / omega);  // R2
+      // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
+      double ph[R];
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        p[j] = r[j] + beta * (p[j] - omega * v[j]);
+        ph[j] = d[j] * p[j];
+        if (act[j]) sg[tid + j * NT] = ph[j];
+      }
+      __syncthreads();
+      // a6: v = A p^
+      spmv(ph, v);
+      ++it;
+      // a7: alpha = rho / (r^ . v)
+      double rv[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
+      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
+      if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
+      alpha = rho / rv[0];                                 // R3
+      // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
+      // barrier in the reduction above separates them)
+      double s[R], sh[R];
+      double ts[3] = {0.0, 0.0, 0.0};  // t.s, t.t, s.s
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        s[j] = r[j] - alpha * v[j];
+        ts[2] += s[j] * s[j];
+        sh[j] = d[j] * s[j];
+        if (act[j]) sg[tid + j * NT] = sh[j];
+      }
+      __syncthreads();  // publish s^
+      // a9: t = A s^ (speculative when stop test 2 fires)
+      double t[R];
+      spmv(sh, t);
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        ts[0] += t[j] * s[j];
+        ts[1] += t[j] * t[j];
+      }
+      block_sum<3, NWARP>(ts, sred, buf, lane, warp);
+      if (sqrt(ts[2]) < tau) {                             // stop test 2
+#pragma unroll
+        for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
+        exit_kind = 2;
+        break;
+      }
+      if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
+      omega = ts[0] / ts[1];
+      if (bad(omega)) { st = SYS_BREAKDOWN; break; }
+      double rr[2] = {0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
+        r[j] = s[j] - omega * t[j];
+        rr[0] += r[j] * r[j];
+        rr[1] += rh[j] * r[j];
+      }
+      rho_old = rho;
+      // next iteration's ||r|| and rho = r^ . r in the same single barrier
+      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
+      rnorm = sqrt(rr[0]);
+      rho = rr[1];
+    }
+    } else {
     while (true) {
       if (have_rnorm && rnorm < tau) { exit_kind = 1; break; }  // stop test 1
       if (it >= P.maxiter) break;
       if (bad(rho)) {
         if (!have_rnorm) {  // rare: settle stop test 1 before declaring breakdown
           double rr[1];
-          double pr[R];
-#pragma unroll
-          for (int j = 0; j < R; ++j) pr[j] = r[j] * r[j];
-          rr[0] = tree_sum<R>(pr);
+          rr[0] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
           block_sum<1, NWARP>(rr, sred, buf, lane, warp);
           rnorm = sqrt(rr[0]);
           have_rnorm = true;
@@ -422,14 +506,9 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       // a6: v = A p^
       spmv(ph, v);
       // a7: r^.v, and ||r|| of the current r for the deferred stop test 1
-      double red[2], pa[R], pb[R];
-#pragma unroll
-      for (int j = 0; j < R; ++j) {
-        pa[j] = rh[j] * v[j];
-        pb[j] = r[j] * r[j];
-      }
-      red[0] = tree_sum<R>(pa);
-      red[1] = tree_sum<R>(pb);
+      double red[2];
+      red[0] = rows_sum<R>([&](int j) { return rh[j] * v[j]; });
+      red[1] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
       block_sum<2, NWARP>(red, sred, buf, lane, warp);
       if (!have_rnorm) {
         rnorm = sqrt(red[1]);
@@ -453,22 +532,11 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       double t[R];
       spmv(sh, t);
       double ts[5];  // t.s, t.t, s.s, r^.s, r^.t
-      {
-        double q0[R], q1[R], q2[R], q3[R], q4[R];
-#pragma unroll
-        for (int j = 0; j < R; ++j) {
-          q0[j] = t[j] * s[j];
-          q1[j] = t[j] * t[j];
-          q2[j] = s[j] * s[j];
-          q3[j] = rh[j] * s[j];
-          q4[j] = rh[j] * t[j];
-        }
-        ts[0] = tree_sum<R>(q0);
-        ts[1] = tree_sum<R>(q1);
-        ts[2] = tree_sum<R>(q2);
-        ts[3] = tree_sum<R>(q3);
-        ts[4] = tree_sum<R>(q4);
-      }
+      ts[0] = rows_sum<R>([&](int j) { return t[j] * s[j]; });
+      ts[1] = rows_sum<R>([&](int j) { return t[j] * t[j]; });
+      ts[2] = rows_sum<R>([&](int j) { return s[j] * s[j]; });
+      ts[3] = rows_sum<R>([&](int j) { return rh[j] * s[j]; });
+      ts[4] = rows_sum<R>([&](int j) { return rh[j] * t[j]; });
       block_sum<5, NWARP>(ts, sred, buf, lane, warp);
       if (sqrt(ts[2]) < tau) {                             // stop test 2
 #pragma unroll
@@ -486,6 +554,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       }
       rho_old = rho;
       rho = ts[3] - omega * ts[4];  // r^ . (s - omega t)
+    }
     }
     if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
     // ---- a11: true-residual guard (DESIGN R4) -----------------------------
@@ -637,7 +706,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
   }
 
   int buf = 0;
-  bicgstab_core<R, NT, false>(
+  bicgstab_core<R, NT, false, 3>(
       P, sys, x, r, d, m.act, r, sg, sred, buf, [&](const double(&own)[R], double(&y)[R]) {
         spmv_rows<FMT, PLACE, WB, EXACT, R, NT, KREG>(V, gb, P, m, own, y);
       });
@@ -754,7 +823,7 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
         issue(nxt);
       }
     }
-    bicgstab_core<R, NT, true>(
+    bicgstab_core<R, NT, true, 2>(
         P, cur, x, r, d, m.act, bv, sg, sred, buf,
         [&](const double(&own)[R], double(&y)[R]) {
           spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, WB - 1>(sval, gb, P, m, own, y);
