@@ -413,7 +413,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   }
   int r = (n + nt - 1) / nt;
   if (r == 3) r = 4;
-  if (nt == 512) r = 4;  // the 512-thread variants own 4 rows per thread
+  if (nt == 512 && r < 4) r = 4;  // the 512-thread variants own 4 rows per thread
   if (nt == 128) {       // hybrid: 8 rows per thread, DIA + SMEM only
     if (n > 1024 || h->kfmt != FMT_DIA || W != 9)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
@@ -425,6 +425,8 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   if (r > 4 && nt != 128)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "n = %d needs more than 4 rows per thread at %d threads", n, nt));
+  if ((long long)r * nt < n)  // every row must be owned by a thread
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "n = %d exceeds %d threads x %d rows", n, nt, r));
   h->nt = nt;
   h->r = r;
   h->n_pad = (n + 1) & ~1;

@@ -354,3 +354,20 @@ def test_hybrid_128_threads(reg_slots):
     g = dict(x=x.cpu().numpy(), iters=it.cpu().numpy(), resnorm=res.cpu().numpy(),
              status=st.cpu().numpy().astype(np.int32))
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+
+
+def test_rows_beyond_capacity_rejected():
+    """Regression: n larger than threads x rows-per-thread must be refused
+    (UNSUPPORTED), never solved partially."""
+    for nx, ny in [(64, 33), (64, 63)]:  # 2112 and 4032 rows
+        pat = X.stencil_pattern(nx, ny)
+        for bt in (0, 512):
+            try:
+                S = Solver(pat.row_ptr, pat.col_idx, 2, block_threads=bt)
+            except BsolveError as e:
+                assert e.code == -3
+                continue
+            # a plan was accepted: it must cover every row -> verify a solve
+            B = X.make_batch(0, 2, pattern=pat)
+            g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, block_threads=bt)
+            compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
