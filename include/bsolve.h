@@ -70,13 +70,19 @@ enum {
 /* Where the matrix values live while a system iterates (PAPER.md:708-721,
  * 738-813: the paper's automatic shared-memory configuration). */
 enum {
-  BSOLVE_PLACE_AUTO = 0,   /* SMEM if one system's values fit, else STREAM   */
+  BSOLVE_PLACE_AUTO = 0,   /* CLUSTER for large 9-point stencils, else SMEM
+                              if one system's values fit, else STREAM         */
   BSOLVE_PLACE_SMEM = 1,   /* staged once into shared memory by TMA bulk copy */
   BSOLVE_PLACE_STREAM = 2, /* re-read from global memory (L2/L1) every SpMV   */
-  BSOLVE_PLACE_REGS = 3    /* persistent kernel, one CTA per SM: values staged by
+  BSOLVE_PLACE_REGS = 3,   /* persistent kernel, one CTA per SM: values staged by
                               TMA, then held in REGISTERS for the whole solve;
                               the next system's TMA overlaps the current one
                               (ELL, 9 entries per row, even n <= 1024)        */
+  BSOLVE_PLACE_CLUSTER = 4 /* one system per thread-block cluster of C CTAs
+                              (1024 rows each, C <= 8) exchanging halo rows
+                              and reduction partials through distributed
+                              shared memory; 9-point stencils, even
+                              1024 < n <= 8192 (AUTO picks it there)         */
 };
 
 /* Stopping criterion (R5). */
@@ -104,9 +110,10 @@ typedef struct bsolve_options {
   int device;              /* CUDA device ordinal, -1 = current (default -1)  */
   int block_threads;       /* threads per CTA: 0 = auto, 128, 256 or 512
                               (default 0); 128 = 8 rows per thread (ELL) */
-  int reg_slots;           /* with block_threads = 128: off-diagonal ELL slots
-                              held in registers instead of SMEM, 0, 2 or 4
-                              (default 0)                                     */
+  int reg_slots;           /* with block_threads = 128 or the cluster plan:
+                              off-diagonal ELL slots held in registers instead
+                              of SMEM, 0, 2, 4, 6 or 8 (default 0 = planner's
+                              choice: 4)                                      */
 } bsolve_options;
 
 typedef struct bsolve_info {
@@ -124,6 +131,7 @@ typedef struct bsolve_info {
   int kernel_mode;         /* 1 CSR column table, 2 ELL column table, 3 DIA:
                               ELL values whose slot k is column row + d_k in
                               every row (stencils; uniform gather offsets)    */
+  int cluster;             /* CTAs per system (PLACE_CLUSTER), else 0        */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

@@ -92,6 +92,22 @@ static const PVariant *find_pvariant(int fmt, int r) {
   return nullptr;
 }
 
+// Cluster variants (PLACE_CLUSTER): one system per cluster of C CTAs of
+// 128 threads x 8 rows (1024 rows per CTA), DIA, W = 9.
+struct CVariant {
+  int c, kreg;
+  solve_fn fn;
+};
+#define CV_(C, KR) {C, KR, (solve_fn)bicgstab_cluster_kernel<FMT_DIA, 9, true, 8, 128, KR, C>}
+static const CVariant kCVariants[] = {CV_(2, 4), CV_(3, 4), CV_(4, 4), CV_(5, 4), CV_(6, 4),
+                                      CV_(7, 4), CV_(8, 4), CV_(2, 2), CV_(3, 2), CV_(4, 2),
+                                      CV_(5, 2), CV_(6, 2), CV_(7, 2), CV_(8, 2)};
+static const CVariant *find_cvariant(int c, int kreg) {
+  for (const CVariant &v : kCVariants)
+    if (v.c == c && v.kreg == kreg) return &v;
+  return nullptr;
+}
+
 static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt,
                                    int kreg = 0) {
   for (const Variant &v : kVariants)
@@ -113,6 +129,8 @@ struct bsolve_plan {
   long long sys_stride = 0;
   const Variant *var = nullptr;      // per-system-CTA kernel (also the REGS fallback)
   const PVariant *pvar = nullptr;    // persistent kernel when place == PLACE_REGS
+  const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
+  int cluster = 0;                   // CTAs per system (cluster plan)
   int smem_bytes_fallback = 0, grid_persist = 0;
   unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
   std::vector<int32_t> h_ell_col;  // [W][n]
@@ -301,7 +319,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   if (opt_in) opt = *opt_in;
   if (opt.format < BSOLVE_FMT_AUTO || opt.format > BSOLVE_FMT_ELL)
     return fail(BSOLVE_ERR_INVALID, "bad format %d", opt.format);
-  if (opt.placement < BSOLVE_PLACE_AUTO || opt.placement > BSOLVE_PLACE_REGS)
+  if (opt.placement < BSOLVE_PLACE_AUTO || opt.placement > BSOLVE_PLACE_CLUSTER)
     return fail(BSOLVE_ERR_INVALID, "bad placement %d", opt.placement);
   if (opt.stop != BSOLVE_STOP_REL_B && opt.stop != BSOLVE_STOP_ABS)
     return fail(BSOLVE_ERR_INVALID, "bad stop mode %d", opt.stop);
@@ -396,10 +414,65 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->num_sms = prop.multiProcessorCount;
   const int smem_optin = (int)prop.sharedMemPerBlockOptin;
 
+  // ---- cluster plan: one system per cluster of C CTAs x 1024 rows ---------
+  // (DESIGN.md "Kernels" 8).  Auto for 9-point stencils with n > 1024.
+  {
+    const int rpc = 1024;
+    const int c = (n + rpc - 1) / rpc;
+    const int last = n - (c - 1) * rpc;
+    const bool cl_ok = h->kfmt == FMT_DIA && W == 9 && n > rpc && c <= 8 && n % 2 == 0 &&
+                       h->guard <= last && (opt.block_threads == 0 || opt.block_threads == 128);
+    const bool want = opt.placement == BSOLVE_PLACE_CLUSTER ||
+                      (opt.placement == BSOLVE_PLACE_AUTO && cl_ok);
+    if (want) {
+      if (!cl_ok)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                              "cluster placement needs a 9-point stencil (DIA) pattern with even "
+                              "1024 < n <= 8192 and stencil reach <= the last CTA's rows"));
+      const int kr = opt.reg_slots ? opt.reg_slots : 4;
+      h->cvar = find_cvariant(c, kr);
+      if (!h->cvar)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no cluster variant for C=%d reg_slots=%d",
+                              c, kr));
+      h->cluster = c;
+      h->place = PLACE_CLUSTER;
+      h->nt = 128;
+      h->r = 8;
+      h->n_pad = (n + 1) & ~1;
+      h->smem_vals = 9 * rpc;
+      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 16;
+      if (h->smem_bytes > smem_optin)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster plan needs %d B of SMEM",
+                              h->smem_bytes));
+      ce = cudaFuncSetAttribute((const void *)h->cvar->fn,
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
+      if (ce != cudaSuccess)
+        return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(c * 64);
+      cfg.blockDim = dim3(128);
+      cfg.dynamicSmemBytes = h->smem_bytes;
+      cudaLaunchAttribute at;
+      at.id = cudaLaunchAttributeClusterDimension;
+      at.val.clusterDim.x = c;
+      at.val.clusterDim.y = 1;
+      at.val.clusterDim.z = 1;
+      cfg.attrs = &at;
+      cfg.numAttrs = 1;
+      int ncl = 0;
+      ce = cudaOccupancyMaxActiveClusters(&ncl, (const void *)h->cvar->fn, &cfg);
+      if (ce != cudaSuccess || ncl < 1)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster of %d CTAs cannot be resident: %s",
+                              c, cudaGetErrorString(ce)));
+      h->ctas_per_sm = std::max(1, ncl * c / h->num_sms);
+      h->grid_persist = ncl;
+    }
+  }
   // rows per thread / CTA size.  Auto: 9-point stencils (DIA) up to 1024 rows
   // take the hybrid 128 threads x 8 rows with 4 off-diagonal slots in
   // registers (measured fastest on B200, DESIGN.md perf log); otherwise 256
   // threads (2 CTAs per SM at <= 128 regs/thread), 512 for 1025..2048 rows.
+  if (h->place != PLACE_CLUSTER) {
   int nt = opt.block_threads;
   int kreg = opt.reg_slots;
   const bool stencil9 = h->kfmt == FMT_DIA && W == 9 && n <= 1024;
@@ -494,6 +567,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   if (h->ctas_per_sm < 1)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "kernel variant cannot be resident on an SM"));
   h->grid_persist = h->num_sms * h->ctas_per_sm;
+  }  // single-CTA plans
 
   // ---- device copy of the pattern ------------------------------------------
   std::vector<int32_t> rp(row_ptr, row_ptr + n + 1);
@@ -538,14 +612,18 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->ell_width = h->W;
   info->format = h->fmt == FMT_ELL ? BSOLVE_FMT_ELL : BSOLVE_FMT_CSR;
   info->placement = h->place == PLACE_SMEM ? BSOLVE_PLACE_SMEM
-                    : h->place == PLACE_REGS ? BSOLVE_PLACE_REGS : BSOLVE_PLACE_STREAM;
+                    : h->place == PLACE_REGS    ? BSOLVE_PLACE_REGS
+                    : h->place == PLACE_CLUSTER ? BSOLVE_PLACE_CLUSTER
+                                                : BSOLVE_PLACE_STREAM;
   info->block_threads = h->nt;
   info->rows_per_thread = h->r;
   info->smem_bytes = h->smem_bytes;
   info->ctas_per_sm = h->ctas_per_sm;
   info->num_sms = h->num_sms;
-  info->grid = h->place == PLACE_REGS ? (int)std::min<long long>(h->grid_persist, h->batch)
-                                      : h->batch;
+  info->grid = h->place == PLACE_REGS      ? (int)std::min<long long>(h->grid_persist, h->batch)
+               : h->place == PLACE_CLUSTER ? h->batch * h->cluster
+                                           : h->batch;
+  info->cluster = h->cluster;
   info->kl = h->kl;
   info->ku = h->ku;
   info->device = h->device;
@@ -602,7 +680,24 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
-  if (h->place == PLACE_REGS && aligned) {
+  if (h->place == PLACE_CLUSTER) {
+    if ((reinterpret_cast<uintptr_t>(values) & 15u) != 0)
+      return fail(BSOLVE_ERR_INVALID, "the cluster plan needs 16-byte aligned values (TMA)");
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)count * (unsigned)h->cluster);
+    cfg.blockDim = dim3(h->nt);
+    cfg.dynamicSmemBytes = h->smem_bytes;
+    cfg.stream = stream;
+    cudaLaunchAttribute at;
+    at.id = cudaLaunchAttributeClusterDimension;
+    at.val.clusterDim.x = h->cluster;
+    at.val.clusterDim.y = 1;
+    at.val.clusterDim.z = 1;
+    cfg.attrs = &at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, h->cvar->fn, P);
+    if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "cluster launch: %s", cudaGetErrorString(e));
+  } else if (h->place == PLACE_REGS && aligned) {
     const int grid = (int)std::min<long long>(h->grid_persist, count);
     h->pvar->fn<<<grid, h->nt, h->smem_bytes, stream>>>(P, h->d_ctr);
   } else {

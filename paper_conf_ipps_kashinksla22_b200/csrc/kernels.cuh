@@ -21,6 +21,7 @@
 //    arithmetic), and reductions that spend as few shuffles as possible.
 #pragma once
 #include <cstdint>
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 namespace bsolve {
@@ -30,7 +31,7 @@ namespace bsolve {
 // in every row r, the entry of column r + d_k (the host detects this for
 // stencil patterns): the gather address is row + d_k with d_k uniform.
 enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
-enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3 };
+enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3, PLACE_CLUSTER = 4 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
 constexpr int kMaxW = 16;
@@ -216,8 +217,8 @@ template <int FMT, int PLACE, int WB, bool EXACT, int R, int KREG, int NB>
 __device__ __forceinline__ void spmv_block(const double *__restrict__ V,
                                            const unsigned char *gb, const SolveParams &P,
                                            const RowMeta<FMT, WB, R, KREG> &m,
-                                           const double (&own)[R], double (&y)[R]) {
-  const int n = P.n;
+                                           const double (&own)[R], double (&y)[R],
+                                           int vstride) {
   double acc[R];
 #pragma unroll
   for (int j = 0; j < NB; ++j) acc[j] = (FMT == FMT_CSR) ? 0.0 : m.a0[j] * own[j];  // slot 0
@@ -246,7 +247,7 @@ __device__ __forceinline__ void spmv_block(const double *__restrict__ V,
         if (k <= KREG) {
           a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];  // slots 1..KREG: registers
         } else {
-          const double *a_p = V + m.vbase[j] + k * n;
+          const double *a_p = V + m.vbase[j] + k * vstride;
           a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
         }
         acc[j] = fma(a, g, acc[j]);
@@ -261,13 +262,17 @@ template <int FMT, int PLACE, int WB, bool EXACT, int R, int NT, int KREG>
 __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
                                           const unsigned char *gb, const SolveParams &P,
                                           const RowMeta<FMT, WB, R, KREG> &m,
-                                          const double (&own)[R], double (&y)[R]) {
+                                          const double (&own)[R], double (&y)[R], int nrows,
+                                          int vstride) {
+  // nrows: rows owned by this CTA (= n unless a cluster splits the system);
+  // vstride: doubles between two ELL slots of the staged values
   const int wrow0 = threadIdx.x & ~31;
-  const int n = P.n;
+  const int n = nrows;
   if (wrow0 + (R - 1) * NT < n) {
-    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, R>(V, gb, P, m, own, y);
+    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, R>(V, gb, P, m, own, y, vstride);
   } else if (R > 1 && wrow0 + (R - 2) * NT < n) {
-    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, (R > 1 ? R - 1 : 1)>(V, gb, P, m, own, y);
+    spmv_block<FMT, PLACE, WB, EXACT, R, KREG, (R > 1 ? R - 1 : 1)>(V, gb, P, m, own, y,
+                                                                     vstride);
   } else {
     // generic tail (small n: several idle row blocks): one block at a time
 #pragma unroll
@@ -298,7 +303,7 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
             if (k <= KREG) {
               a = m.vreg[j][k - 1 < 0 ? 0 : k - 1];
             } else {
-              const double *a_p = V + m.vbase[j] + k * n;
+              const double *a_p = V + m.vbase[j] + k * vstride;
               a = (PLACE == PLACE_STREAM) ? __ldg(a_p) : *a_p;
             }
             acc = fma(a, g, acc);
@@ -311,6 +316,28 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
 }
 
 // ------------------------------------------------------------ the solver --
+// Communication policy of the single-CTA kernels: the gather buffer and the
+// reductions are CTA-local.
+template <int R, int NT>
+struct CtaComm {
+  double *sg;    // gather body
+  double *sred;  // reduction scratch
+  int buf;
+  const bool (&act)[R];
+  __device__ __forceinline__ CtaComm(double *sg_, double *sred_, const bool (&act_)[R])
+      : sg(sg_), sred(sred_), buf(0), act(act_) {}
+  __device__ __forceinline__ int grow(int j) const { return threadIdx.x + j * NT; }
+  __device__ __forceinline__ bool leader() const { return threadIdx.x == 0; }
+  __device__ __forceinline__ void publish(int j, double v) {
+    if (act[j]) sg[threadIdx.x + j * NT] = v;
+  }
+  __device__ __forceinline__ void sync() { __syncthreads(); }
+  template <int K>
+  __device__ __forceinline__ void sum(double (&v)[K]) {
+    block_sum<K, NT / 32>(v, sred, buf, threadIdx.x & 31, threadIdx.x >> 5);
+  }
+};
+
 // Algorithm 1 for ONE system, shared by both kernels.
 //   on entry: x = x0 (or 0), r = b, d = Jacobi diagonal, act = row < n;
 //   spmv(own, y): y = A g for this thread's rows, where g was published to
@@ -318,13 +345,11 @@ __device__ __forceinline__ void spmv_rows(const double *__restrict__ V,
 //   bv: b in registers (B_IN_REGS) for the true residual, else re-read bsys.
 // Writes x, iters, resnorm, status of system `sys`.  Every path executes at
 // least one block_sum (one barrier) after entry.
-template <int R, int NT, bool B_IN_REGS, int ROUNDS, class SpMV>
+template <int R, int NT, bool B_IN_REGS, int ROUNDS, class Comm, class SpMV>
 __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sys, double (&x)[R],
                                               double (&r)[R], const double (&d)[R],
                                               const bool (&act)[R], const double (&bv)[R],
-                                              double *sg, double *sred, int &buf, SpMV &&spmv) {
-  constexpr int NWARP = NT / 32;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+                                              Comm &comm, SpMV &&spmv) {
   const int n = P.n;
   const double *bsys = P.b + sys * n;
   double rh[R], p[R], v[R];
@@ -336,8 +361,8 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   if (P.x0) {
 #pragma unroll
     for (int j = 0; j < R; ++j)
-      if (act[j]) sg[tid + j * NT] = x[j];
-    __syncthreads();
+      comm.publish(j, x[j]);
+    comm.sync();
     double q[R];
     spmv(x, q);
 #pragma unroll
@@ -350,7 +375,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
     v[j] = 0.0;
     red3[1] += r[j] * r[j];
   }
-  block_sum<2, NWARP>(red3, sred, buf, lane, warp);
+  comm.template sum<2>(red3);
   const double bnorm = sqrt(red3[0]);
   const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
   double rnorm = sqrt(red3[1]);
@@ -360,8 +385,8 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   if (P.stop == STOP_REL_B && bnorm == 0.0) {
 #pragma unroll
     for (int j = 0; j < R; ++j)
-      if (act[j]) xout[tid + j * NT] = 0.0;
-    if (tid == 0) {
+      if (act[j]) xout[comm.grow(j)] = 0.0;
+    if (comm.leader()) {
       P.iters[sys] = 0;
       P.resnorm[sys] = 0.0;
       if (P.status) P.status[sys] = SYS_CONVERGED;
@@ -373,17 +398,17 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
     // publish x, q = b - A x, returns ||q||_2 (one more barrier)
 #pragma unroll
     for (int j = 0; j < R; ++j)
-      if (act[j]) sg[tid + j * NT] = x[j];
-    __syncthreads();
+      comm.publish(j, x[j]);
+    comm.sync();
     double tr[1] = {0.0};
     spmv(x, q);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
-      const double bj = B_IN_REGS ? bv[j] : (act[j] ? __ldg(bsys + tid + j * NT) : 0.0);
+      const double bj = B_IN_REGS ? bv[j] : (act[j] ? __ldg(bsys + comm.grow(j)) : 0.0);
       q[j] = act[j] ? bj - q[j] : 0.0;
       tr[0] += q[j] * q[j];
     }
-    block_sum<1, NWARP>(tr, sred, buf, lane, warp);
+    comm.template sum<1>(tr);
     return tr[0];
   };
 
@@ -420,9 +445,9 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       for (int j = 0; j < R; ++j) {
         p[j] = r[j] + beta * (p[j] - omega * v[j]);
         ph[j] = d[j] * p[j];
-        if (act[j]) sg[tid + j * NT] = ph[j];
+        comm.publish(j, ph[j]);
       }
-      __syncthreads();
+      comm.sync();
       // a6: v = A p^
       spmv(ph, v);
       ++it;
@@ -430,7 +455,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       double rv[1] = {0.0};
 #pragma unroll
       for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
-      block_sum<1, NWARP>(rv, sred, buf, lane, warp);
+      comm.template sum<1>(rv);
       if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
       alpha = rho / rv[0];                                 // R3
       // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
@@ -442,9 +467,9 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
         s[j] = r[j] - alpha * v[j];
         ts[2] += s[j] * s[j];
         sh[j] = d[j] * s[j];
-        if (act[j]) sg[tid + j * NT] = sh[j];
+        comm.publish(j, sh[j]);
       }
-      __syncthreads();  // publish s^
+      comm.sync();  // publish s^
       // a9: t = A s^ (speculative when stop test 2 fires)
       double t[R];
       spmv(sh, t);
@@ -453,7 +478,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
         ts[0] += t[j] * s[j];
         ts[1] += t[j] * t[j];
       }
-      block_sum<3, NWARP>(ts, sred, buf, lane, warp);
+      comm.template sum<3>(ts);
       if (sqrt(ts[2]) < tau) {                             // stop test 2
 #pragma unroll
         for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
@@ -473,7 +498,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       }
       rho_old = rho;
       // next iteration's ||r|| and rho = r^ . r in the same single barrier
-      block_sum<2, NWARP>(rr, sred, buf, lane, warp);
+      comm.template sum<2>(rr);
       rnorm = sqrt(rr[0]);
       rho = rr[1];
     }
@@ -485,7 +510,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
         if (!have_rnorm) {  // rare: settle stop test 1 before declaring breakdown
           double rr[1];
           rr[0] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
-          block_sum<1, NWARP>(rr, sred, buf, lane, warp);
+          comm.template sum<1>(rr);
           rnorm = sqrt(rr[0]);
           have_rnorm = true;
           continue;
@@ -500,16 +525,16 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       for (int j = 0; j < R; ++j) {
         p[j] = r[j] + beta * (p[j] - omega * v[j]);
         ph[j] = d[j] * p[j];
-        if (act[j]) sg[tid + j * NT] = ph[j];
+        comm.publish(j, ph[j]);
       }
-      __syncthreads();
+      comm.sync();
       // a6: v = A p^
       spmv(ph, v);
       // a7: r^.v, and ||r|| of the current r for the deferred stop test 1
       double red[2];
       red[0] = rows_sum<R>([&](int j) { return rh[j] * v[j]; });
       red[1] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
-      block_sum<2, NWARP>(red, sred, buf, lane, warp);
+      comm.template sum<2>(red);
       if (!have_rnorm) {
         rnorm = sqrt(red[1]);
         if (rnorm < tau) { exit_kind = 1; break; }         // stop test 1, deferred
@@ -525,9 +550,9 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       for (int j = 0; j < R; ++j) {
         s[j] = r[j] - alpha * v[j];
         sh[j] = d[j] * s[j];
-        if (act[j]) sg[tid + j * NT] = sh[j];
+        comm.publish(j, sh[j]);
       }
-      __syncthreads();  // publish s^
+      comm.sync();  // publish s^
       // a9: t = A s^ (speculative when stop test 2 fires)
       double t[R];
       spmv(sh, t);
@@ -537,7 +562,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       ts[2] = rows_sum<R>([&](int j) { return s[j] * s[j]; });
       ts[3] = rows_sum<R>([&](int j) { return rh[j] * s[j]; });
       ts[4] = rows_sum<R>([&](int j) { return rh[j] * t[j]; });
-      block_sum<5, NWARP>(ts, sred, buf, lane, warp);
+      comm.template sum<5>(ts);
       if (sqrt(ts[2]) < tau) {                             // stop test 2
 #pragma unroll
         for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
@@ -580,7 +605,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
 
   if (final_res < 0.0) {
     // final TRUE residual ||b - A x|| (always reported, R4)
-    __syncthreads();  // previous gather readers done before overwriting
+    comm.sync();  // previous gather readers done before overwriting
     double q[R];
     final_res = sqrt(true_residual(q));
   }
@@ -590,8 +615,8 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   }
 #pragma unroll
   for (int j = 0; j < R; ++j)
-    if (act[j]) xout[tid + j * NT] = x[j];
-  if (tid == 0) {
+    if (act[j]) xout[comm.grow(j)] = x[j];
+  if (comm.leader()) {
     P.iters[sys] = it;
     P.resnorm[sys] = final_res;
     if (P.status) P.status[sys] = static_cast<int8_t>(st);
@@ -705,10 +730,10 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     d[j] = (a != 0.0) ? 1.0 / a : 1.0;
   }
 
-  int buf = 0;
+  CtaComm<R, NT> comm(sg, sred, m.act);
   bicgstab_core<R, NT, false, 3>(
-      P, sys, x, r, d, m.act, r, sg, sred, buf, [&](const double(&own)[R], double(&y)[R]) {
-        spmv_rows<FMT, PLACE, WB, EXACT, R, NT, KREG>(V, gb, P, m, own, y);
+      P, sys, x, r, d, m.act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
+        spmv_rows<FMT, PLACE, WB, EXACT, R, NT, KREG>(V, gb, P, m, own, y, P.n, P.n);
       });
 }
 
@@ -796,7 +821,7 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
   __syncthreads();
   long long cur = *s_next;
   uint32_t phase = 0;
-  int buf = 0;
+  CtaComm<R, NT> comm(sg, sred, m.act);
   while (cur < batch) {
     mbar_wait_parity(mbar, phase);
     phase ^= 1u;
@@ -824,9 +849,9 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
       }
     }
     bicgstab_core<R, NT, true, 2>(
-        P, cur, x, r, d, m.act, bv, sg, sred, buf,
+        P, cur, x, r, d, m.act, bv, comm,
         [&](const double(&own)[R], double(&y)[R]) {
-          spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, WB - 1>(sval, gb, P, m, own, y);
+          spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, WB - 1>(sval, gb, P, m, own, y, P.n, P.n);
         });
     cur = *s_next;  // written before the core's first barrier
   }
@@ -840,6 +865,173 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
       atomicExch(ctr + 1, 0ull);
     }
   }
+}
+
+// ------------------------------------------ thread-block cluster per system --
+// Systems too large for one CTA (n > 1024 rows, e.g. the 63x64 velocity
+// grid, n = 4032) are split over a cluster of C CTAs
+// (one per 1024 rows, C <= 8), all on one GPC, which exchange through
+// distributed shared memory (DSMEM):
+//  * each CTA TMA-stages the values of ITS rows (one bulk copy per ELL slot)
+//    and keeps them in SMEM / registers as the single-CTA hybrid does;
+//  * publishing p^ / s^ writes each row locally and, for the first / last G
+//    rows of the CTA (G = max |stencil offset|), also into the halo of the
+//    left / right neighbour's gather buffer (st.shared::cluster); the
+//    cluster barrier that follows makes them visible, so every SpMV reads
+//    only local SMEM;
+//  * a reduction publishes each warp partial into every CTA's scratch and
+//    crosses ONE cluster barrier; every thread then adds the C x NWARP
+//    partials in the same fixed order (bitwise-identical scalars in the
+//    whole cluster, uniform control flow).
+template <int R, int NT, int C>
+struct ClusterComm {
+  static constexpr int NWARP = NT / 32;
+  static constexpr int RPC = R * NT;  // rows per CTA
+  cooperative_groups::cluster_group cl;
+  double *sg;    // local gather body (local row 0)
+  double *sred;  // scratch [2][8][C * NWARP]
+  double *left, *right;  // neighbours' gather bodies (DSMEM) or nullptr
+  int buf, rank, row0, nloc, G;
+  const bool (&act)[R];
+  __device__ __forceinline__ ClusterComm(cooperative_groups::cluster_group c, double *sg_,
+                                         double *sred_, int rank_, int nloc_, int G_,
+                                         const bool (&act_)[R])
+      : cl(c), sg(sg_), sred(sred_), buf(0), rank(rank_), row0(rank_ * RPC), nloc(nloc_),
+        G(G_), act(act_) {
+    left = rank > 0 ? cl.map_shared_rank(sg, rank - 1) : nullptr;
+    right = rank < C - 1 ? cl.map_shared_rank(sg, rank + 1) : nullptr;
+  }
+  __device__ __forceinline__ int grow(int j) const { return row0 + threadIdx.x + j * NT; }
+  __device__ __forceinline__ bool leader() const { return rank == 0 && threadIdx.x == 0; }
+  __device__ __forceinline__ void publish(int j, double v) {
+    const int i = threadIdx.x + j * NT;
+    if (act[j]) {
+      sg[i] = v;
+      if (i < G && left) left[RPC + i] = v;                // my first rows: left's right halo
+      if (i >= nloc - G && right) right[i - nloc] = v;      // my last rows: right's left halo
+    }
+  }
+  __device__ __forceinline__ void sync() { cl.sync(); }
+  template <int K>
+  __device__ __forceinline__ void sum(double (&v)[K]) {
+    static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    constexpr int KP = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
+    constexpr int SPAN = 32 / KP;
+    double a[KP];
+#pragma unroll
+    for (int i = 0; i < KP; ++i) a[i] = i < K ? v[i] : 0.0;
+#pragma unroll
+    for (int cnt = KP, o = 16; cnt > 1; cnt >>= 1, o >>= 1) {
+      const bool hi = lane & o;
+#pragma unroll
+      for (int i = 0; i < cnt / 2; ++i) {
+        const double send = hi ? a[i] : a[i + cnt / 2];
+        const double keep = hi ? a[i + cnt / 2] : a[i];
+        a[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+      }
+    }
+#pragma unroll
+    for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
+    constexpr int P_ = C * NWARP;  // partials per value
+    double *S = sred + buf * (8 * P_);
+    const int q = lane / SPAN;
+    if ((lane % SPAN) == 0 && q < K) {
+      const int slot = q * P_ + rank * NWARP + warp;
+#pragma unroll
+      for (int r = 0; r < C; ++r) cl.map_shared_rank(S, r)[slot] = a[0];
+    }
+    cl.sync();
+    double part[K][P_];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const double2 *S2 = reinterpret_cast<const double2 *>(S + k * P_);
+#pragma unroll
+      for (int w = 0; w < P_ / 2; ++w) {
+        const double2 qq = S2[w];
+        part[k][2 * w] = qq.x;
+        part[k][2 * w + 1] = qq.y;
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < K; ++k) v[k] = tree_sum<P_>(part[k]);
+    buf ^= 1;
+  }
+};
+
+// One system per cluster of C CTAs; DIA (stencil) values, W = 9.
+//   SMEM per CTA: [values: W x RPC doubles, slot-major] [gather: G | RPC | G]
+//                 [scratch: 2 x 8 x C x NWARP] [mbarrier]
+template <int FMT, int WB, bool EXACT, int R, int NT, int KREG, int C>
+__global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolveParams P) {
+  static_assert(FMT == FMT_DIA, "cluster kernel: DIA addressing only");
+  constexpr int NWARP = NT / 32;
+  constexpr int RPC = R * NT;
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  const int rank = static_cast<int>(cl.block_rank());
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sgf = sval + WB * RPC;
+  double *sg = sgf + P.guard;
+  double *sred = sgf + RPC + 2 * P.guard;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * C * NWARP);
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+
+  const int tid = threadIdx.x;
+  const int n = P.n;
+  const long long sys = blockIdx.x / C;
+  const int row0 = rank * RPC;
+  const int nloc = min(RPC, n - row0);  // host guarantees nloc >= 1, even
+  // ---- stage this CTA's rows of every ELL slot (TMA, one copy per slot) ----
+  if (tid == 0) {
+    mbar_init(mbar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (tid == 0) {
+    const uint32_t bytes = static_cast<uint32_t>(nloc) * 8u;
+    mbar_arrive_expect_tx(mbar, bytes * (EXACT ? WB : P.W));
+    const double *gsys = P.values + sys * P.sys_stride + row0;
+    for (int k = 0; k < (EXACT ? WB : P.W); ++k)
+      tma_bulk_g2s(sval + k * RPC, gsys + (long long)k * n, bytes, mbar);
+  }
+  // zero guards: global boundary halos and the unused tail of the last CTA
+  for (int i = tid; i < P.guard; i += NT) {
+    if (rank == 0) sgf[i] = 0.0;
+    if (rank == C - 1) sg[RPC + i] = 0.0;
+  }
+  for (int i = nloc + tid; i < RPC; i += NT) sg[i] = 0.0;
+
+  RowMeta<FMT, WB, R, KREG> m;
+  double x[R], r[R], d[R];
+  const double *bsys = P.b + sys * n;
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    const int li = tid + j * NT;
+    m.act[j] = li < nloc;
+    m.vbase[j] = li < nloc ? li : nloc - 1;
+    m.vlen[j] = 0;
+    m.a0[j] = 0.0;
+    r[j] = m.act[j] ? __ldg(bsys + row0 + li) : 0.0;
+    x[j] = (m.act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + li) : 0.0;
+  }
+  cl.sync();  // every CTA of the cluster runs (DSMEM is live) and zeroed its guards
+  mbar_wait_parity(mbar, 0);
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    const double a = m.act[j] ? sval[m.vbase[j]] : 0.0;  // slot 0 = diagonal
+    m.a0[j] = a;
+    d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+#pragma unroll
+    for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k) m.vreg[j][k] = sval[m.vbase[j] + (k + 1) * RPC];
+  }
+  ClusterComm<R, NT, C> comm(cl, sg, sred, rank, nloc, P.guard, m.act);
+  bicgstab_core<R, NT, false, 3>(
+      P, sys, x, r, d, m.act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
+        spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, KREG>(sval, gb, P, m, own, y, nloc, RPC);
+      });
+  cl.sync();  // peers may write into this CTA's SMEM until they are done
 }
 
 // -------------------------------------------------- standalone batched SpMV --

@@ -371,3 +371,37 @@ def test_rows_beyond_capacity_rejected():
             B = X.make_batch(0, 2, pattern=pat)
             g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, block_threads=bt)
             compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+
+
+# ------------------------------------------------ cluster (n > 1024) plan --
+@pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4), (96, 80, 8)])
+def test_cluster_large_systems(nx, ny, C):
+    """BASELINE configs[4]: 63x64 grid (n = 4032) and other sizes split over a
+    thread-block cluster of C CTAs (halo exchange + reductions via DSMEM)."""
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 6, pattern=pat)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b)
+    assert g["info"]["placement"] == 4 and g["info"]["cluster"] == C
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+
+
+def test_cluster_warm_start_ill_conditioned_and_deterministic():
+    pat = X.stencil_pattern(64, 63)
+    ill = X.Species(X.ELECTRON_K, cross=0.0, margin=1e-2)
+    B = X.make_batch(0, 8, pattern=pat, electron=ill)
+    p = pat
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3000)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3000)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o,
+            iter_tol=max(10, int(0.5 * o["iters"].max())))
+    # warm start from a perturbed direct solution
+    xd = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b)
+    x0 = xd * (1 + 1e-5)
+    g2 = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3000)
+    o2 = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3000)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g2, o=o2, xd=xd,
+            iter_tol=max(10, int(0.5 * o2["iters"].max())))
+    # bitwise identical across runs and batch slicing
+    g3 = gpu_solve(p.row_ptr, p.col_idx, B.values[3:], B.b[3:], maxiter=3000)
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(g[k][3:], g3[k])
