@@ -421,14 +421,15 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const int c = (n + rpc - 1) / rpc;
     const int last = n - (c - 1) * rpc;
     const bool cl_ok = h->kfmt == FMT_DIA && W == 9 && n > rpc && c <= 8 && n % 2 == 0 &&
-                       h->guard <= last && (opt.block_threads == 0 || opt.block_threads == 128);
+                       last >= 1 && h->guard <= rpc &&
+                       (opt.block_threads == 0 || opt.block_threads == 128);
     const bool want = opt.placement == BSOLVE_PLACE_CLUSTER ||
                       (opt.placement == BSOLVE_PLACE_AUTO && cl_ok);
     if (want) {
       if (!cl_ok)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                               "cluster placement needs a 9-point stencil (DIA) pattern with even "
-                              "1024 < n <= 8192 and stencil reach <= the last CTA's rows"));
+                              "1024 < n <= 8192 and stencil reach <= 1024 rows"));
       const int kr = opt.reg_slots ? opt.reg_slots : 4;
       h->cvar = find_cvariant(c, kr);
       if (!h->cvar)

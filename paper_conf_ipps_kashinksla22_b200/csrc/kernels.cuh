@@ -1002,6 +1002,10 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
     if (rank == C - 1) sg[RPC + i] = 0.0;
   }
   for (int i = nloc + tid; i < RPC; i += NT) sg[i] = 0.0;
+  if (rank < C - 1) {  // right-halo entries of rows >= n (next CTA shorter than the reach)
+    const int nnext = min(RPC, n - (rank + 1) * RPC);
+    for (int i = nnext + tid; i < P.guard; i += NT) sg[RPC + i] = 0.0;
+  }
 
   RowMeta<FMT, WB, R, KREG> m;
   double x[R], r[R], d[R];
