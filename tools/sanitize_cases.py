@@ -1,0 +1,48 @@
+"""Small solves through every kernel family, for compute-sanitizer runs:
+  compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_cases.py
+Exits non-zero if any result fails the parity bar against the direct solve."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import oracle as O  # noqa: E402  (test infrastructure: checks the results)
+import xgcgen as X  # noqa: E402
+from paper_conf_ipps_kashinksla22_b200 import Solver  # noqa: E402
+
+CASES = [
+    ("hybrid 128x8 DIA (default 992)", dict(nx=32, ny=31), dict()),
+    ("smem 256x4 DIA", dict(nx=32, ny=31), dict(block_threads=256)),
+    ("csr smem", dict(nx=32, ny=31), dict(format="csr")),
+    ("stream ell", dict(nx=32, ny=31), dict(placement="stream")),
+    ("persistent regs", dict(nx=32, ny=31), dict(placement="regs")),
+    ("cluster C=4 (n=4032)", dict(nx=64, ny=63), dict()),
+    ("cluster C=3 (n=2112)", dict(nx=64, ny=33), dict()),
+]
+
+
+def main():
+    batch = int(os.environ.get("SAN_BATCH", "3"))
+    bad = 0
+    for name, grid, opts in CASES:
+        pat = X.stencil_pattern(**grid)
+        B = X.make_batch(0, batch, pattern=pat)
+        S = Solver(pat.row_ptr, pat.col_idx, batch, **opts)
+        vals = S.ell_values(B.values) if S.format == "ell" else B.values
+        x, it, res, st = S.run(torch.from_numpy(vals).cuda(), torch.from_numpy(B.b).cuda())
+        torch.cuda.synchronize()
+        x = x.cpu().numpy()
+        xd = O.batch_banded(pat.row_ptr, pat.col_idx, B.values, B.b)
+        err = np.max(np.linalg.norm(x - xd, axis=1) / np.linalg.norm(xd, axis=1))
+        ok = err <= 1e-8 and bool(np.all(st.cpu().numpy() == 0))
+        bad += not ok
+        print(f"{name:32s} iters={it.cpu().tolist()} fwd_err={err:.2e} {'ok' if ok else 'FAIL'}",
+              flush=True)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
