@@ -441,7 +441,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->r = 8;
       h->n_pad = (n + 1) & ~1;
       h->smem_vals = 9 * rpc;
-      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 16;
+      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 4 * 8;  // + 4 mbarriers
       if (h->smem_bytes > smem_optin)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster plan needs %d B of SMEM",
                               h->smem_bytes));

@@ -94,6 +94,30 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity)
       : "memory");
 }
 
+// Distributed shared memory helpers (thread-block clusters).
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+// 8-byte store into a (possibly remote) CTA's SMEM that completes 8 bytes
+// of transaction count on that CTA's mbarrier.
+__device__ __forceinline__ void st_async_f64(uint32_t raddr, double v, uint32_t rbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b64 [%0], %1, [%2];" ::"r"(
+                   raddr),
+               "l"(__double_as_longlong(v)), "r"(rbar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity_cluster(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n"
+      "WAITC_%=:\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAITC_%=;\n}" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
+
 __device__ __forceinline__ bool bad(double v) { return v == 0.0 || !isfinite(v); }
 
 // Sum over this thread's R rows of f(j) with two interleaved accumulators
@@ -876,42 +900,65 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
 //    and keeps them in SMEM / registers as the single-CTA hybrid does;
 //  * publishing p^ / s^ writes each row locally and, for the first / last G
 //    rows of the CTA (G = max |stencil offset|), also into the halo of the
-//    left / right neighbour's gather buffer (st.shared::cluster); the
-//    cluster barrier that follows makes them visible, so every SpMV reads
-//    only local SMEM;
-//  * a reduction publishes each warp partial into every CTA's scratch and
-//    crosses ONE cluster barrier; every thread then adds the C x NWARP
-//    partials in the same fixed order (bitwise-identical scalars in the
-//    whole cluster, uniform control flow).
+//    left / right neighbour's gather buffer with st.async, which completes
+//    transaction bytes on the neighbour's halo mbarrier: point-to-point
+//    synchronisation, no cluster barrier; every SpMV reads only local SMEM;
+//  * a reduction st.async's each warp partial into every CTA's scratch and
+//    waits on its own mbarrier for the C x NWARP partials, then every
+//    thread adds them in the same fixed order (bitwise-identical scalars in
+//    the whole cluster, uniform control flow).  cluster.sync() is used only
+//    at kernel entry and exit.
 template <int R, int NT, int C>
 struct ClusterComm {
   static constexpr int NWARP = NT / 32;
   static constexpr int RPC = R * NT;  // rows per CTA
-  cooperative_groups::cluster_group cl;
-  double *sg;    // local gather body (local row 0)
-  double *sred;  // scratch [2][8][C * NWARP]
-  double *left, *right;  // neighbours' gather bodies (DSMEM) or nullptr
-  int buf, rank, row0, nloc, G;
+  double *sg;            // local gather body (local row 0)
+  double *sred;          // scratch [2][8][C * NWARP]
+  uint64_t *hbar;        // halo mbarrier (complete_tx from the neighbours' st.async)
+  uint64_t *rbar;        // reduction mbarriers [2]
+  uint32_t left_sg, right_sg, left_hbar, right_hbar;  // neighbours (shared::cluster)
+  uint32_t sred_s, rbar_s;                             // own shared::cta addresses
+  uint32_t hphase = 0, rphase = 0;                     // phase parity bits
+  int buf = 0, rank, nloc, G, halo_bytes;
   const bool (&act)[R];
-  __device__ __forceinline__ ClusterComm(cooperative_groups::cluster_group c, double *sg_,
-                                         double *sred_, int rank_, int nloc_, int G_,
-                                         const bool (&act_)[R])
-      : cl(c), sg(sg_), sred(sred_), buf(0), rank(rank_), row0(rank_ * RPC), nloc(nloc_),
-        G(G_), act(act_) {
-    left = rank > 0 ? cl.map_shared_rank(sg, rank - 1) : nullptr;
-    right = rank < C - 1 ? cl.map_shared_rank(sg, rank + 1) : nullptr;
+  __device__ __forceinline__ ClusterComm(double *sg_, double *sred_, uint64_t *bars, int rank_,
+                                         int n, int G_, const bool (&act_)[R])
+      : sg(sg_), sred(sred_), hbar(bars), rbar(bars + 1), rank(rank_),
+        nloc(min(RPC, n - rank_ * RPC)), G(G_), act(act_) {
+    const uint32_t sg_s = smem_addr(sg), hb_s = smem_addr(hbar);
+    left_sg = rank > 0 ? mapa_u32(sg_s, rank - 1) : 0u;
+    left_hbar = rank > 0 ? mapa_u32(hb_s, rank - 1) : 0u;
+    right_sg = rank < C - 1 ? mapa_u32(sg_s, rank + 1) : 0u;
+    right_hbar = rank < C - 1 ? mapa_u32(hb_s, rank + 1) : 0u;
+    sred_s = smem_addr(sred);
+    rbar_s = smem_addr(rbar);
+    // halo rows this CTA receives: the left neighbour's last G rows and the
+    // right neighbour's first min(G, its rows) rows
+    const int nright = rank < C - 1 ? min(RPC, n - (rank + 1) * RPC) : 0;
+    halo_bytes = 8 * ((rank > 0 ? G : 0) + min(G, nright));
   }
-  __device__ __forceinline__ int grow(int j) const { return row0 + threadIdx.x + j * NT; }
+  __device__ __forceinline__ int grow(int j) const { return rank * RPC + threadIdx.x + j * NT; }
   __device__ __forceinline__ bool leader() const { return rank == 0 && threadIdx.x == 0; }
   __device__ __forceinline__ void publish(int j, double v) {
     const int i = threadIdx.x + j * NT;
     if (act[j]) {
       sg[i] = v;
-      if (i < G && left) left[RPC + i] = v;                // my first rows: left's right halo
-      if (i >= nloc - G && right) right[i - nloc] = v;      // my last rows: right's left halo
+      if (i < G && rank > 0)  // my first rows -> left neighbour's right halo
+        st_async_f64(left_sg + 8u * static_cast<uint32_t>(RPC + i), v, left_hbar);
+      if (i >= nloc - G && rank < C - 1)  // my last rows -> right neighbour's left halo
+        st_async_f64(right_sg + 8u * static_cast<uint32_t>(i - nloc), v, right_hbar);
     }
   }
-  __device__ __forceinline__ void sync() { cl.sync(); }
+  // local writes: CTA barrier; neighbours' halo rows: their st.async bytes
+  // complete this CTA's halo mbarrier.  (Two consecutive publishes are always
+  // separated by a reduction that depends on every CTA's SpMV, so a halo is
+  // never overwritten while it is still being gathered.)
+  __device__ __forceinline__ void sync() {
+    if (threadIdx.x == 0) mbar_arrive_expect_tx(hbar, static_cast<uint32_t>(halo_bytes));
+    __syncthreads();
+    mbar_wait_parity_cluster(hbar, hphase);
+    hphase ^= 1u;
+  }
   template <int K>
   __device__ __forceinline__ void sum(double (&v)[K]) {
     static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
@@ -934,14 +981,21 @@ struct ClusterComm {
 #pragma unroll
     for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
     constexpr int P_ = C * NWARP;  // partials per value
-    double *S = sred + buf * (8 * P_);
+    const uint32_t bit = 1u << buf;
+    if (threadIdx.x == 0) mbar_arrive_expect_tx(rbar + buf, K * P_ * 8);
     const int q = lane / SPAN;
     if ((lane % SPAN) == 0 && q < K) {
-      const int slot = q * P_ + rank * NWARP + warp;
+      // every CTA receives every warp partial (one 8-byte st.async each);
+      // a round can only start after the previous one completed everywhere
+      // (each depends on the last result), so double buffering is enough
+      const uint32_t off = static_cast<uint32_t>((buf * 8 * P_ + q * P_ + rank * NWARP + warp) * 8);
 #pragma unroll
-      for (int r = 0; r < C; ++r) cl.map_shared_rank(S, r)[slot] = a[0];
+      for (int r = 0; r < C; ++r)
+        st_async_f64(mapa_u32(sred_s + off, r), a[0], mapa_u32(rbar_s + 8u * buf, r));
     }
-    cl.sync();
+    mbar_wait_parity_cluster(rbar + buf, (rphase & bit) ? 1u : 0u);
+    rphase ^= bit;
+    const double *S = sred + buf * (8 * P_);
     double part[K][P_];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
@@ -984,8 +1038,9 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
   const int row0 = rank * RPC;
   const int nloc = min(RPC, n - row0);  // host guarantees nloc >= 1, even
   // ---- stage this CTA's rows of every ELL slot (TMA, one copy per slot) ----
+  // mbar[0]: TMA, mbar[1]: halo rows, mbar[2..3]: reduction buffers
   if (tid == 0) {
-    mbar_init(mbar, 1);
+    for (int i = 0; i < 4; ++i) mbar_init(mbar + i, 1);
     fence_mbar_init();
   }
   __syncthreads();
@@ -1020,7 +1075,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
     r[j] = m.act[j] ? __ldg(bsys + row0 + li) : 0.0;
     x[j] = (m.act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + li) : 0.0;
   }
-  cl.sync();  // every CTA of the cluster runs (DSMEM is live) and zeroed its guards
+  cl.sync();  // every CTA of the cluster runs (DSMEM and its mbarriers are live)
   mbar_wait_parity(mbar, 0);
 #pragma unroll
   for (int j = 0; j < R; ++j) {
@@ -1030,7 +1085,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
 #pragma unroll
     for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k) m.vreg[j][k] = sval[m.vbase[j] + (k + 1) * RPC];
   }
-  ClusterComm<R, NT, C> comm(cl, sg, sred, rank, nloc, P.guard, m.act);
+  ClusterComm<R, NT, C> comm(sg, sred, mbar + 1, rank, n, P.guard, m.act);
   bicgstab_core<R, NT, false, 3>(
       P, sys, x, r, d, m.act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
         spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, KREG>(sval, gb, P, m, own, y, nloc, RPC);
