@@ -95,16 +95,18 @@ static const PVariant *find_pvariant(int fmt, int r) {
 // Cluster variants (PLACE_CLUSTER): one system per cluster of C CTAs of
 // 128 threads x 8 rows (1024 rows per CTA), DIA, W = 9.
 struct CVariant {
-  int c, kreg;
+  int c, kreg, rounds;
   solve_fn fn;
 };
-#define CV_(C, KR) {C, KR, (solve_fn)bicgstab_cluster_kernel<FMT_DIA, 9, true, 8, 128, KR, C>}
-static const CVariant kCVariants[] = {CV_(2, 4), CV_(3, 4), CV_(4, 4), CV_(5, 4), CV_(6, 4),
-                                      CV_(7, 4), CV_(8, 4), CV_(2, 2), CV_(3, 2), CV_(4, 2),
-                                      CV_(5, 2), CV_(6, 2), CV_(7, 2), CV_(8, 2)};
-static const CVariant *find_cvariant(int c, int kreg) {
+#define CV_(C, KR, RD) \
+  {C, KR, RD, (solve_fn)bicgstab_cluster_kernel<FMT_DIA, 9, true, 8, 128, KR, C, RD>}
+#define CV_ALLC(KR, RD) \
+  CV_(2, KR, RD), CV_(3, KR, RD), CV_(4, KR, RD), CV_(5, KR, RD), CV_(6, KR, RD), \
+      CV_(7, KR, RD), CV_(8, KR, RD)
+static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3), CV_ALLC(2, 2), CV_ALLC(0, 2)};
+static const CVariant *find_cvariant(int c, int kreg, int rounds) {
   for (const CVariant &v : kCVariants)
-    if (v.c == c && v.kreg == kreg) return &v;
+    if (v.c == c && v.kreg == kreg && v.rounds == rounds) return &v;
   return nullptr;
 }
 
@@ -431,7 +433,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                               "cluster placement needs a 9-point stencil (DIA) pattern with even "
                               "1024 < n <= 8192 and stencil reach <= 1024 rows"));
       const int kr = opt.reg_slots ? opt.reg_slots : 4;
-      h->cvar = find_cvariant(c, kr);
+      // iteration schedule (reduction rounds per iteration); developer knob
+      const char *rd_env = getenv("BSOLVE_CLUSTER_ROUNDS");
+      const int rd = rd_env ? atoi(rd_env) : 3;
+      h->cvar = find_cvariant(c, kr, rd);
       if (!h->cvar)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no cluster variant for C=%d reg_slots=%d",
                               c, kr));

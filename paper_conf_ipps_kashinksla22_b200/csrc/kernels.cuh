@@ -1016,7 +1016,7 @@ struct ClusterComm {
 // One system per cluster of C CTAs; DIA (stencil) values, W = 9.
 //   SMEM per CTA: [values: W x RPC doubles, slot-major] [gather: G | RPC | G]
 //                 [scratch: 2 x 8 x C x NWARP] [mbarrier]
-template <int FMT, int WB, bool EXACT, int R, int NT, int KREG, int C>
+template <int FMT, int WB, bool EXACT, int R, int NT, int KREG, int C, int ROUNDS = 3>
 __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolveParams P) {
   static_assert(FMT == FMT_DIA, "cluster kernel: DIA addressing only");
   constexpr int NWARP = NT / 32;
@@ -1086,7 +1086,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
     for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k) m.vreg[j][k] = sval[m.vbase[j] + (k + 1) * RPC];
   }
   ClusterComm<R, NT, C> comm(sg, sred, mbar + 1, rank, n, P.guard, m.act);
-  bicgstab_core<R, NT, false, 3>(
+  bicgstab_core<R, NT, false, ROUNDS>(
       P, sys, x, r, d, m.act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
         spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, KREG>(sval, gb, P, m, own, y, nloc, RPC);
       });
