@@ -103,7 +103,8 @@ struct CVariant {
 #define CV_ALLC(KR, RD) \
   CV_(2, KR, RD), CV_(3, KR, RD), CV_(4, KR, RD), CV_(5, KR, RD), CV_(6, KR, RD), \
       CV_(7, KR, RD), CV_(8, KR, RD)
-static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3), CV_ALLC(2, 2), CV_ALLC(0, 2)};
+// (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
+static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
 static const CVariant *find_cvariant(int c, int kreg, int rounds) {
   for (const CVariant &v : kCVariants)
     if (v.c == c && v.kreg == kreg && v.rounds == rounds) return &v;
@@ -433,10 +434,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                               "cluster placement needs a 9-point stencil (DIA) pattern with even "
                               "1024 < n <= 8192 and stencil reach <= 1024 rows"));
       const int kr = opt.reg_slots ? opt.reg_slots : 4;
-      // iteration schedule (reduction rounds per iteration); developer knob
-      const char *rd_env = getenv("BSOLVE_CLUSTER_ROUNDS");
-      const int rd = rd_env ? atoi(rd_env) : 3;
-      h->cvar = find_cvariant(c, kr, rd);
+      h->cvar = find_cvariant(c, kr, 3);
       if (!h->cvar)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no cluster variant for C=%d reg_slots=%d",
                               c, kr));
