@@ -47,7 +47,8 @@ def parse():
     ap.add_argument("--nx", type=int, default=32)
     ap.add_argument("--ny", type=int, default=31)
     ap.add_argument("--format", choices=["ell", "csr"], default="ell")
-    ap.add_argument("--placement", choices=["auto", "smem", "stream", "regs"], default="auto")
+    ap.add_argument("--placement", choices=["auto", "smem", "stream", "regs", "cluster", "tmem"],
+                    default="auto")
     ap.add_argument("--block-threads", type=int, default=0)
     ap.add_argument("--reg-slots", type=int, default=0)
     ap.add_argument("--tol", type=float, default=1e-10)

@@ -78,11 +78,15 @@ enum {
                               TMA, then held in REGISTERS for the whole solve;
                               the next system's TMA overlaps the current one
                               (ELL, 9 entries per row, even n <= 1024)        */
-  BSOLVE_PLACE_CLUSTER = 4 /* one system per thread-block cluster of C CTAs
+  BSOLVE_PLACE_CLUSTER = 4, /* one system per thread-block cluster of C CTAs
                               (1024 rows each, C <= 8) exchanging halo rows
                               and reduction partials through distributed
                               shared memory; 9-point stencils, even
                               1024 < n <= 8192 (AUTO picks it there)         */
+  BSOLVE_PLACE_TMEM = 5    /* values staged by TMA, then held in TENSOR MEMORY
+                              (tcgen05.st / tcgen05.ld, each thread its own
+                              TMEM lane); SMEM carries only the gathered
+                              vector; 9-point stencils, n <= 1024             */
 };
 
 /* Stopping criterion (R5). */

@@ -18,13 +18,13 @@ LIB_PATH = os.path.join(_HERE, "libbsolve.so")
 OK = 0
 ERR_INVALID, ERR_PATTERN, ERR_UNSUPPORTED, ERR_CUDA, ERR_NOMEM = -1, -2, -3, -4, -5
 FMT_AUTO, FMT_CSR, FMT_ELL = 0, 1, 2
-PLACE_AUTO, PLACE_SMEM, PLACE_STREAM, PLACE_REGS, PLACE_CLUSTER = 0, 1, 2, 3, 4
+PLACE_AUTO, PLACE_SMEM, PLACE_STREAM, PLACE_REGS, PLACE_CLUSTER, PLACE_TMEM = 0, 1, 2, 3, 4, 5
 STOP_REL_B, STOP_ABS = 0, 1
 SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN = 0, 1, 2
 
 _FMT = {"auto": FMT_AUTO, "csr": FMT_CSR, "ell": FMT_ELL}
 _PLACE = {"auto": PLACE_AUTO, "smem": PLACE_SMEM, "stream": PLACE_STREAM, "regs": PLACE_REGS,
-          "cluster": PLACE_CLUSTER}
+          "cluster": PLACE_CLUSTER, "tmem": PLACE_TMEM}
 _STOP = {"rel_b": STOP_REL_B, "rel": STOP_REL_B, "abs": STOP_ABS}
 
 

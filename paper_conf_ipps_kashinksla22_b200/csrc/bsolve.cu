@@ -103,6 +103,15 @@ struct CVariant {
 #define CV_ALLC(KR, RD) \
   CV_(2, KR, RD), CV_(3, KR, RD), CV_(4, KR, RD), CV_(5, KR, RD), CV_(6, KR, RD), \
       CV_(7, KR, RD), CV_(8, KR, RD)
+// TMEM-resident values (PLACE_TMEM): 128 threads x 8 rows, G rows per load group.
+struct TVariant {
+  int g;
+  solve_fn fn;
+};
+static const TVariant kTVariants[] = {{1, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
+                                      {2, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
+                                      {4, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>}};
+
 // (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
 static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
 static const CVariant *find_cvariant(int c, int kreg, int rounds) {
@@ -133,6 +142,7 @@ struct bsolve_plan {
   const Variant *var = nullptr;      // per-system-CTA kernel (also the REGS fallback)
   const PVariant *pvar = nullptr;    // persistent kernel when place == PLACE_REGS
   const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
+  solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
   int cluster = 0;                   // CTAs per system (cluster plan)
   int smem_bytes_fallback = 0, grid_persist = 0;
   unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
@@ -322,7 +332,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   if (opt_in) opt = *opt_in;
   if (opt.format < BSOLVE_FMT_AUTO || opt.format > BSOLVE_FMT_ELL)
     return fail(BSOLVE_ERR_INVALID, "bad format %d", opt.format);
-  if (opt.placement < BSOLVE_PLACE_AUTO || opt.placement > BSOLVE_PLACE_CLUSTER)
+  if (opt.placement < BSOLVE_PLACE_AUTO || opt.placement > BSOLVE_PLACE_TMEM)
     return fail(BSOLVE_ERR_INVALID, "bad placement %d", opt.placement);
   if (opt.stop != BSOLVE_STOP_REL_B && opt.stop != BSOLVE_STOP_ABS)
     return fail(BSOLVE_ERR_INVALID, "bad stop mode %d", opt.stop);
@@ -472,11 +482,38 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->grid_persist = ncl;
     }
   }
+  // ---- TMEM plan: values in tensor memory (DESIGN.md "Kernels" 9) ---------
+  if (h->place != PLACE_CLUSTER && opt.placement == BSOLVE_PLACE_TMEM) {
+    if (!(h->kfmt == FMT_DIA && W == 9 && n <= 1024 && (h->sys_stride * 8) % 16 == 0))
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                            "TMEM placement needs a 9-point stencil (DIA) pattern, n <= 1024"));
+    const char *genv = getenv("BSOLVE_TMEM_GROUP");  // developer knob: rows per TMEM load group
+    const int gsel = genv ? atoi(genv) : 2;
+    for (const TVariant &v : kTVariants)
+      if (v.g == gsel) h->var_tmem = v.fn;
+    if (!h->var_tmem) return fail_free(fail(BSOLVE_ERR_INVALID, "bad BSOLVE_TMEM_GROUP"));
+    h->place = PLACE_TMEM;
+    h->nt = 128;
+    h->r = 8;
+    h->n_pad = (n + 1) & ~1;
+    h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
+    h->smem_bytes = h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * 4 * 8 + 16;
+    if (h->smem_bytes > smem_optin)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM plan needs %d B of SMEM", h->smem_bytes));
+    ce = cudaFuncSetAttribute((const void *)h->var_tmem,
+                              cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
+    if (ce != cudaSuccess)
+      return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, 128,
+                                                       h->smem_bytes);
+    if (ce != cudaSuccess || h->ctas_per_sm < 1)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));
+  }
   // rows per thread / CTA size.  Auto: 9-point stencils (DIA) up to 1024 rows
   // take the hybrid 128 threads x 8 rows with 4 off-diagonal slots in
   // registers (measured fastest on B200, DESIGN.md perf log); otherwise 256
   // threads (2 CTAs per SM at <= 128 regs/thread), 512 for 1025..2048 rows.
-  if (h->place != PLACE_CLUSTER) {
+  if (h->place != PLACE_CLUSTER && h->place != PLACE_TMEM) {
   int nt = opt.block_threads;
   int kreg = opt.reg_slots;
   const bool stencil9 = h->kfmt == FMT_DIA && W == 9 && n <= 1024;
@@ -618,6 +655,7 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->placement = h->place == PLACE_SMEM ? BSOLVE_PLACE_SMEM
                     : h->place == PLACE_REGS    ? BSOLVE_PLACE_REGS
                     : h->place == PLACE_CLUSTER ? BSOLVE_PLACE_CLUSTER
+                    : h->place == PLACE_TMEM    ? BSOLVE_PLACE_TMEM
                                                 : BSOLVE_PLACE_STREAM;
   info->block_threads = h->nt;
   info->rows_per_thread = h->r;
@@ -684,7 +722,11 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
-  if (h->place == PLACE_CLUSTER) {
+  if (h->place == PLACE_TMEM) {
+    if ((reinterpret_cast<uintptr_t>(values) & 15u) != 0)
+      return fail(BSOLVE_ERR_INVALID, "the TMEM plan needs 16-byte aligned values (TMA)");
+    h->var_tmem<<<count, h->nt, h->smem_bytes, stream>>>(P);
+  } else if (h->place == PLACE_CLUSTER) {
     if ((reinterpret_cast<uintptr_t>(values) & 15u) != 0)
       return fail(BSOLVE_ERR_INVALID, "the cluster plan needs 16-byte aligned values (TMA)");
     cudaLaunchConfig_t cfg = {};

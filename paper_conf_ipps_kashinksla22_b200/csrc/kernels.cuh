@@ -31,7 +31,7 @@ namespace bsolve {
 // in every row r, the entry of column r + d_k (the host detects this for
 // stencil patterns): the gather address is row + d_k with d_k uniform.
 enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
-enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3, PLACE_CLUSTER = 4 };
+enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3, PLACE_CLUSTER = 4, PLACE_TMEM = 5 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
 constexpr int kMaxW = 16;
@@ -889,6 +889,159 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
       atomicExch(ctr + 1, 0ull);
     }
   }
+}
+
+// ----------------------------------------------- TMEM-resident matrix values --
+// PLACE_TMEM (DESIGN.md "Kernels" 9): the register-limited hybrid keeps only
+// ELL slots 1..4 in registers and reads slots 5..8 from SMEM.  Tensor memory
+// (256 KB per SM, a separate read path measured at ~280 B/clk/SM with 8
+// warps -- more than twice the shared-memory data pipe) holds ALL
+// off-diagonal values instead: each thread owns its TMEM lane (warp w ->
+// lanes 32*(w%4)..+31) and stores its R rows x 8 slots there once per system
+// (16 32-bit columns per row; 128 columns per CTA, 2 CTAs per SM).  Every
+// SpMV then reads values with tcgen05.ld while the gathered operands come
+// from SMEM: the shared-memory pipe carries only gathers, the two publishes
+// and the reductions.
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,"
+      "%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,"
+      "%14,%15,%16};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+      "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() {
+  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+
+// One CTA per system; 9-point DIA values (W = 9, slot 0 = diagonal kept in a
+// register); NT = 128 threads x R = 8 rows; G rows per TMEM load group.
+//   SMEM: [values staging: smem_vals] [gather: guard | n_pad | guard]
+//         [reduction scratch: 16*NWARP] [mbarrier] [TMEM base address]
+template <int R, int NT, int G>
+__global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams P) {
+  constexpr int NWARP = NT / 32;
+  constexpr int WB = 9;
+  constexpr int TCOLS = 16 * R;  // 32-bit TMEM columns per lane
+  static_assert(NT == 128 && TCOLS <= 256, "one warp per TMEM lane quarter");
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sgf = sval + P.smem_vals;
+  double *sg = sgf + P.guard;
+  double *sred = sgf + P.n_pad + 2 * P.guard;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 1);
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long sys = blockIdx.x;
+  const double *gval = P.values + sys * P.sys_stride;
+
+  // ---- TMEM allocation (warp 0) + TMA staging of the values (thread 0) -----
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(TCOLS < 32 ? 32 : TCOLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 32) {
+    mbar_init(mbar, 1);
+    fence_mbar_init();
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
+  if (tid == 0) {
+    const uint32_t bytes = static_cast<uint32_t>(P.sys_stride * 8);
+    mbar_arrive_expect_tx(mbar, bytes);
+    constexpr uint32_t CH = 32768;
+    for (uint32_t off = 0; off < bytes; off += CH)
+      tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off,
+                   reinterpret_cast<const unsigned char *>(gval) + off,
+                   bytes - off < CH ? bytes - off : CH, mbar);
+  }
+  for (int i = tid; i < P.guard; i += NT) {
+    sgf[i] = 0.0;
+    sg[P.n_pad + i] = 0.0;
+  }
+  bool act[R];
+  int vrow[R];
+  double x[R], r[R], d[R], a0[R];
+  const double *bsys = P.b + sys * n;
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    const int row = tid + j * NT;
+    act[j] = row < n;
+    vrow[j] = row < n ? row : n - 1;
+    r[j] = act[j] ? __ldg(bsys + row) : 0.0;
+    x[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row) : 0.0;
+  }
+  mbar_wait_parity(mbar, 0);
+  // ---- values: diagonal -> register, slots 1..8 -> this thread's TMEM lane --
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    a0[j] = act[j] ? sval[vrow[j]] : 0.0;
+    d[j] = (a0[j] != 0.0) ? 1.0 / a0[j] : 1.0;
+    uint32_t w[16];
+#pragma unroll
+    for (int k = 1; k < WB; ++k) {
+      const double v = act[j] ? sval[k * n + vrow[j]] : 0.0;
+      w[2 * (k - 1)] = static_cast<uint32_t>(__double2loint(v));
+      w[2 * (k - 1) + 1] = static_cast<uint32_t>(__double2hiint(v));
+    }
+    tmem_st16(tlane + 16 * j, w);
+  }
+  tmem_wait_st();
+
+  CtaComm<R, NT> comm(sg, sred, act);
+  bicgstab_core<R, NT, false, 3>(
+      P, sys, x, r, d, act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
+#pragma unroll
+        for (int j0 = 0; j0 < R; j0 += G) {
+          uint32_t w[G][16];
+          double gat[G][WB - 1];
+#pragma unroll
+          for (int g = 0; g < G; ++g) tmem_ld16(tlane + 16 * (j0 + g), w[g]);
+#pragma unroll
+          for (int g = 0; g < G; ++g)
+#pragma unroll
+            for (int k = 1; k < WB; ++k)
+              gat[g][k - 1] = *reinterpret_cast<const double *>(gb + vrow[j0 + g] * 8 + P.doff[k]);
+          tmem_wait_ld();
+#pragma unroll
+          for (int g = 0; g < G; ++g) {
+            const int j = j0 + g;
+            double acc = a0[j] * own[j];
+#pragma unroll
+            for (int k = 1; k < WB; ++k)
+              acc = fma(__hiloint2double(static_cast<int>(w[g][2 * k - 1]),
+                                         static_cast<int>(w[g][2 * k - 2])),
+                        gat[g][k - 1], acc);
+            y[j] = act[j] ? acc : 0.0;
+          }
+        }
+      });
+  // ---- release TMEM -------------------------------------------------------
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s),
+                 "n"(TCOLS < 32 ? 32 : TCOLS));
 }
 
 // ------------------------------------------ thread-block cluster per system --

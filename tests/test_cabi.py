@@ -85,7 +85,7 @@ def test_invalid_arguments():
     assert rc == B.ERR_INVALID
     rc, _ = _create(1, rp, ci, placement=9)
     assert rc == B.ERR_INVALID
-    rc, _ = _create(1, rp, ci, placement=5)
+    rc, _ = _create(1, rp, ci, placement=6)
     assert rc == B.ERR_INVALID
     rc, _ = _create(1, rp, ci, stop=3)
     assert rc == B.ERR_INVALID

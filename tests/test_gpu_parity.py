@@ -405,3 +405,27 @@ def test_cluster_warm_start_ill_conditioned_and_deterministic():
     g3 = gpu_solve(p.row_ptr, p.col_idx, B.values[3:], B.b[3:], maxiter=3000)
     for k in ("x", "iters", "resnorm", "status"):
         assert np.array_equal(g[k][3:], g3[k])
+
+
+# --------------------------------------------- TMEM-resident values plan --
+@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32), (5, 5), (1, 1), (40, 25)])
+def test_tmem_values(nx, ny):
+    """PLACE_TMEM: off-diagonal values in tensor memory (tcgen05.st/ld)."""
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 12, pattern=pat)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, placement="tmem")
+    assert g["info"]["placement"] == 5
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+
+
+def test_tmem_warm_start_and_determinism():
+    B = X.make_batch(0, 300, picard=2)
+    p = B.pattern
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-4)
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, placement="tmem")
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+    g2 = gpu_solve(p.row_ptr, p.col_idx, B.values[100:], B.b[100:], x0=x0[100:],
+                   placement="tmem")
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(g[k][100:], g2[k])
