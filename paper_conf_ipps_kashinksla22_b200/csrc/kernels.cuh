@@ -966,15 +966,18 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
-  if (tid == 0) {
-    const uint32_t bytes = static_cast<uint32_t>(P.sys_stride * 8);
-    mbar_arrive_expect_tx(mbar, bytes);
+  const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
+  const bool use_tma = (vbytes % 16u == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0);
+  if (use_tma && tid == 0) {
+    mbar_arrive_expect_tx(mbar, vbytes);
     constexpr uint32_t CH = 32768;
-    for (uint32_t off = 0; off < bytes; off += CH)
+    for (uint32_t off = 0; off < vbytes; off += CH)
       tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off,
                    reinterpret_cast<const unsigned char *>(gval) + off,
-                   bytes - off < CH ? bytes - off : CH, mbar);
+                   vbytes - off < CH ? vbytes - off : CH, mbar);
   }
+  if (!use_tma)  // unaligned system block: plain cooperative copy
+    for (long long i = tid; i < P.sys_stride; i += NT) sval[i] = __ldg(gval + i);
   for (int i = tid; i < P.guard; i += NT) {
     sgf[i] = 0.0;
     sg[P.n_pad + i] = 0.0;
@@ -991,7 +994,8 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
     r[j] = act[j] ? __ldg(bsys + row) : 0.0;
     x[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row) : 0.0;
   }
-  mbar_wait_parity(mbar, 0);
+  if (use_tma) mbar_wait_parity(mbar, 0);
+  else __syncthreads();
   // ---- values: diagonal -> register, slots 1..8 -> this thread's TMEM lane --
 #pragma unroll
   for (int j = 0; j < R; ++j) {

@@ -14,7 +14,9 @@ import xgcgen as X  # noqa: E402
 from paper_conf_ipps_kashinksla22_b200 import Solver  # noqa: E402
 
 CASES = [
-    ("hybrid 128x8 DIA (default 992)", dict(nx=32, ny=31), dict()),
+    ("tmem values (default 992)", dict(nx=32, ny=31), dict()),
+    ("tmem values, unaligned block (5x5)", dict(nx=5, ny=5), dict(placement="tmem")),
+    ("hybrid 128x8 DIA, 4 reg slots", dict(nx=32, ny=31), dict(block_threads=128, reg_slots=4)),
     ("smem 256x4 DIA", dict(nx=32, ny=31), dict(block_threads=256)),
     ("csr smem", dict(nx=32, ny=31), dict(format="csr")),
     ("stream ell", dict(nx=32, ny=31), dict(placement="stream")),
