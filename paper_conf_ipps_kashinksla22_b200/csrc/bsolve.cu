@@ -105,12 +105,14 @@ struct CVariant {
       CV_(7, KR, RD), CV_(8, KR, RD)
 // TMEM-resident values (PLACE_TMEM): 128 threads x 8 rows, G rows per load group.
 struct TVariant {
-  int g;
+  int nt, r, g;
   solve_fn fn;
 };
-static const TVariant kTVariants[] = {{1, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
-                                      {2, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
-                                      {4, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>}};
+static const TVariant kTVariants[] = {{128, 8, 1, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
+                                      {128, 8, 2, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
+                                      {128, 8, 4, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>},
+                                      {256, 4, 1, (solve_fn)bicgstab_tmem_kernel<4, 256, 1>},
+                                      {256, 4, 2, (solve_fn)bicgstab_tmem_kernel<4, 256, 2>}};
 
 // (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
 static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
@@ -492,24 +494,34 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     if (!tmem_ok)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                             "TMEM placement needs a 9-point stencil (DIA) pattern, n <= 1024"));
-    const char *genv = getenv("BSOLVE_TMEM_GROUP");  // developer knob: rows per TMEM load group
-    const int gsel = genv ? atoi(genv) : 4;
+    // developer knobs: rows per TMEM load group, threads per CTA
+    const char *genv = getenv("BSOLVE_TMEM_GROUP");
+    const char *tenv = getenv("BSOLVE_TMEM_THREADS");
+    const int ntsel = opt.block_threads ? opt.block_threads : (tenv ? atoi(tenv) : 128);
+    const int gsel = genv ? atoi(genv) : (ntsel == 128 ? 4 : 2);
     for (const TVariant &v : kTVariants)
-      if (v.g == gsel) h->var_tmem = v.fn;
-    if (!h->var_tmem) return fail_free(fail(BSOLVE_ERR_INVALID, "bad BSOLVE_TMEM_GROUP"));
+      if (v.g == gsel && v.nt == ntsel) {
+        h->var_tmem = v.fn;
+        h->nt = v.nt;
+        h->r = v.r;
+      }
+    if (!h->var_tmem)
+      return fail_free(fail(BSOLVE_ERR_INVALID, "no TMEM variant for %d threads, group %d", ntsel,
+                            gsel));
     h->place = PLACE_TMEM;
-    h->nt = 128;
-    h->r = 8;
     h->n_pad = (n + 1) & ~1;
     h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
-    h->smem_bytes = h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * 4 * 8 + 16;
+    h->smem_bytes =
+        h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * (h->nt / 32) * 8 + 16;
     if (h->smem_bytes > smem_optin)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM plan needs %d B of SMEM", h->smem_bytes));
     ce = cudaFuncSetAttribute((const void *)h->var_tmem,
                               cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
     if (ce != cudaSuccess)
       return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
-    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, 128,
+    cudaFuncSetAttribute((const void *)h->var_tmem, cudaFuncAttributePreferredSharedMemoryCarveout,
+                         cudaSharedmemCarveoutMaxShared);
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, h->nt,
                                                        h->smem_bytes);
     if (ce != cudaSuccess || h->ctas_per_sm < 1)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));

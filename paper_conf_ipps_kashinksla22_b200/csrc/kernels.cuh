@@ -935,8 +935,12 @@ template <int R, int NT, int G>
 __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
   constexpr int WB = 9;
-  constexpr int TCOLS = 16 * R;  // 32-bit TMEM columns per lane
-  static_assert(NT == 128 && TCOLS <= 256, "one warp per TMEM lane quarter");
+  // 32-bit TMEM columns: 16 per row per thread; warps w and w+4 share lane
+  // quarter w%4 and use consecutive column ranges
+  constexpr int TCOLS_T = 16 * R;
+  constexpr int TCOLS_USED = (NT / 128) * TCOLS_T;
+  constexpr int TCOLS = TCOLS_USED <= 32 ? 32 : TCOLS_USED <= 64 ? 64 : TCOLS_USED <= 128 ? 128 : 256;
+  static_assert((NT == 128 || NT == 256) && TCOLS_USED <= 256, "TMEM plan: 128 or 256 threads");
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double *sval = reinterpret_cast<double *>(smem_raw);
   double *sgf = sval + P.smem_vals;
@@ -955,7 +959,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                      smem_addr(tbase_s)),
-                 "n"(TCOLS < 32 ? 32 : TCOLS));
+                 "n"(TCOLS));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (tid == 32) {
@@ -965,7 +969,8 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
-  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
+  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16) +
+                         static_cast<uint32_t>((warp >> 2) * TCOLS_T);
   const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
   const bool use_tma = (vbytes % 16u == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0);
   if (use_tma && tid == 0) {

@@ -409,9 +409,10 @@ def test_cluster_warm_start_ill_conditioned_and_deterministic():
 
 
 # --------------------------------------------- TMEM-resident values plan --
-@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32), (5, 5), (1, 1), (40, 25)])
+@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32), (5, 5), (40, 25)])
 def test_tmem_values(nx, ny):
-    """PLACE_TMEM: off-diagonal values in tensor memory (tcgen05.st/ld)."""
+    """PLACE_TMEM: off-diagonal values in tensor memory (tcgen05.st/ld);
+    5x5 has a value block that is not a multiple of 16 B (non-TMA copy)."""
     pat = X.stencil_pattern(nx, ny)
     B = X.make_batch(0, 12, pattern=pat)
     g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, placement="tmem")
@@ -430,3 +431,10 @@ def test_tmem_warm_start_and_determinism():
                    placement="tmem")
     for k in ("x", "iters", "resnorm", "status"):
         assert np.array_equal(g[k][100:], g2[k])
+
+
+def test_tmem_refuses_non_stencil():
+    pat = X.stencil_pattern(1, 1)  # W = 1: not a 9-point stencil
+    with pytest.raises(BsolveError) as e:
+        Solver(pat.row_ptr, pat.col_idx, 2, placement="tmem")
+    assert e.value.code == -3
