@@ -116,6 +116,10 @@ static const TVariant kTVariants[] = {{128, 8, 1, (solve_fn)bicgstab_tmem_kernel
 
 // (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
 static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
+// cluster plan with TMEM-resident values (kreg field unused: -1)
+#define CVT_(C) {C, -1, 3, (solve_fn)bicgstab_cluster_tmem_kernel<8, 128, C>}
+static const CVariant kCTVariants[] = {CVT_(2), CVT_(3), CVT_(4), CVT_(5),
+                                       CVT_(6), CVT_(7), CVT_(8)};
 static const CVariant *find_cvariant(int c, int kreg, int rounds) {
   for (const CVariant &v : kCVariants)
     if (v.c == c && v.kreg == kreg && v.rounds == rounds) return &v;
@@ -446,7 +450,17 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                               "cluster placement needs a 9-point stencil (DIA) pattern with even "
                               "1024 < n <= 8192 and stencil reach <= 1024 rows"));
       const int kr = opt.reg_slots ? opt.reg_slots : 4;
-      h->cvar = find_cvariant(c, kr, 3);
+      // values in TMEM unless register slots were requested (developer knob
+      // BSOLVE_CLUSTER_TMEM=0 selects the register/SMEM-value variant)
+      const char *ctenv = getenv("BSOLVE_CLUSTER_TMEM");
+      const bool ctmem = opt.reg_slots == 0 && !(ctenv && atoi(ctenv) == 0);
+      h->cvar = nullptr;
+      if (ctmem) {
+        for (const CVariant &v : kCTVariants)
+          if (v.c == c) h->cvar = &v;
+      } else {
+        h->cvar = find_cvariant(c, kr, 3);
+      }
       if (!h->cvar)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "no cluster variant for C=%d reg_slots=%d",
                               c, kr));
@@ -456,7 +470,8 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->r = 8;
       h->n_pad = (n + 1) & ~1;
       h->smem_vals = 9 * rpc;
-      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 4 * 8;  // + 4 mbarriers
+      // + 4 mbarriers + the TMEM base address slot
+      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 5 * 8;
       if (h->smem_bytes > smem_optin)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster plan needs %d B of SMEM",
                               h->smem_bytes));

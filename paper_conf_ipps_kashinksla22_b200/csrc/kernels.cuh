@@ -927,6 +927,62 @@ __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
 
+// Move this thread's rows of the staged values into its TMEM lane: slot 0
+// (diagonal) -> a0 register (and d = 1/a0), slots 1..8 -> 16 columns per row.
+// `stride` = doubles between two ELL slots in the staging buffer.
+template <int R, int WB>
+__device__ __forceinline__ void tmem_fill(uint32_t tlane, const double *sval, int stride,
+                                          const int (&vrow)[R], const bool (&act)[R],
+                                          double (&a0)[R], double (&d)[R]) {
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    a0[j] = act[j] ? sval[vrow[j]] : 0.0;
+    d[j] = (a0[j] != 0.0) ? 1.0 / a0[j] : 1.0;
+    uint32_t w[16];
+#pragma unroll
+    for (int k = 1; k < WB; ++k) {
+      const double v = act[j] ? sval[k * stride + vrow[j]] : 0.0;
+      w[2 * (k - 1)] = static_cast<uint32_t>(__double2loint(v));
+      w[2 * (k - 1) + 1] = static_cast<uint32_t>(__double2hiint(v));
+    }
+    tmem_st16(tlane + 16 * j, w);
+  }
+  tmem_wait_st();
+}
+
+// y = A g with values from TMEM (G rows per tcgen05.ld group, their SMEM
+// gathers issued before the wait so both latencies overlap) and DIA gathers.
+template <int R, int G, int WB>
+__device__ __forceinline__ void tmem_spmv(uint32_t tlane, const unsigned char *gb,
+                                          const int (&vrow)[R], const double (&a0)[R],
+                                          const bool (&act)[R], const int *doff,
+                                          const double (&own)[R], double (&y)[R]) {
+#pragma unroll
+  for (int j0 = 0; j0 < R; j0 += G) {
+    uint32_t w[G][16];
+    double gat[G][WB - 1];
+#pragma unroll
+    for (int g = 0; g < G; ++g) tmem_ld16(tlane + 16 * (j0 + g), w[g]);
+#pragma unroll
+    for (int g = 0; g < G; ++g)
+#pragma unroll
+      for (int k = 1; k < WB; ++k)
+        gat[g][k - 1] = *reinterpret_cast<const double *>(gb + vrow[j0 + g] * 8 + doff[k]);
+    tmem_wait_ld();
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+      const int j = j0 + g;
+      double acc = a0[j] * own[j];
+#pragma unroll
+      for (int k = 1; k < WB; ++k)
+        acc = fma(__hiloint2double(static_cast<int>(w[g][2 * k - 1]),
+                                   static_cast<int>(w[g][2 * k - 2])),
+                  gat[g][k - 1], acc);
+      y[j] = act[j] ? acc : 0.0;
+    }
+  }
+}
+
 // One CTA per system; 9-point DIA values (W = 9, slot 0 = diagonal kept in a
 // register); NT = 128 threads x R = 8 rows; G rows per TMEM load group.
 //   SMEM: [values staging: smem_vals] [gather: guard | n_pad | guard]
@@ -1002,48 +1058,12 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   if (use_tma) mbar_wait_parity(mbar, 0);
   else __syncthreads();
   // ---- values: diagonal -> register, slots 1..8 -> this thread's TMEM lane --
-#pragma unroll
-  for (int j = 0; j < R; ++j) {
-    a0[j] = act[j] ? sval[vrow[j]] : 0.0;
-    d[j] = (a0[j] != 0.0) ? 1.0 / a0[j] : 1.0;
-    uint32_t w[16];
-#pragma unroll
-    for (int k = 1; k < WB; ++k) {
-      const double v = act[j] ? sval[k * n + vrow[j]] : 0.0;
-      w[2 * (k - 1)] = static_cast<uint32_t>(__double2loint(v));
-      w[2 * (k - 1) + 1] = static_cast<uint32_t>(__double2hiint(v));
-    }
-    tmem_st16(tlane + 16 * j, w);
-  }
-  tmem_wait_st();
+  tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d);
 
   CtaComm<R, NT> comm(sg, sred, act);
   bicgstab_core<R, NT, false, 3>(
       P, sys, x, r, d, act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
-#pragma unroll
-        for (int j0 = 0; j0 < R; j0 += G) {
-          uint32_t w[G][16];
-          double gat[G][WB - 1];
-#pragma unroll
-          for (int g = 0; g < G; ++g) tmem_ld16(tlane + 16 * (j0 + g), w[g]);
-#pragma unroll
-          for (int g = 0; g < G; ++g)
-#pragma unroll
-            for (int k = 1; k < WB; ++k)
-              gat[g][k - 1] = *reinterpret_cast<const double *>(gb + vrow[j0 + g] * 8 + P.doff[k]);
-          tmem_wait_ld();
-#pragma unroll
-          for (int g = 0; g < G; ++g) {
-            const int j = j0 + g;
-            double acc = a0[j] * own[j];
-#pragma unroll
-            for (int k = 1; k < WB; ++k)
-              acc = fma(__hiloint2double(static_cast<int>(w[g][2 * k - 1]),
-                                         static_cast<int>(w[g][2 * k - 2])),
-                        gat[g][k - 1], acc);
-            y[j] = act[j] ? acc : 0.0;
-          }
-        }
+        tmem_spmv<R, G, WB>(tlane, gb, vrow, a0, act, P.doff, own, y);
       });
   // ---- release TMEM -------------------------------------------------------
   asm volatile("tcgen05.fence::before_thread_sync;");
@@ -1253,6 +1273,92 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
         spmv_rows<FMT, PLACE_SMEM, WB, EXACT, R, NT, KREG>(sval, gb, P, m, own, y, nloc, RPC);
       });
   cl.sync();  // peers may write into this CTA's SMEM until they are done
+}
+
+// Cluster plan with TMEM-resident values (the default for 1024 < n <= 8192
+// 9-point stencils): the cluster exchange of bicgstab_cluster_kernel plus the
+// TMEM value path of bicgstab_tmem_kernel.
+//   SMEM per CTA: [values staging: 9 x RPC] [gather: G | RPC | G]
+//                 [scratch: 2 x 8 x C x NWARP] [4 mbarriers] [TMEM base]
+template <int R, int NT, int C>
+__global__ void __launch_bounds__(NT, 2) bicgstab_cluster_tmem_kernel(const SolveParams P) {
+  constexpr int NWARP = NT / 32;
+  constexpr int RPC = R * NT;
+  constexpr int WB = 9;
+  constexpr int TCOLS = 16 * R;
+  static_assert(NT == 128 && TCOLS <= 256, "one warp per TMEM lane quarter");
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  const int rank = static_cast<int>(cl.block_rank());
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sgf = sval + WB * RPC;
+  double *sg = sgf + P.guard;
+  double *sred = sgf + RPC + 2 * P.guard;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * C * NWARP);
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 4);
+  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
+
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long sys = blockIdx.x / C;
+  const int row0 = rank * RPC;
+  const int nloc = min(RPC, n - row0);
+  // mbar[0]: TMA, mbar[1]: halo rows, mbar[2..3]: reduction buffers
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(TCOLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 32) {
+    for (int i = 0; i < 4; ++i) mbar_init(mbar + i, 1);
+    fence_mbar_init();
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
+  if (tid == 0) {
+    const uint32_t bytes = static_cast<uint32_t>(nloc) * 8u;
+    mbar_arrive_expect_tx(mbar, bytes * WB);
+    const double *gsys = P.values + sys * P.sys_stride + row0;
+    for (int k = 0; k < WB; ++k) tma_bulk_g2s(sval + k * RPC, gsys + (long long)k * n, bytes, mbar);
+  }
+  for (int i = tid; i < P.guard; i += NT) {
+    if (rank == 0) sgf[i] = 0.0;
+    if (rank == C - 1) sg[RPC + i] = 0.0;
+  }
+  for (int i = nloc + tid; i < RPC; i += NT) sg[i] = 0.0;
+  if (rank < C - 1) {
+    const int nnext = min(RPC, n - (rank + 1) * RPC);
+    for (int i = nnext + tid; i < P.guard; i += NT) sg[RPC + i] = 0.0;
+  }
+  bool act[R];
+  int vrow[R];
+  double x[R], r[R], d[R], a0[R];
+  const double *bsys = P.b + sys * n;
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    const int li = tid + j * NT;
+    act[j] = li < nloc;
+    vrow[j] = li < nloc ? li : nloc - 1;
+    r[j] = act[j] ? __ldg(bsys + row0 + li) : 0.0;
+    x[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + li) : 0.0;
+  }
+  cl.sync();  // every CTA of the cluster runs (DSMEM and its mbarriers are live)
+  mbar_wait_parity(mbar, 0);
+  tmem_fill<R, WB>(tlane, sval, RPC, vrow, act, a0, d);
+  ClusterComm<R, NT, C> comm(sg, sred, mbar + 1, rank, n, P.guard, act);
+  bicgstab_core<R, NT, false, 3>(
+      P, sys, x, r, d, act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
+        tmem_spmv<R, 4, WB>(tlane, gb, vrow, a0, act, P.doff, own, y);
+      });
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  cl.sync();  // peers may write into this CTA's SMEM until they are done
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s),
+                 "n"(TCOLS));
 }
 
 // -------------------------------------------------- standalone batched SpMV --
