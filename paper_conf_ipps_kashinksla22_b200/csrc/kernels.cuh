@@ -909,8 +909,7 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
       : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
         "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
         "=r"(r[14]), "=r"(r[15])
-      : "r"(taddr)
-      : "memory");
+      : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&r)[16]) {
   asm volatile(
@@ -921,7 +920,17 @@ __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&r)[16
       : "memory");
 }
 __device__ __forceinline__ void tmem_wait_ld() {
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+  asm volatile("tcgen05.wait::ld.sync.aligned;");
+}
+// After tcgen05.wait::ld: make every later use of the loaded registers depend
+// on an (empty) volatile asm that is ordered after the wait, so the compiler
+// cannot schedule a use before the asynchronous TMEM load completed.  (No
+// "memory" clobber on the wait: SMEM loads may be hoisted across it.)
+__device__ __forceinline__ void tmem_regs_ready(uint32_t (&r)[16]) {
+  asm volatile(""
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]),
+                 "+r"(r[6]), "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]),
+                 "+r"(r[12]), "+r"(r[13]), "+r"(r[14]), "+r"(r[15]));
 }
 __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
@@ -969,6 +978,8 @@ __device__ __forceinline__ void tmem_spmv(uint32_t tlane, const unsigned char *g
       for (int k = 1; k < WB; ++k)
         gat[g][k - 1] = *reinterpret_cast<const double *>(gb + vrow[j0 + g] * 8 + doff[k]);
     tmem_wait_ld();
+#pragma unroll
+    for (int g = 0; g < G; ++g) tmem_regs_ready(w[g]);
 #pragma unroll
     for (int g = 0; g < G; ++g) {
       const int j = j0 + g;
