@@ -149,6 +149,8 @@ struct bsolve_plan {
   const PVariant *pvar = nullptr;    // persistent kernel when place == PLACE_REGS
   const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
   solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
+  persist_fn var_tmem_p = nullptr;   // persistent TMEM kernel (aligned buffers)
+  int smem_bytes_tmem_p = 0, grid_tmem_p = 0;
   int cluster = 0;                   // CTAs per system (cluster plan)
   int smem_bytes_fallback = 0, grid_persist = 0;
   unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
@@ -540,6 +542,31 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                                                        h->smem_bytes);
     if (ce != cudaSuccess || h->ctas_per_sm < 1)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));
+    // persistent variant with TMA prefetch of the next system (needs 16-byte
+    // aligned system blocks; the launch also checks the buffer addresses)
+    const char *penv = getenv("BSOLVE_TMEM_PERSIST");
+    const bool persist = !(penv && atoi(penv) == 0) && h->nt == 128 && h->r == 8 &&
+                         n % 2 == 0 && (h->sys_stride * 8) % 16 == 0;
+    if (persist) {
+      h->var_tmem_p = (persist_fn)bicgstab_tmem_persist_kernel<8, 128, 4>;
+      h->smem_bytes_tmem_p = h->smem_vals * 8 + 2 * h->n_pad * 8 +
+                             (h->n_pad + 2 * h->guard) * 8 + 16 * 4 * 8 + 32;
+      if (h->smem_bytes_tmem_p > smem_optin ||
+          cudaFuncSetAttribute((const void *)h->var_tmem_p,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               h->smem_bytes_tmem_p) != cudaSuccess) {
+        cudaGetLastError();
+        h->var_tmem_p = nullptr;
+      } else {
+        cudaFuncSetAttribute((const void *)h->var_tmem_p,
+                             cudaFuncAttributePreferredSharedMemoryCarveout,
+                             cudaSharedmemCarveoutMaxShared);
+        h->grid_tmem_p = 2 * h->num_sms;  // 2 CTAs per SM (255 regs x 128 threads, ~96 KB)
+        if (cudaMalloc(&h->d_ctr, 2 * sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMemset(h->d_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
+          return fail_free(fail(BSOLVE_ERR_NOMEM, "work counter allocation failed"));
+      }
+    }
   }
   // rows per thread / CTA size.  Auto: 9-point stencils (DIA) up to 1024 rows
   // take the hybrid 128 threads x 8 rows with 4 off-diagonal slots in
@@ -755,7 +782,12 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)
-    h->var_tmem<<<count, h->nt, h->smem_bytes, stream>>>(P);
+    if (h->var_tmem_p && aligned) {
+      const int grid = (int)std::min<long long>(h->grid_tmem_p, count);
+      h->var_tmem_p<<<grid, h->nt, h->smem_bytes_tmem_p, stream>>>(P, h->d_ctr);
+    } else {
+      h->var_tmem<<<count, h->nt, h->smem_bytes, stream>>>(P);
+    }
   } else if (h->place == PLACE_CLUSTER) {
     if ((reinterpret_cast<uintptr_t>(values) & 15u) != 0)
       return fail(BSOLVE_ERR_INVALID, "the cluster plan needs 16-byte aligned values (TMA)");

@@ -438,3 +438,31 @@ def test_tmem_refuses_non_stencil():
     with pytest.raises(BsolveError) as e:
         Solver(pat.row_ptr, pat.col_idx, 2, placement="tmem")
     assert e.value.code == -3
+
+
+@pytest.mark.parametrize("batch", [3, 296, 1000])
+def test_tmem_persistent_repeated_launches_and_fallback(batch):
+    """Default TMEM plan launches the persistent kernel (self-resetting work
+    counter, TMA prefetch of the next system): back-to-back launches on one
+    handle are identical; batches below / above the 296-CTA grid; misaligned
+    buffers take the per-system kernel with identical results."""
+    B = X.make_batch(0, batch)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, batch)
+    assert S.info["placement"] == 5
+    v = to_dev(S.ell_values(B.values))
+    b = to_dev(B.b)
+    outs = [S.run(v, b) for _ in range(3)]
+    torch.cuda.synchronize()
+    for o in outs[1:]:
+        for a, c in zip(outs[0], o):
+            assert torch.equal(a, c)
+    g = dict(x=outs[0][0].cpu().numpy(), iters=outs[0][1].cpu().numpy(),
+             resnorm=outs[0][2].cpu().numpy(), status=outs[0][3].cpu().numpy().astype(np.int32))
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+    vbig = torch.empty(v.numel() + 1, dtype=torch.float64, device="cuda")
+    vbig[1:] = v.reshape(-1)
+    xf, itf, rf, sf = S.run(vbig[1:].view_as(v), b)
+    torch.cuda.synchronize()
+    assert np.array_equal(itf.cpu().numpy(), g["iters"])
+    assert np.array_equal(xf.cpu().numpy(), g["x"])
