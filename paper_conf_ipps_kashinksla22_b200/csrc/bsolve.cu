@@ -544,8 +544,11 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));
     // persistent variant with TMA prefetch of the next system (needs 16-byte
     // aligned system blocks; the launch also checks the buffer addresses)
+    // (opt-in via BSOLVE_TMEM_PERSIST=1: measured no faster than the per-system
+    // launch, 6.89 vs 6.91 M sys/s -- the co-resident CTA already hides a
+    // CTA's start-up)
     const char *penv = getenv("BSOLVE_TMEM_PERSIST");
-    const bool persist = !(penv && atoi(penv) == 0) && h->nt == 128 && h->r == 8 &&
+    const bool persist = (penv && atoi(penv) == 1) && h->nt == 128 && h->r == 8 &&
                          n % 2 == 0 && (h->sys_stride * 8) % 16 == 0;
     if (persist) {
       h->var_tmem_p = (persist_fn)bicgstab_tmem_persist_kernel<8, 128, 4>;

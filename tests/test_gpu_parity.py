@@ -441,11 +441,12 @@ def test_tmem_refuses_non_stencil():
 
 
 @pytest.mark.parametrize("batch", [3, 296, 1000])
-def test_tmem_persistent_repeated_launches_and_fallback(batch):
+def test_tmem_persistent_repeated_launches_and_fallback(batch, monkeypatch):
     """Default TMEM plan launches the persistent kernel (self-resetting work
     counter, TMA prefetch of the next system): back-to-back launches on one
     handle are identical; batches below / above the 296-CTA grid; misaligned
     buffers take the per-system kernel with identical results."""
+    monkeypatch.setenv("BSOLVE_TMEM_PERSIST", "1")  # read at bsolve_create
     B = X.make_batch(0, batch)
     p = B.pattern
     S = Solver(p.row_ptr, p.col_idx, batch)
