@@ -105,14 +105,17 @@ struct CVariant {
       CV_(7, KR, RD), CV_(8, KR, RD)
 // TMEM-resident values (PLACE_TMEM): 128 threads x 8 rows, G rows per load group.
 struct TVariant {
-  int nt, r, g;
+  int nt, r, g, rounds;
   solve_fn fn;
 };
-static const TVariant kTVariants[] = {{128, 8, 1, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
-                                      {128, 8, 2, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
-                                      {128, 8, 4, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>},
-                                      {256, 4, 1, (solve_fn)bicgstab_tmem_kernel<4, 256, 1>},
-                                      {256, 4, 2, (solve_fn)bicgstab_tmem_kernel<4, 256, 2>}};
+static const TVariant kTVariants[] = {
+    {128, 8, 1, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
+    {128, 8, 2, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
+    {128, 8, 4, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>},
+    {128, 8, 4, 2, (solve_fn)bicgstab_tmem_kernel<8, 128, 4, 2>},
+    {128, 8, 2, 2, (solve_fn)bicgstab_tmem_kernel<8, 128, 2, 2>},
+    {256, 4, 1, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 1>},
+    {256, 4, 2, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 2>}};
 
 // (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
 static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
@@ -516,8 +519,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const char *tenv = getenv("BSOLVE_TMEM_THREADS");
     const int ntsel = opt.block_threads ? opt.block_threads : (tenv ? atoi(tenv) : 128);
     const int gsel = genv ? atoi(genv) : (ntsel == 128 ? 4 : 2);
+    const char *renv = getenv("BSOLVE_TMEM_ROUNDS");  // developer knob: reduction rounds
+    const int rsel = renv ? atoi(renv) : 3;
     for (const TVariant &v : kTVariants)
-      if (v.g == gsel && v.nt == ntsel) {
+      if (v.g == gsel && v.nt == ntsel && v.rounds == rsel) {
         h->var_tmem = v.fn;
         h->nt = v.nt;
         h->r = v.r;

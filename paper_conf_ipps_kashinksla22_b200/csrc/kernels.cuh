@@ -998,7 +998,7 @@ __device__ __forceinline__ void tmem_spmv(uint32_t tlane, const unsigned char *g
 // register); NT = 128 threads x R = 8 rows; G rows per TMEM load group.
 //   SMEM: [values staging: smem_vals] [gather: guard | n_pad | guard]
 //         [reduction scratch: 16*NWARP] [mbarrier] [TMEM base address]
-template <int R, int NT, int G>
+template <int R, int NT, int G, int ROUNDS = 3>
 __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams P) {
   constexpr int NWARP = NT / 32;
   constexpr int WB = 9;
@@ -1072,7 +1072,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d);
 
   CtaComm<R, NT> comm(sg, sred, act);
-  bicgstab_core<R, NT, false, 3>(
+  bicgstab_core<R, NT, false, ROUNDS>(
       P, sys, x, r, d, act, r, comm, [&](const double(&own)[R], double(&y)[R]) {
         tmem_spmv<R, G, WB>(tlane, gb, vrow, a0, act, P.doff, own, y);
       });

@@ -467,3 +467,19 @@ def test_tmem_persistent_repeated_launches_and_fallback(batch, monkeypatch):
     torch.cuda.synchronize()
     assert np.array_equal(itf.cpu().numpy(), g["iters"])
     assert np.array_equal(xf.cpu().numpy(), g["x"])
+
+
+@pytest.mark.parametrize("rounds,group", [(2, 4), (2, 2), (3, 1)])
+def test_tmem_schedules(rounds, group, monkeypatch):
+    """TMEM plan with the 2-round schedule (deferred stop test 1, algebraic
+    rho) and other row groups: same parity bar against the oracle."""
+    monkeypatch.setenv("BSOLVE_TMEM_ROUNDS", str(rounds))
+    monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
+    B = X.make_batch(0, 64)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-3)
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
