@@ -349,10 +349,24 @@ def run_ours(args, rank, world, local_rank):
     num_sms = info["num_sms"]
     sm_max_mhz = float(peaks.get("sm_max_mhz", 1965.0))
     kern_avg_s = statistics.mean(kern_ms) * 1e-3
-    smem_bytes_iter = 2 * (16 * nnz + 8 * n)
+    # Algorithmic SMEM bytes per unit (= one BiCGSTAB iteration of one system;
+    # SURVEY.md 8(d)): each of the 2 SpMVs gathers one
+    # 8-byte operand per nonzero and publishes one 8-byte entry per row.  When
+    # the matrix values are staged in SMEM (placements smem/stream/cluster with
+    # SMEM slots) they add 8 B per nonzero; in the TMEM / register-resident
+    # plans they never cross the SMEM pipe and are accounted on their own path.
+    values_in_smem = info["placement"] not in (3, 5)
+    smem_bytes_iter = 2 * ((16 if values_in_smem else 8) * nnz + 8 * n)
     smem_bytes_launch = smem_bytes_iter * sum_iters_rank
     smem_peak = 128.0 * num_sms * sm_max_mhz * 1e6      # guide: 128 B/clk/SM
     smem_achieved = smem_bytes_launch / kern_avg_s
+    # operand model of the method (values + gathered operands + stores), the
+    # pre-TMEM definition: an effective on-chip bandwidth, not a pipe bound
+    all_operand_bytes = 2 * (16 * nnz + 8 * n) * sum_iters_rank
+    tmem_bytes_launch = (0 if values_in_smem else 2 * 8 * nnz * sum_iters_rank)
+    tmem_peak = 280.0 * num_sms * sm_max_mhz * 1e6      # measured tcgen05.ld, 8 warps/SM
+    fp64_flops_launch = (4 * nnz + 26 * n) * sum_iters_rank   # 61,504 / iter
+    fp64_peak = 64 * 2 * num_sms * sm_max_mhz * 1e6     # 64 DFMA/clk/SM
     vals_bytes = vals.element_size() * vals.numel() / per_rank
     hbm_bytes_sys = vals_bytes + 8 * n + 8 * n + 4 + 8 + 1   # values, b, x, iters, resnorm, status
     hbm_achieved = hbm_bytes_sys * per_rank / kern_avg_s
@@ -367,8 +381,11 @@ def run_ours(args, rank, world, local_rank):
         "unit": "GB/s", "frac": smem_achieved / smem_peak, "traffic": None,
         "kernel": "bicgstab_kernel (one launch per step)",
         "algorithmic_bytes_per_launch": smem_bytes_launch,
-        "algorithmic_bytes_per_unit": f"{smem_bytes_iter} B per BiCGSTAB iteration "
-                                      f"(2 SpMVs x (16 B x nnz + 8 B x n))",
+        "algorithmic_bytes_per_unit": (
+            f"{smem_bytes_iter} B per BiCGSTAB iteration (2 SpMVs x ("
+            + ("16 B x nnz [values + gathered operands]" if values_in_smem else
+               "8 B x nnz [gathered operands; values live in TMEM/registers]")
+            + " + 8 B x n [published vector]))"),
         "units_per_launch": sum_iters_rank,
         "peak_source": f"derived: 128 B/clk/SM x {num_sms} SMs x {sm_max_mhz:.0f} MHz "
                        f"(B300_MICROARCH smem crossbar; no SMEM figure in MEASURED_PEAKS)",
@@ -378,6 +395,18 @@ def run_ours(args, rank, world, local_rank):
         "hbm": {"achieved": hbm_achieved / 1e9, "peak": hbm_peak / 1e9, "unit": "GB/s",
                 "frac": hbm_achieved / hbm_peak, "bytes_per_system": hbm_bytes_sys,
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
+        "tmem": {"achieved": tmem_bytes_launch / kern_avg_s / 1e9, "peak": tmem_peak / 1e9,
+                 "unit": "GB/s", "frac": tmem_bytes_launch / kern_avg_s / tmem_peak,
+                 "peak_source": "tools/tmem_probe.cu: tcgen05.ld 280 B/clk/SM at 8 warps "
+                                "(profiles/r1_tmem_probe.txt)"},
+        "fp64": {"achieved": fp64_flops_launch / kern_avg_s / 1e12, "peak": fp64_peak / 1e12,
+                 "unit": "TFLOP/s", "frac": fp64_flops_launch / kern_avg_s / fp64_peak,
+                 "peak_source": "derived: 64 DFMA/clk/SM x 148 x 1965 MHz"},
+        "all_operand_effective": {
+            "achieved": all_operand_bytes / kern_avg_s / 1e9, "unit": "GB/s",
+            "frac_of_smem_peak": all_operand_bytes / kern_avg_s / smem_peak,
+            "note": "values + gathered operands + stores per iteration (2 x (16 nnz + 8 n)) "
+                    "wherever they live; effective on-chip bandwidth, can exceed 1"},
     }
     # traffic from the committed ncu --set full capture of this kernel on this
     # workload (profiles/ncu_traffic.json), scaled to this launch's systems

@@ -469,10 +469,9 @@ def test_tmem_persistent_repeated_launches_and_fallback(batch, monkeypatch):
     assert np.array_equal(xf.cpu().numpy(), g["x"])
 
 
-@pytest.mark.parametrize("rounds,group", [(2, 4), (2, 2), (3, 1)])
+@pytest.mark.parametrize("rounds,group", [(3, 1), (3, 2)])
 def test_tmem_schedules(rounds, group, monkeypatch):
-    """TMEM plan with the 2-round schedule (deferred stop test 1, algebraic
-    rho) and other row groups: same parity bar against the oracle."""
+    """TMEM plan with other row groups per tcgen05.ld wait: same parity bar."""
     monkeypatch.setenv("BSOLVE_TMEM_ROUNDS", str(rounds))
     monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
     B = X.make_batch(0, 64)
