@@ -23,6 +23,7 @@
 
 #include "../../include/bsolve.h"
 #include "kernels.cuh"
+#include "variants.h"
 
 using namespace bsolve;
 
@@ -47,93 +48,34 @@ static int fail(int code, const char *fmt, ...) {
   } while (0)
 
 // ------------------------------------------------------- kernel table --
-typedef void (*solve_fn)(const SolveParams);
-
-struct Variant {
-  int fmt, place, wb;
-  bool exact;
-  int r, nt;
-  int kreg;  // off-diagonal ELL slots held in registers (hybrid variants)
-  solve_fn fn;
-};
-
-#define V_(F, PL, WB, EX, R, NT, MB) \
-  {F, PL, WB, EX, R, NT, 0, (solve_fn)bicgstab_kernel<F, PL, WB, EX, R, NT, MB>}
-#define VK_(F, R, NT, MB, KR) \
-  {F, PLACE_SMEM, 9, true, R, NT, KR, (solve_fn)bicgstab_kernel<F, PLACE_SMEM, 9, true, R, NT, MB, KR>}
-#define V_FP(WB, EX, R, NT, MB)                                                         \
-  V_(FMT_ELL, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_ELL, PLACE_STREAM, WB, EX, R, NT, MB), \
-      V_(FMT_DIA, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_DIA, PLACE_STREAM, WB, EX, R, NT, MB), \
-      V_(FMT_CSR, PLACE_SMEM, WB, EX, R, NT, MB), V_(FMT_CSR, PLACE_STREAM, WB, EX, R, NT, MB)
-
-// W = 9 (the paper's 9-point stencil) gets exact-width variants; any other
-// width <= 16 runs the generic WB = 16 variants with a per-slot test.
-static const Variant kVariants[] = {
-    V_FP(9, true, 1, 256, 2),   V_FP(9, true, 2, 256, 2),   V_FP(9, true, 4, 256, 2),
-    V_FP(9, true, 4, 512, 1),   V_FP(16, false, 1, 256, 2), V_FP(16, false, 2, 256, 2),
-    V_FP(16, false, 4, 256, 2), V_FP(16, false, 4, 512, 1),
-    // experimental hybrid: 128 threads x 8 rows, 2 CTAs/SM, slots 1..KREG in registers
-    VK_(FMT_DIA, 8, 128, 2, 0), VK_(FMT_DIA, 8, 128, 2, 2), VK_(FMT_DIA, 8, 128, 2, 4),
-    VK_(FMT_DIA, 8, 128, 2, 6), VK_(FMT_DIA, 8, 128, 2, 8),
-};
-
-// Persistent register-resident variants (PLACE_REGS): ELL/DIA, W = 9.
-typedef void (*persist_fn)(const SolveParams, unsigned long long *);
-struct PVariant {
-  int fmt, r;
-  persist_fn fn;
-};
-#define PV_(F, R) {F, R, (persist_fn)bicgstab_persist_kernel<F, 9, true, R, 256>}
-static const PVariant kPVariants[] = {PV_(FMT_DIA, 1), PV_(FMT_DIA, 2), PV_(FMT_DIA, 4),
-                                      PV_(FMT_ELL, 1), PV_(FMT_ELL, 2), PV_(FMT_ELL, 4)};
+// The instantiations live in k_generic.cu / k_special.cu / k_line.cu
+// (compiled in parallel); variants.h declares the tables.
 static const PVariant *find_pvariant(int fmt, int r) {
-  for (const PVariant &v : kPVariants)
-    if (v.fmt == fmt && v.r == r) return &v;
+  int cnt = 0;
+  const PVariant *t = variants_persist(&cnt);
+  for (int i = 0; i < cnt; ++i)
+    if (t[i].fmt == fmt && t[i].r == r) return &t[i];
   return nullptr;
 }
 
-// Cluster variants (PLACE_CLUSTER): one system per cluster of C CTAs of
-// 128 threads x 8 rows (1024 rows per CTA), DIA, W = 9.
-struct CVariant {
-  int c, kreg, rounds;
-  solve_fn fn;
-};
-#define CV_(C, KR, RD) \
-  {C, KR, RD, (solve_fn)bicgstab_cluster_kernel<FMT_DIA, 9, true, 8, 128, KR, C, RD>}
-#define CV_ALLC(KR, RD) \
-  CV_(2, KR, RD), CV_(3, KR, RD), CV_(4, KR, RD), CV_(5, KR, RD), CV_(6, KR, RD), \
-      CV_(7, KR, RD), CV_(8, KR, RD)
-// TMEM-resident values (PLACE_TMEM): 128 threads x 8 rows, G rows per load group.
-struct TVariant {
-  int nt, r, g, rounds;
-  solve_fn fn;
-};
-static const TVariant kTVariants[] = {
-    {128, 8, 1, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
-    {128, 8, 2, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
-    {128, 8, 4, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>},
-    // (2-round schedule variants measured 6.1-6.4 vs 6.9 M sys/s: removed)
-    {256, 4, 1, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 1>},
-    {256, 4, 2, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 2>}};
-
-// (a 2-round schedule spills at 255 registers and measured slower at n = 4032)
-static const CVariant kCVariants[] = {CV_ALLC(4, 3), CV_ALLC(2, 3)};
-// cluster plan with TMEM-resident values (kreg field unused: -1)
-#define CVT_(C) {C, -1, 3, (solve_fn)bicgstab_cluster_tmem_kernel<8, 128, C>}
-static const CVariant kCTVariants[] = {CVT_(2), CVT_(3), CVT_(4), CVT_(5),
-                                       CVT_(6), CVT_(7), CVT_(8)};
 static const CVariant *find_cvariant(int c, int kreg, int rounds) {
-  for (const CVariant &v : kCVariants)
-    if (v.c == c && v.kreg == kreg && v.rounds == rounds) return &v;
+  int cnt = 0;
+  const CVariant *t = variants_cluster(&cnt);
+  for (int i = 0; i < cnt; ++i)
+    if (t[i].c == c && t[i].kreg == kreg && t[i].rounds == rounds) return &t[i];
   return nullptr;
 }
 
 static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r, int nt,
                                    int kreg = 0) {
-  for (const Variant &v : kVariants)
+  int cnt = 0;
+  const Variant *t = variants_generic(&cnt);
+  for (int i = 0; i < cnt; ++i) {
+    const Variant &v = t[i];
     if (v.fmt == fmt && v.place == place && v.wb == wb && v.exact == exact && v.r == r &&
         v.nt == nt && v.kreg == kreg)
       return &v;
+  }
   return nullptr;
 }
 
@@ -151,6 +93,8 @@ struct bsolve_plan {
   const PVariant *pvar = nullptr;    // persistent kernel when place == PLACE_REGS
   const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
   solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
+  int line_nx = 0;                   // > 0: line-tiled TMEM kernel for an NX-wide 9-point grid
+  int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};  // its canonical offset -> ELL slot map
   persist_fn var_tmem_p = nullptr;   // persistent TMEM kernel (aligned buffers)
   int smem_bytes_tmem_p = 0, grid_tmem_p = 0;
   int cluster = 0;                   // CTAs per system (cluster plan)
@@ -460,8 +404,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       const bool ctmem = opt.reg_slots == 0 && !(ctenv && atoi(ctenv) == 0);
       h->cvar = nullptr;
       if (ctmem) {
-        for (const CVariant &v : kCTVariants)
-          if (v.c == c) h->cvar = &v;
+        int cnt = 0;
+        const CVariant *t = variants_cluster_tmem(&cnt);
+        for (int i = 0; i < cnt; ++i)
+          if (t[i].c == c) h->cvar = &t[i];
       } else {
         h->cvar = find_cvariant(c, kr, 3);
       }
@@ -503,45 +449,96 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->grid_persist = ncl;
     }
   }
-  // ---- TMEM plan: values in tensor memory (DESIGN.md "Kernels" 9) ---------
-  // Auto for 9-point stencils up to 1024 rows (measured fastest: 6.9 M sys/s
-  // vs 5.5 for the register hybrid at n = 992).
-  const bool tmem_ok = h->kfmt == FMT_DIA && W == 9 && n <= 1024;
+  // ---- TMEM plan: values in tensor memory (DESIGN.md "Kernels" 9, 10) -----
+  // Auto for 9-point stencils up to 1024 rows (measured fastest at n = 992).
+  // Line-tiled variant (DESIGN.md "Kernels" 10): the pattern is a 2D 9-point
+  // (or 5-point, ...) stencil on an NX-wide grid for a compiled NX, i.e. every
+  // slot offset is one of {+-1, +-NX, +-NX+-1}; it is preferred whenever it
+  // applies.  Developer knobs: BSOLVE_TMEM_LINE=0 keeps the strided kernel,
+  // BSOLVE_TMEM_GROUP = rows per TMEM load group.
+  const char *genv = getenv("BSOLVE_TMEM_GROUP");
+  const LVariant *line_v = nullptr;
+  int line_c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
+  {
+    const char *lenv = getenv("BSOLVE_TMEM_LINE");
+    const bool line_on = !(lenv && atoi(lenv) == 0) && opt.block_threads == 0 &&
+                         opt.reg_slots == 0 && h->kfmt == FMT_DIA && W <= 9 && n <= 1024;
+    int lcnt = 0;
+    const LVariant *lv = line_on ? variants_line(&lcnt) : nullptr;
+    const int lg = genv ? atoi(genv) : 4;  // measured best: 7.33 vs 7.05 (G=2) M sys/s
+    const char *rowsenv = getenv("BSOLVE_TMEM_LINE_ROWS");  // rows per thread: 8 or 4
+    const int lr = rowsenv ? atoi(rowsenv) : 8;
+    // first pass: the requested geometry; second pass: any variant for the grid
+    for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
+      if (i < lcnt && (lv[i % lcnt].g != lg || lv[i % lcnt].r != lr)) continue;
+      const LVariant &cand = lv[i % lcnt];
+      const int NX = cand.nx;
+      const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
+      int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
+      bool ok = true;
+      for (int k = 1; k < W && ok; ++k) {
+        bool real = false;  // slot k holds at least one entry of the pattern
+        for (int r = 0; r < n && !real; ++r) real = h->h_csr2ell[(size_t)k * n + r] >= 0;
+        if (!real) continue;
+        const int o = h->doff[k] / 8;
+        int c = 0;
+        while (c < 8 && canon[c] != o) ++c;
+        if (c == 8 || c2s[c] >= 0) ok = false;
+        else c2s[c] = k;
+      }
+      if (!ok) continue;
+      line_v = &cand;
+      for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
+    }
+  }
+  const bool tmem_ok = (h->kfmt == FMT_DIA && W == 9 && n <= 1024) || line_v;
   const bool tmem_auto = opt.placement == BSOLVE_PLACE_AUTO && opt.block_threads == 0 &&
                          opt.reg_slots == 0 && tmem_ok;
   if (h->place != PLACE_CLUSTER && (opt.placement == BSOLVE_PLACE_TMEM || tmem_auto)) {
     if (!tmem_ok)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                             "TMEM placement needs a 9-point stencil (DIA) pattern, n <= 1024"));
-    // developer knobs: rows per TMEM load group, threads per CTA
-    const char *genv = getenv("BSOLVE_TMEM_GROUP");
-    const char *tenv = getenv("BSOLVE_TMEM_THREADS");
-    const int ntsel = opt.block_threads ? opt.block_threads : (tenv ? atoi(tenv) : 128);
-    const int gsel = genv ? atoi(genv) : (ntsel == 128 ? 4 : 2);
-    const char *renv = getenv("BSOLVE_TMEM_ROUNDS");  // developer knob: reduction rounds
-    const int rsel = renv ? atoi(renv) : 3;
-    for (const TVariant &v : kTVariants)
-      if (v.g == gsel && v.nt == ntsel && v.rounds == rsel) {
-        h->var_tmem = v.fn;
-        h->nt = v.nt;
-        h->r = v.r;
-      }
-    if (!h->var_tmem)
-      return fail_free(fail(BSOLVE_ERR_INVALID, "no TMEM variant for %d threads, group %d", ntsel,
-                            gsel));
     h->place = PLACE_TMEM;
     h->n_pad = (n + 1) & ~1;
     h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
-    h->smem_bytes =
-        h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * (h->nt / 32) * 8 + 16;
+    if (line_v) {
+      h->line_nx = line_v->nx;
+      h->var_tmem = line_v->fn;
+      h->smem_bytes = line_v->smem_bytes;
+      for (int c = 0; c < 8; ++c) h->c2s[c] = line_c2s[c];
+      h->nt = 1024 / line_v->r;
+      h->r = line_v->r;
+    } else {
+      // developer knobs: rows per TMEM load group, threads per CTA
+      const char *tenv = getenv("BSOLVE_TMEM_THREADS");
+      const int ntsel = opt.block_threads ? opt.block_threads : (tenv ? atoi(tenv) : 128);
+      const int gsel = genv ? atoi(genv) : (ntsel == 128 ? 4 : 2);
+      const char *renv = getenv("BSOLVE_TMEM_ROUNDS");  // developer knob: reduction rounds
+      const int rsel = renv ? atoi(renv) : 3;
+      int tcnt = 0;
+      const TVariant *tv = variants_tmem(&tcnt);
+      for (int i = 0; i < tcnt; ++i)
+        if (tv[i].g == gsel && tv[i].nt == ntsel && tv[i].rounds == rsel) {
+          h->var_tmem = tv[i].fn;
+          h->nt = tv[i].nt;
+          h->r = tv[i].r;
+        }
+      if (!h->var_tmem)
+        return fail_free(fail(BSOLVE_ERR_INVALID, "no TMEM variant for %d threads, group %d",
+                              ntsel, gsel));
+      h->smem_bytes =
+          h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * (h->nt / 32) * 8 + 16;
+    }
     if (h->smem_bytes > smem_optin)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM plan needs %d B of SMEM", h->smem_bytes));
     ce = cudaFuncSetAttribute((const void *)h->var_tmem,
                               cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
     if (ce != cudaSuccess)
       return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+    // the line kernel stages nothing in SMEM (~10 KB per CTA): leave most of
+    // the unified L1 to the 16-byte value loads
     cudaFuncSetAttribute((const void *)h->var_tmem, cudaFuncAttributePreferredSharedMemoryCarveout,
-                         cudaSharedmemCarveoutMaxShared);
+                         h->line_nx ? 25 : (int)cudaSharedmemCarveoutMaxShared);
     ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, h->nt,
                                                        h->smem_bytes);
     if (ce != cudaSuccess || h->ctas_per_sm < 1)
@@ -552,10 +549,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     // launch, 6.89 vs 6.91 M sys/s -- the co-resident CTA already hides a
     // CTA's start-up)
     const char *penv = getenv("BSOLVE_TMEM_PERSIST");
-    const bool persist = (penv && atoi(penv) == 1) && h->nt == 128 && h->r == 8 &&
+    const bool persist = (penv && atoi(penv) == 1) && !h->line_nx && h->nt == 128 && h->r == 8 &&
                          n % 2 == 0 && (h->sys_stride * 8) % 16 == 0;
     if (persist) {
-      h->var_tmem_p = (persist_fn)bicgstab_tmem_persist_kernel<8, 128, 4>;
+      h->var_tmem_p = variant_tmem_persist();
       h->smem_bytes_tmem_p = h->smem_vals * 8 + 2 * h->n_pad * 8 +
                              (h->n_pad + 2 * h->guard) * 8 + 16 * 4 * 8 + 32;
       if (h->smem_bytes_tmem_p > smem_optin ||
@@ -735,7 +732,7 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->kl = h->kl;
   info->ku = h->ku;
   info->device = h->device;
-  info->kernel_mode = h->kfmt;
+  info->kernel_mode = h->line_nx ? 4 : h->kfmt;
   return BSOLVE_OK;
 }
 
@@ -786,10 +783,11 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   P.n_pad = h->n_pad;
   P.guard = h->guard;
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
+  for (int c = 0; c < 8; ++c) P.c2s[c] = h->c2s[c];
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)
-    if (h->var_tmem_p && aligned) {
+    if (h->var_tmem_p && aligned && !h->line_nx) {
       const int grid = (int)std::min<long long>(h->grid_tmem_p, count);
       h->var_tmem_p<<<grid, h->nt, h->smem_bytes_tmem_p, stream>>>(P, h->d_ctr);
     } else {

@@ -1,0 +1,19 @@
+// k_line.cu -- instantiations of the line-tiled TMEM kernel for 2D 9-point
+// stencils (line_kernel.cuh): grid widths NX with 8 | rows per thread, G rows
+// per TMEM load group.  NX = 32 is the paper's 32 x 31 velocity grid
+// (PAPER.md:519-530); NX = 31 its transpose (tests).  Launched from bsolve.cu.
+#include "line_kernel.cuh"
+#include "variants.h"
+
+using namespace bsolve;
+
+#define LV_(NX, R, G)                                                                   \
+  {NX, R, G, (R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 + 16,       \
+   (solve_fn)bicgstab_tmem_line_kernel<NX, R, G>}
+static const LVariant kLVariants[] = {LV_(32, 8, 2), LV_(32, 8, 4), LV_(32, 4, 2),
+                                      LV_(32, 4, 4), LV_(31, 8, 4), LV_(31, 4, 2)};
+
+const LVariant *variants_line(int *count) {
+  *count = (int)(sizeof(kLVariants) / sizeof(kLVariants[0]));
+  return kLVariants;
+}

@@ -54,6 +54,7 @@ struct SolveParams {
   int n_pad;                // doubles of the gather buffer body (even)
   int guard;                // zero doubles before and after the gather body (DIA)
   int doff[kMaxW];          // DIA: byte offset d_k * 8 of slot k
+  int c2s[8];               // line-tiled stencil plan: ELL slot of canonical offset c, -1 none
 };
 
 // ------------------------------------------------------------ PTX helpers --
@@ -462,7 +463,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1
       if (it >= P.maxiter) break;
       if (bad(rho)) { st = SYS_BREAKDOWN; break; }
-      const double beta = (rho / rho_old) * (alpha / omega);  // R2
+      const double beta = (rho * alpha) / (rho_old * omega);  // R2, one division
       // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
       double ph[R];
 #pragma unroll
@@ -476,32 +477,28 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       spmv(ph, v);
       ++it;
       // a7: alpha = rho / (r^ . v)
-      double rv[1] = {0.0};
-#pragma unroll
-      for (int j = 0; j < R; ++j) rv[0] += rh[j] * v[j];
+      double rv[1];
+      rv[0] = rows_sum<R>([&](int j) { return rh[j] * v[j]; });
       comm.template sum<1>(rv);
       if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
       alpha = rho / rv[0];                                 // R3
       // s = r - alpha v ; publish s^ = d s (all SpMV-1 reads finished: the
       // barrier in the reduction above separates them)
       double s[R], sh[R];
-      double ts[3] = {0.0, 0.0, 0.0};  // t.s, t.t, s.s
+      double ts[3];  // t.s, t.t, s.s
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         s[j] = r[j] - alpha * v[j];
-        ts[2] += s[j] * s[j];
         sh[j] = d[j] * s[j];
         comm.publish(j, sh[j]);
       }
       comm.sync();  // publish s^
+      ts[2] = rows_sum<R>([&](int j) { return s[j] * s[j]; });
       // a9: t = A s^ (speculative when stop test 2 fires)
       double t[R];
       spmv(sh, t);
-#pragma unroll
-      for (int j = 0; j < R; ++j) {
-        ts[0] += t[j] * s[j];
-        ts[1] += t[j] * t[j];
-      }
+      ts[0] = rows_sum<R>([&](int j) { return t[j] * s[j]; });
+      ts[1] = rows_sum<R>([&](int j) { return t[j] * t[j]; });
       comm.template sum<3>(ts);
       if (sqrt(ts[2]) < tau) {                             // stop test 2
 #pragma unroll
@@ -512,14 +509,14 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
       omega = ts[0] / ts[1];
       if (bad(omega)) { st = SYS_BREAKDOWN; break; }
-      double rr[2] = {0.0, 0.0};
+      double rr[2];
 #pragma unroll
       for (int j = 0; j < R; ++j) {
         x[j] = x[j] + alpha * (d[j] * p[j]) + omega * (d[j] * s[j]);
         r[j] = s[j] - omega * t[j];
-        rr[0] += r[j] * r[j];
-        rr[1] += rh[j] * r[j];
       }
+      rr[0] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
+      rr[1] = rows_sum<R>([&](int j) { return rh[j] * r[j]; });
       rho_old = rho;
       // next iteration's ||r|| and rho = r^ . r in the same single barrier
       comm.template sum<2>(rr);
@@ -542,7 +539,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
         st = SYS_BREAKDOWN;
         break;
       }
-      const double beta = (rho / rho_old) * (alpha / omega);  // R2
+      const double beta = (rho * alpha) / (rho_old * omega);  // R2, one division
       // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
       double ph[R];
 #pragma unroll
@@ -1522,7 +1519,7 @@ __global__ void __launch_bounds__(NT) spmv_kernel(const double *__restrict__ val
 }
 
 // ------------------------------------------------------- CSR -> ELL values --
-__global__ void csr_to_ell_kernel(const double *__restrict__ csr, double *__restrict__ ell,
+static __global__ void csr_to_ell_kernel(const double *__restrict__ csr, double *__restrict__ ell,
                                   const int32_t *__restrict__ src, long long slots, int nnz,
                                   long long total) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;

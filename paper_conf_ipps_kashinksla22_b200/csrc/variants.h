@@ -1,0 +1,51 @@
+// variants.h -- kernel variant tables shared by the host plan (bsolve.cu) and
+// the translation units that instantiate the kernels (k_*.cu).  Splitting the
+// instantiations over several .cu files lets the build compile them in
+// parallel; the tables hold host-side kernel stubs, launched from bsolve.cu.
+#pragma once
+#include <cstdint>
+
+namespace bsolve {
+struct SolveParams;
+}
+
+typedef void (*solve_fn)(const bsolve::SolveParams);
+typedef void (*persist_fn)(const bsolve::SolveParams, unsigned long long *);
+
+// per-system-CTA kernels (bicgstab_kernel), k_generic.cu
+struct Variant {
+  int fmt, place, wb;
+  bool exact;
+  int r, nt;
+  int kreg;  // off-diagonal ELL slots held in registers (hybrid variants)
+  solve_fn fn;
+};
+// persistent register-resident kernels (PLACE_REGS), k_special.cu
+struct PVariant {
+  int fmt, r;
+  persist_fn fn;
+};
+// one system per thread-block cluster (PLACE_CLUSTER), k_special.cu
+struct CVariant {
+  int c, kreg, rounds;
+  solve_fn fn;
+};
+// TMEM-resident values (PLACE_TMEM), k_special.cu
+struct TVariant {
+  int nt, r, g, rounds;
+  solve_fn fn;
+};
+// TMEM + line-tiled 9-point stencil (PLACE_TMEM, kernel_mode 4), k_line.cu
+struct LVariant {
+  int nx, r, g;  // grid width, rows per thread (CTA = 1024 / r threads), TMEM load group
+  int smem_bytes;  // dynamic SMEM of one CTA (gather planes + scratch + TMEM slot)
+  solve_fn fn;
+};
+
+const Variant *variants_generic(int *count);
+const PVariant *variants_persist(int *count);
+const CVariant *variants_cluster(int *count);
+const CVariant *variants_cluster_tmem(int *count);
+const TVariant *variants_tmem(int *count);
+persist_fn variant_tmem_persist();
+const LVariant *variants_line(int *count);

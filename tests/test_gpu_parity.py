@@ -434,10 +434,14 @@ def test_tmem_warm_start_and_determinism():
 
 
 def test_tmem_refuses_non_stencil():
-    pat = X.stencil_pattern(1, 1)  # W = 1: not a 9-point stencil
+    rp, ci = X.random_pattern(200, 6, seed=4)  # not a stencil: no uniform slot offsets
     with pytest.raises(BsolveError) as e:
-        Solver(pat.row_ptr, pat.col_idx, 2, placement="tmem")
+        Solver(rp, ci, 2, placement="tmem")
     assert e.value.code == -3
+    # a diagonal-only pattern is a (degenerate) stencil: the line kernel takes it
+    pat = X.stencil_pattern(1, 1)
+    S = Solver(pat.row_ptr, pat.col_idx, 2, placement="tmem")
+    assert S.info["kernel_mode"] == 4
 
 
 @pytest.mark.parametrize("batch", [3, 296, 1000])
@@ -477,6 +481,94 @@ def test_tmem_schedules(rounds, group, monkeypatch):
     B = X.make_batch(0, 64)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-3)
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
+
+
+# ------------------------------------------ line-tiled TMEM kernel (mode 4) --
+def _five_point(nx, ny):
+    """5-point stencil pattern (the 9-point pattern without its corners)."""
+    pat = X.stencil_pattern(nx, ny)
+    r, c = pat.row_of.astype(int), pat.col_idx.astype(int)
+    keep = (np.abs(c % nx - r % nx) + np.abs(c // nx - r // nx)) <= 1
+    rows, cols = r[keep], c[keep]
+    rp = np.zeros(nx * ny + 1, np.int32)
+    np.add.at(rp, rows + 1, 1)
+    return np.cumsum(rp).astype(np.int32), cols.astype(np.int32)
+
+
+@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32), (32, 5), (31, 31), (32, 32), (32, 1)])
+def test_line_tmem_kernel(nx, ny):
+    """Line-tiled TMEM plan (thread owns 8 consecutive rows, 22 gathers per
+    SpMV): 32x31 (paper grid), its transpose, short grids (idle threads), odd
+    n (scalar loads), n = 1024 (all 128 threads busy), a single grid line."""
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 40, nx=nx, ny=ny)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, placement="tmem")
+    assert g["info"]["kernel_mode"] == 4 and g["info"]["placement"] == 5
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+
+
+def test_line_tmem_five_point_and_random_values():
+    """5-point stencil (canonical corner slots absent -> zero values) with
+    random diagonally dominant values and right-hand sides."""
+    rp, ci = _five_point(32, 31)
+    vals = X.random_dd_values(rp, ci, 24, seed=5, margin=0.5)
+    b = X.random_rhs(24, 992, seed=6)
+    g = gpu_solve(rp, ci, vals, b, placement="tmem")
+    assert g["info"]["kernel_mode"] == 4
+    compare(rp, ci, vals, b, g)
+
+
+def test_line_tmem_matches_strided_plan_and_is_deterministic(monkeypatch):
+    """Line and strided TMEM kernels solve the same batch to the same parity
+    bar; the line kernel is bitwise independent of batch slicing, of x0 = 0
+    vs NULL, and of a misaligned values buffer (scalar-load path)."""
+    B = X.make_batch(0, 300, picard=1)
+    p = B.pattern
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-4)
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
+    assert g["info"]["kernel_mode"] == 4
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+    g2 = gpu_solve(p.row_ptr, p.col_idx, B.values[100:], B.b[100:], x0=x0[100:])
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(g[k][100:], g2[k])
+    monkeypatch.setenv("BSOLVE_TMEM_LINE", "0")
+    gs = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0)
+    monkeypatch.delenv("BSOLVE_TMEM_LINE")
+    assert gs["info"]["kernel_mode"] == 3
+    compare(p.row_ptr, p.col_idx, B.values, B.b, gs, o=o)
+    assert np.abs(gs["iters"].astype(int) - g["iters"].astype(int)).max() <= 2
+    # zero guess: NULL == explicit zeros; misaligned values -> identical results
+    S = Solver(p.row_ptr, p.col_idx, 300)
+    v = to_dev(S.ell_values(B.values))
+    b = to_dev(B.b)
+    xa, ia, ra, sa = S.run(v, b)
+    xz, iz, rz, sz = S.run(v, b, torch.zeros_like(b))
+    vbig = torch.empty(v.numel() + 1, dtype=torch.float64, device="cuda")
+    vbig[1:] = v.reshape(-1)
+    xm, im, rm, sm = S.run(vbig[1:].view_as(v), b)
+    torch.cuda.synchronize()
+    assert torch.equal(xa, xz) and torch.equal(ia, iz)
+    assert torch.equal(xa, xm) and torch.equal(ia, im) and torch.equal(ra, rm)
+
+
+@pytest.mark.parametrize("rows,group,nx,ny", [(8, 2, 32, 31), (4, 2, 32, 31), (4, 4, 32, 31),
+                                               (4, 2, 31, 32), (4, 2, 32, 5), (4, 2, 31, 31)])
+def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
+    """Line kernel with 8 rows x 128 threads or 4 rows x 256 threads per CTA
+    (two warps per TMEM lane quarter) and other TMEM load groups: same parity
+    bar, warm start included."""
+    monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
+    monkeypatch.setenv("BSOLVE_TMEM_LINE_ROWS", str(rows))
+    B = X.make_batch(0, 64, nx=nx, ny=ny)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    assert g["info"]["kernel_mode"] == 4 and g["info"]["rows_per_thread"] == rows
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
     x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-3)
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
