@@ -403,7 +403,14 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   comm.template sum<2>(red3);
   const double bnorm = sqrt(red3[0]);
   const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
+  // stop tests compare squared norms (no sqrt on the critical path) whenever
+  // tau^2 neither underflows nor overflows; sqrt(a) < tau <=> a < tau^2 for
+  // a >= 0 up to the rounding of tau^2 (R7)
+  const double tau2 = tau * tau;
+  const bool sq = tau2 > 1e-300 && tau2 < 1e300;
+  auto below = [&](double nrm2) { return sq ? nrm2 < tau2 : sqrt(nrm2) < tau; };
   double rnorm = sqrt(red3[1]);
+  double rnorm2 = red3[1];  // ||r||^2 of the current r (3-round schedule)
   double rho = red3[1];  // r^ . r with r^ = r
 
   double *xout = P.x + sys * n;
@@ -454,16 +461,19 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
   // rounding of rho differs (fp sums in another order).
   int it = 0, st = -1, exit_kind = 0;
   double rho_old = 1.0, alpha = 1.0, omega = 1.0;
+  double beta_c = 1.0;  // alpha / (rho_old * omega): beta = rho * beta_c (R2)
   double final_res = -1.0;
   bool have_rnorm = true;  // rnorm holds ||r|| of the current r
   for (;;) {
     exit_kind = 0;
     if constexpr (ROUNDS == 3) {
     while (true) {
-      if (rnorm < tau) { exit_kind = 1; break; }          // stop test 1
+      if (below(rnorm2)) { exit_kind = 1; break; }        // stop test 1
       if (it >= P.maxiter) break;
       if (bad(rho)) { st = SYS_BREAKDOWN; break; }
-      const double beta = (rho * alpha) / (rho_old * omega);  // R2, one division
+      // R2: beta = (rho / rho') (alpha / omega); the division alpha / (rho'
+      // omega) was done before the last reduction, off the critical path
+      const double beta = rho * beta_c;
       // a5: p = r + beta (p - omega v); publish p^ = d p for the gather
       double ph[R];
 #pragma unroll
@@ -500,7 +510,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       ts[0] = rows_sum<R>([&](int j) { return t[j] * s[j]; });
       ts[1] = rows_sum<R>([&](int j) { return t[j] * t[j]; });
       comm.template sum<3>(ts);
-      if (sqrt(ts[2]) < tau) {                             // stop test 2
+      if (below(ts[2])) {                                  // stop test 2
 #pragma unroll
         for (int j = 0; j < R; ++j) x[j] = x[j] + alpha * (d[j] * p[j]);
         exit_kind = 2;
@@ -509,6 +519,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
       omega = ts[0] / ts[1];
       if (bad(omega)) { st = SYS_BREAKDOWN; break; }
+      beta_c = alpha / (rho * omega);  // rho becomes rho' below
       double rr[2];
 #pragma unroll
       for (int j = 0; j < R; ++j) {
@@ -520,7 +531,7 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       rho_old = rho;
       // next iteration's ||r|| and rho = r^ . r in the same single barrier
       comm.template sum<2>(rr);
-      rnorm = sqrt(rr[0]);
+      rnorm2 = rr[0];
       rho = rr[1];
     }
     } else {
@@ -617,8 +628,9 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
       p[j] = 0.0;
       v[j] = 0.0;
     }
-    rho_old = alpha = omega = 1.0;
+    rho_old = alpha = omega = beta_c = 1.0;
     rnorm = final_res;
+    rnorm2 = tr2;
     have_rnorm = true;
     rho = tr2;
     final_res = -1.0;

@@ -64,9 +64,12 @@ struct LineComm {
       : gq(sg + L::GQ + threadIdx.x), sred(sred_), buf(0), act(act_) {}
   __device__ __forceinline__ int grow(int j) const { return R * threadIdx.x + j; }
   __device__ __forceinline__ bool leader() const { return threadIdx.x == 0; }
-  // every thread writes all R of its entries (0.0 for rows >= n), so the body
-  // [GQ, GQ + NT) of every plane is fully rewritten by each publish
-  __device__ __forceinline__ void publish(int j, double v) { gq[j * L::S] = act[j] ? v : 0.0; }
+  // every thread writes all R of its entries, so the body [GQ, GQ + NT) of
+  // every plane is fully rewritten by each publish.  Rows >= n need no select:
+  // their diagonal and values are 0 and their b, x0 are 0, so every vector
+  // entry of theirs stays 0 (unless a scalar is already non-finite, i.e. the
+  // system breaks down anyway).
+  __device__ __forceinline__ void publish(int j, double v) { gq[j * L::S] = v; }
   __device__ __forceinline__ void sync() { __syncthreads(); }
   template <int K>
   __device__ __forceinline__ void sum(double (&v)[K]) {
