@@ -7,7 +7,8 @@ shares no code with it (see oracle.c for the algorithm and its citations).
 
 Functions mirror oracle.c:
   spmv, dense_solve, banded_solve, bandwidth, bicgstab (one system, with
-  optional invariant trace), batch_bicgstab, batch_banded (host threads).
+  optional invariant trace), gmres (restarted GMRES(m)),
+  batch_bicgstab, batch_krylov, batch_banded (host threads).
 """
 from __future__ import annotations
 
@@ -24,6 +25,8 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 
 STOP_REL_B = 0
 STOP_ABS = 1
+PREC_JACOBI, PREC_NONE = 0, 1
+SOLVER_BICGSTAB, SOLVER_GMRES = 0, 2
 CONVERGED, MAXITER, BREAKDOWN = 0, 1, 2
 
 _lock = threading.Lock()
@@ -69,6 +72,17 @@ def lib():
                                                 C.c_double, C.c_int, C.c_int, C.c_int,
                                                 _P, _P, _P, _P, _P, C.c_int]
             L.oracle_batch_bicgstab.restype = C.c_int
+            L.oracle_bicgstab_p.argtypes = [C.c_int, _P, _P, _P, _P, _P, C.c_double, C.c_int,
+                                            C.c_int, C.c_int, C.c_int, _P, C.POINTER(Result),
+                                            _P]
+            L.oracle_bicgstab_p.restype = C.c_int
+            L.oracle_gmres.argtypes = [C.c_int, _P, _P, _P, _P, _P, C.c_double, C.c_int,
+                                       C.c_int, C.c_int, C.c_int, _P, C.POINTER(Result), _P]
+            L.oracle_gmres.restype = C.c_int
+            L.oracle_batch_krylov.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_int,
+                                              C.c_int, _P, _P, _P, _P, _P, C.c_double, C.c_int,
+                                              C.c_int, C.c_int, _P, _P, _P, _P, _P, C.c_int]
+            L.oracle_batch_krylov.restype = C.c_int
             L.oracle_batch_banded.argtypes = [C.c_int, C.c_int, C.c_int, _P, _P, _P, _P, _P,
                                               _P, C.c_int]
             L.oracle_batch_banded.restype = C.c_int
@@ -122,7 +136,7 @@ def banded_solve(row_ptr, col_idx, val, b):
 
 
 def bicgstab(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, stop=STOP_REL_B,
-             true_res_check=True, trace=False):
+             true_res_check=True, trace=False, precond=PREC_JACOBI):
     """One system through Algorithm 1.  Returns (x, Result[, trace])."""
     rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(b)
     n = rp.size - 1
@@ -130,9 +144,9 @@ def bicgstab(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, stop=ST
     x = np.empty(n)
     R = Result()
     tr = np.full(max(maxiter, 1), np.nan) if trace else None
-    rc = lib().oracle_bicgstab(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x0a), float(tol),
-                               int(maxiter), int(stop), int(bool(true_res_check)), _ptr(x),
-                               C.byref(R), _ptr(tr))
+    rc = lib().oracle_bicgstab_p(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x0a),
+                                 float(tol), int(maxiter), int(stop), int(bool(true_res_check)),
+                                 int(precond), _ptr(x), C.byref(R), _ptr(tr))
     if rc:
         raise MemoryError("oracle_bicgstab")
     if trace:
@@ -172,3 +186,45 @@ def batch_banded(row_ptr, col_idx, values, b, threads=0):
     if rc or np.any(st != 0):
         raise np.linalg.LinAlgError("batch banded LU failed")
     return x
+
+
+def gmres(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, restart=8,
+          stop=STOP_REL_B, precond=PREC_JACOBI, trace=False):
+    """One system through restarted GMRES(restart) (oracle.c oracle_gmres).
+    Returns (x, Result[, trace (iters, 2): |g_{k+1}|, ||b - A x_k||])."""
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(b)
+    n = rp.size - 1
+    x0a = None if x0 is None else _f64(x0)
+    x = np.empty(n)
+    R = Result()
+    tr = np.full(2 * max(maxiter, 1), np.nan) if trace else None
+    rc = lib().oracle_gmres(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x0a), float(tol),
+                            int(maxiter), int(restart), int(stop), int(precond), _ptr(x),
+                            C.byref(R), _ptr(tr))
+    if rc:
+        raise ValueError("oracle_gmres: allocation failure or restart < 1")
+    if trace:
+        return x, R, tr[: 2 * R.iters].reshape(-1, 2)
+    return x, R
+
+
+def batch_krylov(row_ptr, col_idx, values, b, solver=SOLVER_BICGSTAB, precond=PREC_JACOBI,
+                 restart=8, x0=None, tol=1e-10, maxiter=1000, stop=STOP_REL_B,
+                 true_res_check=True, threads=0):
+    """BiCGSTAB or GMRES(restart) with Jacobi or no preconditioner on every
+    system.  Returns dict(x, iters, resnorm, status, restarts)."""
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(values), _f64(b)
+    batch, nnz = v.shape
+    n = rp.size - 1
+    x0a = None if x0 is None else _f64(x0)
+    out = dict(x=np.empty((batch, n)), iters=np.empty(batch, np.int32),
+               resnorm=np.empty(batch), status=np.empty(batch, np.int32),
+               restarts=np.empty(batch, np.int32))
+    rc = lib().oracle_batch_krylov(int(solver), int(precond), int(restart), n, nnz, batch,
+                                   _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x0a), float(tol),
+                                   int(maxiter), int(stop), int(bool(true_res_check)),
+                                   _ptr(out["x"]), _ptr(out["iters"]), _ptr(out["resnorm"]),
+                                   _ptr(out["status"]), _ptr(out["restarts"]), int(threads))
+    if rc:
+        raise ValueError("oracle_batch_krylov failed")
+    return out
