@@ -96,6 +96,23 @@ enum {
                             PAPER.md:869-870)                                  */
 };
 
+/* Krylov solver ("several preconditionable iterative
+ * solvers"; BiCGSTAB is the paper's method, SURVEY.md 8(f) f3 the others). */
+enum {
+  BSOLVE_SOLVER_BICGSTAB = 0, /* Algorithm 1               */
+  BSOLVE_SOLVER_GMRES = 1     /* restarted right-preconditioned GMRES(m)
+                                 (Saad Alg. 6.9/6.11/9.5); every cycle starts
+                                 from the true residual; 2D stencil patterns
+                                 with n <= 1024 (line-tiled TMEM plan)        */
+};
+#define BSOLVE_MAX_RESTART 7
+
+/* Preconditioner M^-1 = diag(d) applied on the right. */
+enum {
+  BSOLVE_PREC_JACOBI = 0, /* d_i = 1 / a_ii (a zero diagonal gives 1)          */
+  BSOLVE_PREC_NONE = 1    /* d_i = 1                                           */
+};
+
 /* Per-system outcome written to status[] (R10). */
 enum {
   BSOLVE_SYS_CONVERGED = 0, /* final TRUE ||b - A x||_2 < tau                 */
@@ -118,6 +135,10 @@ typedef struct bsolve_options {
                               off-diagonal ELL slots held in registers instead
                               of SMEM, 0, 2, 4, 6 or 8 (default 0 = planner's
                               choice: 4)                                      */
+  int solver;              /* BSOLVE_SOLVER_* (default BICGSTAB)               */
+  int precond;             /* BSOLVE_PREC_*   (default JACOBI)                 */
+  int restart;             /* GMRES: Krylov steps per restart cycle m,
+                              1 <= m <= BSOLVE_MAX_RESTART (default 7)        */
 } bsolve_options;
 
 typedef struct bsolve_info {
@@ -134,8 +155,11 @@ typedef struct bsolve_info {
   int device;
   int kernel_mode;         /* 1 CSR column table, 2 ELL column table, 3 DIA:
                               ELL values whose slot k is column row + d_k in
-                              every row (stencils; uniform gather offsets)    */
+                              every row (stencils; uniform gather offsets),
+                              4 LINE: DIA on a 2D grid, each thread owns
+                              consecutive grid rows (DESIGN.md Kernels 10)   */
   int cluster;             /* CTAs per system (PLACE_CLUSTER), else 0        */
+  int solver, precond, restart; /* resolved BSOLVE_SOLVER_*, BSOLVE_PREC_*, m  */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

@@ -20,12 +20,17 @@ ERR_INVALID, ERR_PATTERN, ERR_UNSUPPORTED, ERR_CUDA, ERR_NOMEM = -1, -2, -3, -4,
 FMT_AUTO, FMT_CSR, FMT_ELL = 0, 1, 2
 PLACE_AUTO, PLACE_SMEM, PLACE_STREAM, PLACE_REGS, PLACE_CLUSTER, PLACE_TMEM = 0, 1, 2, 3, 4, 5
 STOP_REL_B, STOP_ABS = 0, 1
+SOLVER_BICGSTAB, SOLVER_GMRES = 0, 1
+PREC_JACOBI, PREC_NONE = 0, 1
+MAX_RESTART = 7
 SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN = 0, 1, 2
 
 _FMT = {"auto": FMT_AUTO, "csr": FMT_CSR, "ell": FMT_ELL}
 _PLACE = {"auto": PLACE_AUTO, "smem": PLACE_SMEM, "stream": PLACE_STREAM, "regs": PLACE_REGS,
           "cluster": PLACE_CLUSTER, "tmem": PLACE_TMEM}
 _STOP = {"rel_b": STOP_REL_B, "rel": STOP_REL_B, "abs": STOP_ABS}
+_SOLVER = {"bicgstab": SOLVER_BICGSTAB, "gmres": SOLVER_GMRES}
+_PREC = {"jacobi": PREC_JACOBI, "none": PREC_NONE}
 
 
 class BsolveError(RuntimeError):
@@ -37,14 +42,15 @@ class BsolveError(RuntimeError):
 class Options(C.Structure):
     _fields_ = [("format", C.c_int), ("placement", C.c_int), ("stop", C.c_int),
                 ("true_residual_check", C.c_int), ("device", C.c_int),
-                ("block_threads", C.c_int), ("reg_slots", C.c_int)]
+                ("block_threads", C.c_int), ("reg_slots", C.c_int), ("solver", C.c_int),
+                ("precond", C.c_int), ("restart", C.c_int)]
 
 
 class Info(C.Structure):
     _fields_ = [(f, C.c_int) for f in (
         "n", "nnz", "batch", "ell_width", "format", "placement", "block_threads",
         "rows_per_thread", "smem_bytes", "ctas_per_sm", "num_sms", "grid", "kl", "ku", "device",
-        "kernel_mode", "cluster")]
+        "kernel_mode", "cluster", "solver", "precond", "restart")]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -128,16 +134,18 @@ def probe_smem_bandwidth(device: int = -1):
 
 
 class Solver:
-    """Batched Jacobi-preconditioned BiCGSTAB over one shared sparsity pattern.
+    """Batched preconditioned Krylov solve over one shared sparsity pattern.
 
     Solver(row_ptr, col_idx, batch, format="ell", placement="auto",
-           stop="rel_b", true_residual_check=True, device=None)
+           stop="rel_b", true_residual_check=True, device=None,
+           solver="bicgstab" | "gmres", precond="jacobi" | "none", restart=7)
     .run(values, b, x0=None, tol=1e-10, maxiter=1000) -> (x, iters, resnorm, status)
     """
 
     def __init__(self, row_ptr, col_idx, batch: int, *, format: str = "ell",
                  placement: str = "auto", stop: str = "rel_b", true_residual_check: bool = True,
-                 device: int | None = None, block_threads: int = 0, reg_slots: int = 0):
+                 device: int | None = None, block_threads: int = 0, reg_slots: int = 0,
+                 solver: str = "bicgstab", precond: str = "jacobi", restart: int = MAX_RESTART):
         L = lib()
         rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
         ci = np.ascontiguousarray(col_idx, dtype=np.int32)
@@ -152,6 +160,9 @@ class Solver:
         opt.device = -1 if device is None else int(device)
         opt.block_threads = int(block_threads)
         opt.reg_slots = int(reg_slots)
+        opt.solver = _SOLVER[solver]
+        opt.precond = _PREC[precond]
+        opt.restart = int(restart)
         h = _P()
         check(L.bsolve_create(C.byref(h), self.n, self.batch, rp.ctypes.data, ci.ctypes.data,
                               C.byref(opt)))

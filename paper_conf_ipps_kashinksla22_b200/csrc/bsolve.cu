@@ -82,6 +82,7 @@ static const Variant *find_variant(int fmt, int place, int wb, bool exact, int r
 // ------------------------------------------------------------- handle --
 struct bsolve_plan {
   int n = 0, nnz = 0, batch = 0, W = 0, wb = 0;
+  int solver = 0, precond = 0, restart = 0;
   int fmt = 0, place = 0, stop = 0, trc = 1, device = 0;
   int nt = 0, r = 0, smem_bytes = 0, smem_vals = 0, n_pad = 0, ctas_per_sm = 0, num_sms = 0;
   int kl = 0, ku = 0;
@@ -122,6 +123,9 @@ extern "C" void bsolve_default_options(bsolve_options *o) {
   o->device = -1;
   o->block_threads = 0;
   o->reg_slots = 0;
+  o->solver = BSOLVE_SOLVER_BICGSTAB;
+  o->precond = BSOLVE_PREC_JACOBI;
+  o->restart = BSOLVE_MAX_RESTART;
 }
 
 static void free_plan(bsolve_plan *h) {
@@ -296,6 +300,14 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                 opt.block_threads);
   if (opt.reg_slots < 0 || opt.reg_slots > 8 || (opt.reg_slots & 1))
     return fail(BSOLVE_ERR_INVALID, "reg_slots must be 0, 2, 4, 6 or 8 (got %d)", opt.reg_slots);
+  if (opt.solver != BSOLVE_SOLVER_BICGSTAB && opt.solver != BSOLVE_SOLVER_GMRES)
+    return fail(BSOLVE_ERR_INVALID, "bad solver %d", opt.solver);
+  if (opt.precond != BSOLVE_PREC_JACOBI && opt.precond != BSOLVE_PREC_NONE)
+    return fail(BSOLVE_ERR_INVALID, "bad preconditioner %d", opt.precond);
+  if (opt.solver == BSOLVE_SOLVER_GMRES && (opt.restart < 1 || opt.restart > BSOLVE_MAX_RESTART))
+    return fail(BSOLVE_ERR_INVALID, "GMRES restart must be 1..%d (got %d)", BSOLVE_MAX_RESTART,
+                opt.restart);
+  static_assert(BSOLVE_MAX_RESTART == kMaxRestart, "header and kernel restart bound");
 
   std::vector<int32_t> diag;
   int W = 0;
@@ -317,6 +329,9 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->fmt = opt.format == BSOLVE_FMT_CSR ? FMT_CSR : FMT_ELL;
   h->stop = opt.stop;
   h->trc = opt.true_residual_check ? 1 : 0;
+  h->solver = opt.solver;
+  h->precond = opt.precond;
+  h->restart = opt.solver == BSOLVE_SOLVER_GMRES ? opt.restart : 0;
   h->sys_stride = h->fmt == FMT_ELL ? (long long)W * n : nnz;
 
   // bandwidth (for bsolve_info; the banded structure is not used by the solve)
@@ -461,8 +476,12 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   int line_c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
   {
     const char *lenv = getenv("BSOLVE_TMEM_LINE");
-    const bool line_on = !(lenv && atoi(lenv) == 0) && opt.block_threads == 0 &&
-                         opt.reg_slots == 0 && h->kfmt == FMT_DIA && W <= 9 && n <= 1024;
+    const bool gm = opt.solver == BSOLVE_SOLVER_GMRES;
+    const bool line_on = (gm || !(lenv && atoi(lenv) == 0)) && opt.block_threads == 0 &&
+                         opt.reg_slots == 0 && h->kfmt == FMT_DIA && W <= 9 && n <= 1024 &&
+                         h->place != PLACE_CLUSTER &&
+                         (opt.placement == BSOLVE_PLACE_AUTO ||
+                          opt.placement == BSOLVE_PLACE_TMEM);
     int lcnt = 0;
     const LVariant *lv = line_on ? variants_line(&lcnt) : nullptr;
     const int lg = genv ? atoi(genv) : 4;  // measured best: 7.33 vs 7.05 (G=2) M sys/s
@@ -470,8 +489,9 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const int lr = rowsenv ? atoi(rowsenv) : 8;
     // first pass: the requested geometry; second pass: any variant for the grid
     for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
-      if (i < lcnt && (lv[i % lcnt].g != lg || lv[i % lcnt].r != lr)) continue;
       const LVariant &cand = lv[i % lcnt];
+      if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
+      if (i < lcnt && (cand.g != lg || cand.r != lr)) continue;
       const int NX = cand.nx;
       const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
       int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
@@ -491,6 +511,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
     }
   }
+  if (opt.solver == BSOLVE_SOLVER_GMRES && !line_v)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                          "GMRES needs a 2D stencil pattern (9- or 5-point, grid width 31 or "
+                          "32) with n <= 1024 and placement AUTO or TMEM"));
   const bool tmem_ok = (h->kfmt == FMT_DIA && W == 9 && n <= 1024) || line_v;
   const bool tmem_auto = opt.placement == BSOLVE_PLACE_AUTO && opt.block_threads == 0 &&
                          opt.reg_slots == 0 && tmem_ok;
@@ -535,10 +559,17 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                               cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
     if (ce != cudaSuccess)
       return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
-    // the line kernel stages nothing in SMEM (~10 KB per CTA): leave most of
-    // the unified L1 to the 16-byte value loads
+    // the line kernel stages nothing in SMEM (~10 KB per CTA; + the Krylov
+    // basis for GMRES): carve out just enough shared memory for 2 CTAs per SM
+    // and leave the rest of the unified L1 to the 16-byte value loads
+    int carve = (int)cudaSharedmemCarveoutMaxShared;
+    if (h->line_nx) {
+      const long long need = 2LL * (h->smem_bytes + 1024);
+      carve = (int)std::min<long long>(100, (need * 100 + prop.sharedMemPerMultiprocessor - 1) /
+                                                 prop.sharedMemPerMultiprocessor + 5);
+    }
     cudaFuncSetAttribute((const void *)h->var_tmem, cudaFuncAttributePreferredSharedMemoryCarveout,
-                         h->line_nx ? 25 : (int)cudaSharedmemCarveoutMaxShared);
+                         carve);
     ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, h->nt,
                                                        h->smem_bytes);
     if (ce != cudaSuccess || h->ctas_per_sm < 1)
@@ -733,6 +764,9 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->ku = h->ku;
   info->device = h->device;
   info->kernel_mode = h->line_nx ? 4 : h->kfmt;
+  info->solver = h->solver;
+  info->precond = h->precond;
+  info->restart = h->restart;
   return BSOLVE_OK;
 }
 
@@ -784,6 +818,8 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   P.guard = h->guard;
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
   for (int c = 0; c < 8; ++c) P.c2s[c] = h->c2s[c];
+  P.precond = h->precond;
+  P.restart = h->restart;
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)

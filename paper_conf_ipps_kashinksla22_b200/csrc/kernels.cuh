@@ -34,7 +34,10 @@ enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
 enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3, PLACE_CLUSTER = 4, PLACE_TMEM = 5 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
+enum { PREC_JACOBI = 0, PREC_NONE = 1 };     // PRECOND(y) = d .* y
+enum { SOLVER_BICGSTAB = 0, SOLVER_GMRES = 1 };
 constexpr int kMaxW = 16;
+constexpr int kMaxRestart = 7;  // GMRES: CGS2 pass 2 reduces kMaxRestart + 1 <= 8 values at once
 
 struct SolveParams {
   const double *values;     // [batch][sys_stride]
@@ -55,7 +58,14 @@ struct SolveParams {
   int guard;                // zero doubles before and after the gather body (DIA)
   int doff[kMaxW];          // DIA: byte offset d_k * 8 of slot k
   int c2s[8];               // line-tiled stencil plan: ELL slot of canonical offset c, -1 none
+  int precond;              // PREC_JACOBI (d = 1 / a_ii) or PREC_NONE (d = 1)
+  int restart;              // GMRES: Krylov steps per restart cycle (1 .. kMaxRestart)
 };
+
+// Jacobi entry d_i for diagonal a (R11: zero diagonal -> 1); 1 without preconditioner.
+__device__ __forceinline__ double jacobi_inv(int precond, double a) {
+  return (precond == PREC_JACOBI && a != 0.0) ? 1.0 / a : 1.0;
+}
 
 // ------------------------------------------------------------ PTX helpers --
 __device__ __forceinline__ uint32_t smem_addr(const void *p) {
@@ -760,7 +770,7 @@ __global__ void __launch_bounds__(NT, MINB) bicgstab_kernel(const SolveParams P)
     for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k)  // hybrid: slots 1..KREG -> registers
       m.vreg[j][k] = (PLACE == PLACE_STREAM) ? __ldg(V + m.vbase[j] + (k + 1) * n)
                                              : V[m.vbase[j] + (k + 1) * n];
-    d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+    d[j] = jacobi_inv(P.precond, a);
   }
 
   CtaComm<R, NT> comm(sg, sred, m.act);
@@ -867,7 +877,7 @@ __global__ void __launch_bounds__(NT, 1) bicgstab_persist_kernel(const SolvePara
       for (int k = 1; k < WB; ++k)
         m.vreg[j][k - 1] = (EXACT || k < P.W) ? sval[k * n + m.vbase[j]] : 0.0;
       const double a = m.act[j] ? m.a0[j] : 0.0;
-      d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+      d[j] = jacobi_inv(P.precond, a);
       bv[j] = m.act[j] ? sb[m.vbase[j]] : 0.0;
       r[j] = bv[j];
       x[j] = (P.x0 && m.act[j]) ? sx0[m.vbase[j]] : 0.0;
@@ -951,11 +961,11 @@ __device__ __forceinline__ void tmem_wait_st() {
 template <int R, int WB>
 __device__ __forceinline__ void tmem_fill(uint32_t tlane, const double *sval, int stride,
                                           const int (&vrow)[R], const bool (&act)[R],
-                                          double (&a0)[R], double (&d)[R]) {
+                                          double (&a0)[R], double (&d)[R], int precond) {
 #pragma unroll
   for (int j = 0; j < R; ++j) {
     a0[j] = act[j] ? sval[vrow[j]] : 0.0;
-    d[j] = (a0[j] != 0.0) ? 1.0 / a0[j] : 1.0;
+    d[j] = jacobi_inv(precond, a0[j]);
     uint32_t w[16];
 #pragma unroll
     for (int k = 1; k < WB; ++k) {
@@ -1078,7 +1088,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
   if (use_tma) mbar_wait_parity(mbar, 0);
   else __syncthreads();
   // ---- values: diagonal -> register, slots 1..8 -> this thread's TMEM lane --
-  tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d);
+  tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d, P.precond);
 
   CtaComm<R, NT> comm(sg, sred, act);
   bicgstab_core<R, NT, false, ROUNDS>(
@@ -1173,7 +1183,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_persist_kernel(const Solv
     mbar_wait_parity(mbar, phase);
     phase ^= 1u;
     double x[R], r[R], d[R], a0[R], bv[R];
-    tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d);
+    tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d, P.precond);
 #pragma unroll
     for (int j = 0; j < R; ++j) {
       bv[j] = act[j] ? sb[vrow[j]] : 0.0;
@@ -1401,7 +1411,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_kernel(const SolvePara
   for (int j = 0; j < R; ++j) {
     const double a = m.act[j] ? sval[m.vbase[j]] : 0.0;  // slot 0 = diagonal
     m.a0[j] = a;
-    d[j] = (a != 0.0) ? 1.0 / a : 1.0;
+    d[j] = jacobi_inv(P.precond, a);
 #pragma unroll
     for (int k = 0; k < (KREG > 0 ? KREG : 0); ++k) m.vreg[j][k] = sval[m.vbase[j] + (k + 1) * RPC];
   }
@@ -1486,7 +1496,7 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_cluster_tmem_kernel(const Solv
   }
   cl.sync();  // every CTA of the cluster runs (DSMEM and its mbarriers are live)
   mbar_wait_parity(mbar, 0);
-  tmem_fill<R, WB>(tlane, sval, RPC, vrow, act, a0, d);
+  tmem_fill<R, WB>(tlane, sval, RPC, vrow, act, a0, d, P.precond);
   ClusterComm<R, NT, C> comm(sg, sred, mbar + 1, rank, n, P.guard, act);
   bicgstab_core<R, NT, false, 3>(
       P, sys, x, r, d, act, r, comm, [&](const double(&own)[R], double(&y)[R]) {

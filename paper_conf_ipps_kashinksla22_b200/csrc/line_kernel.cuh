@@ -30,6 +30,7 @@
 // the diagonal stays in a register.  Every SpMV reads them back with
 // tcgen05.ld, software-pipelined one row group ahead of the FMAs.
 #pragma once
+#include "gmres.cuh"
 #include "kernels.cuh"
 
 namespace bsolve {
@@ -134,8 +135,10 @@ __device__ __forceinline__ void line_spmv(uint32_t tlane, const double *gq, cons
 // One CTA of NT = 1024 / R threads per system (n <= 1024), 2 CTAs per SM.
 // TMEM: 16 columns per row; with 256 threads warps w and w + 4 share lane
 // quarter w % 4 and use consecutive column ranges (128 columns per CTA).
-//   SMEM: [gather planes: R * S] [reduction scratch: 16 * NWARP] [TMEM base]
-template <int NX, int R, int G>
+//   SMEM: [gather planes: R * S] [reduction scratch: 16 * NWARP] [TMEM base: 16 B]
+//         GMRES only: [Krylov basis: kMaxRestart * R * NT] [R factor: kMaxRestart^2]
+// SOLVER: SOLVER_BICGSTAB (Algorithm 1) or SOLVER_GMRES (gmres.cuh).
+template <int NX, int R, int G, int SOLVER = SOLVER_BICGSTAB>
 __global__ void __launch_bounds__(1024 / R, 2) bicgstab_tmem_line_kernel(const SolveParams P) {
   constexpr int NT = 1024 / R, NWARP = NT / 32;
   static_assert(R == 4 || R == 8, "4 or 8 rows per thread");
@@ -200,7 +203,7 @@ __global__ void __launch_bounds__(1024 / R, 2) bicgstab_tmem_line_kernel(const S
   const double *bsys = P.b + sys * n;
 #pragma unroll
   for (int j = 0; j < R; ++j) {
-    d[j] = (a0[j] != 0.0) ? 1.0 / a0[j] : 1.0;
+    d[j] = jacobi_inv(P.precond, a0[j]);
     r[j] = act[j] ? __ldg(bsys + row0 + j) : 0.0;
     x[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + j) : 0.0;
   }
@@ -222,10 +225,16 @@ __global__ void __launch_bounds__(1024 / R, 2) bicgstab_tmem_line_kernel(const S
   tmem_wait_st();
 
   LineComm<NX, NT, R> comm(sg, sred, act);
-  bicgstab_core<R, NT, false, 3>(P, sys, x, r, d, act, r, comm,
-                                 [&](const double(&own)[R], double(&y)[R]) {
-                                   line_spmv<NX, NT, R, G>(tlane, comm.gq, a0, own, y);
-                                 });
+  auto spmv = [&](const double(&own)[R], double(&y)[R]) {
+    line_spmv<NX, NT, R, G>(tlane, comm.gq, a0, own, y);
+  };
+  if constexpr (SOLVER == SOLVER_GMRES) {
+    double *sV = sred + 16 * NWARP + 2;
+    gmres_core<R, NT, kMaxRestart>(P, sys, x, r, d, act, sV, sV + kMaxRestart * R * NT, comm,
+                                   spmv);
+  } else {
+    bicgstab_core<R, NT, false, 3>(P, sys, x, r, d, act, r, comm, spmv);
+  }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 0)

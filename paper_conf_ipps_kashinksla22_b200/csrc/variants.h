@@ -38,6 +38,7 @@ struct TVariant {
 // TMEM + line-tiled 9-point stencil (PLACE_TMEM, kernel_mode 4), k_line.cu
 struct LVariant {
   int nx, r, g;  // grid width, rows per thread (CTA = 1024 / r threads), TMEM load group
+  int solver;    // SOLVER_BICGSTAB or SOLVER_GMRES
   int smem_bytes;  // dynamic SMEM of one CTA (gather planes + scratch + TMEM slot)
   solve_fn fn;
 };

@@ -23,10 +23,12 @@ def to_dev(a, dtype=torch.float64):
 
 
 def gpu_solve(row_ptr, col_idx, csr_values, b, x0=None, fmt="ell", placement="auto", tol=1e-10,
-              maxiter=1000, stop="rel_b", trc=True, block_threads=0):
+              maxiter=1000, stop="rel_b", trc=True, block_threads=0, solver="bicgstab",
+              precond="jacobi", restart=7):
     batch = csr_values.shape[0]
     S = Solver(row_ptr, col_idx, batch, format=fmt, placement=placement, stop=stop,
-               true_residual_check=trc, block_threads=block_threads)
+               true_residual_check=trc, block_threads=block_threads, solver=solver,
+               precond=precond, restart=restart)
     vals = (S.ell_values(csr_values) if S.format == "ell"
             else csr_values)
     x, it, res, st = S.run(to_dev(vals), to_dev(b), None if x0 is None else to_dev(x0), tol=tol,
