@@ -236,6 +236,29 @@ int bsolve_ell_map(bsolve_handle h, int32_t *cols, int32_t *src);
 int bsolve_ell_layout(int n, const int32_t *row_ptr, const int32_t *col_idx, int32_t *width,
                       int32_t *cols, int32_t *src);
 
+/* Batched banded LU with partial pivoting and solve -- the GPU analogue of
+ * LAPACK dgbsv, the paper's CPU solver for these systems (PAPER.md:97-99,
+ * Sec. I; 556-559, Sec. III; 915-925, Sec. V-A).  For
+ * every system i: P_i A_i = L_i U_i by dgbtf2's column order (pivot = FIRST
+ * row of largest |a_kj| among rows j..j+kl), then x_i = U_i^-1 L_i^-1 P_i b_i
+ * as in dgbtrs.  kl, ku are the pattern's bandwidths (bsolve_info.kl/ku).
+ *   values  DEVICE, in the handle's format (as bsolve_run).
+ *   b       DEVICE, batch * n doubles (read only).
+ *   x       DEVICE, batch * n doubles (out; must not alias b).  Unspecified
+ *           for a system with info > 0.
+ *   info    DEVICE, batch int32 (out): 0, or j+1 for the first j with an
+ *           exactly zero pivot u_jj (LAPACK convention: singular).
+ *   ipiv    DEVICE, batch * n int32 (out) or NULL: 0-based row interchanged
+ *           with row j at step j (ipiv[j] >= j).
+ *   stream  cudaStream_t or NULL.  Asynchronous: one kernel launch.
+ * The handle owns a workspace of (number of resident CTAs) x n x (2 kb + 2)
+ * doubles, kb = max(kl, ku) rounded up to 4, 8, 16, 33 or 65, allocated on
+ * the first call.  Errors: INVALID (NULL / foreign pointers), UNSUPPORTED
+ * (max(kl, ku) > 65, or a row with more entries than the instance has
+ * loader lanes), NOMEM, CUDA. */
+int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b, double *x,
+                        int32_t *info, int32_t *ipiv, void *stream);
+
 /* Release the handle and its device memory.  NULL-safe; returns BSOLVE_OK. */
 int bsolve_destroy(bsolve_handle h);
 

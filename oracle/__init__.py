@@ -6,7 +6,8 @@ The product package (paper_conf_ipps_kashinksla22_b200) never imports it and
 shares no code with it (see oracle.c for the algorithm and its citations).
 
 Functions mirror oracle.c:
-  spmv, dense_solve, banded_solve, bandwidth, bicgstab (one system, with
+  spmv, dense_solve, banded_solve, banded_factor_solve (with pivots),
+  bandwidth, bicgstab (one system, with
   optional invariant trace), gmres (restarted GMRES(m)),
   batch_bicgstab, batch_krylov, batch_banded (host threads).
 """
@@ -65,6 +66,8 @@ def lib():
             L.oracle_bandwidth.restype = None
             L.oracle_banded_solve.argtypes = [C.c_int, _P, _P, _P, _P, _P]
             L.oracle_banded_solve.restype = C.c_int
+            L.oracle_banded_solve_piv.argtypes = [C.c_int, _P, _P, _P, _P, _P, _P]
+            L.oracle_banded_solve_piv.restype = C.c_int
             L.oracle_bicgstab.argtypes = [C.c_int, _P, _P, _P, _P, _P, C.c_double, C.c_int,
                                           C.c_int, C.c_int, _P, C.POINTER(Result), _P]
             L.oracle_bicgstab.restype = C.c_int
@@ -133,6 +136,21 @@ def banded_solve(row_ptr, col_idx, val, b):
     if info:
         raise np.linalg.LinAlgError(f"banded LU: zero pivot / error {info}")
     return x
+
+
+def banded_factor_solve(row_ptr, col_idx, val, b):
+    """dgbtf2 + dgbtrs on one system without raising: (x, info, ipiv).
+    info = 0 or j+1 for the first zero pivot (x is then not written: NaN);
+    ipiv[j] = 0-based row interchanged with row j."""
+    rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(b)
+    n = rp.size - 1
+    x = np.full(n, np.nan)
+    piv = np.empty(n, np.int32)
+    info = lib().oracle_banded_solve_piv(n, _ptr(rp), _ptr(ci), _ptr(v), _ptr(bb), _ptr(x),
+                                         _ptr(piv))
+    if info < 0:
+        raise MemoryError("oracle_banded_solve_piv")
+    return x, int(info), piv
 
 
 def bicgstab(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, stop=STOP_REL_B,

@@ -78,6 +78,7 @@ def lib():
             L.bsolve_csr_to_ell.argtypes = [_P, _P, _P, C.c_int, _P]
             L.bsolve_query.argtypes = [_P, C.POINTER(Info)]
             L.bsolve_ell_map.argtypes = [_P, _P, _P]
+            L.bsolve_banded_solve.argtypes = [_P, _P, _P, _P, _P, _P, _P]
             L.bsolve_ell_layout.argtypes = [C.c_int, _P, _P, C.POINTER(C.c_int32), _P, _P]
             L.bsolve_destroy.argtypes = [_P]
             L.bsolve_last_error.argtypes = []
@@ -86,7 +87,7 @@ def lib():
                                                       C.POINTER(C.c_double)]
             for f in ("bsolve_create", "bsolve_run", "bsolve_run_host", "bsolve_spmv",
                       "bsolve_csr_to_ell", "bsolve_query", "bsolve_ell_map", "bsolve_destroy",
-                      "bsolve_ell_layout",
+                      "bsolve_ell_layout", "bsolve_banded_solve",
                       "bsolve_probe_smem_bandwidth"):
                 getattr(L, f).restype = C.c_int
             _lib = L
@@ -244,6 +245,24 @@ class Solver:
         check(lib().bsolve_spmv(self._h, values.data_ptr(), x.data_ptr(), y.data_ptr(), int(batch),
                                 _stream_ptr(stream)))
         return y
+
+    def banded_solve(self, values, b, out=None, ipiv: bool = False, stream=None):
+        """Batched banded LU with partial pivoting + solve (dgbsv analogue,
+        SURVEY.md 8(f) f4): returns (x, info) or (x, info, ipiv)."""
+        import torch
+        self._dev_check(values, "values", (self.batch, self.values_per_system), torch.float64)
+        self._dev_check(b, "b", (self.batch, self.n), torch.float64)
+        dev = torch.device("cuda", self.device)
+        if out is None:
+            x = torch.empty((self.batch, self.n), dtype=torch.float64, device=dev)
+            info = torch.empty(self.batch, dtype=torch.int32, device=dev)
+        else:
+            x, info = out
+        piv = torch.empty((self.batch, self.n), dtype=torch.int32, device=dev) if ipiv else None
+        check(lib().bsolve_banded_solve(self._h, values.data_ptr(), b.data_ptr(), x.data_ptr(),
+                                        info.data_ptr(), None if piv is None else piv.data_ptr(),
+                                        _stream_ptr(stream)))
+        return (x, info, piv) if ipiv else (x, info)
 
     def csr_to_ell(self, csr_values, out=None, stream=None):
         import torch

@@ -22,6 +22,7 @@
 #include <vector>
 
 #include "../../include/bsolve.h"
+#include "banded.cuh"
 #include "kernels.cuh"
 #include "variants.h"
 
@@ -112,6 +113,10 @@ struct bsolve_plan {
          *h_res[kSlots] = {};
   int32_t *h_it[kSlots] = {};
   int8_t *h_st[kSlots] = {};
+  // banded direct solver (bsolve_banded_solve, lazily set up)
+  int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
+  double *d_bws = nullptr;    // per-CTA U + y workspace
+  size_t bws_bytes = 0;
 };
 
 extern "C" void bsolve_default_options(bsolve_options *o) {
@@ -138,6 +143,8 @@ static void free_plan(bsolve_plan *h) {
   cudaFree(h->d_diag);
   cudaFree(h->d_src);
   cudaFree(h->d_ctr);
+  cudaFree(h->d_bnd);
+  cudaFree(h->d_bws);
   for (int s = 0; s < bsolve_plan::kSlots; ++s) {
     if (h->hs[s]) cudaStreamDestroy(h->hs[s]);
     cudaFree(h->h_val[s]);
@@ -1011,6 +1018,96 @@ extern "C" int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, doub
   if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "csr_to_ell launch: %s", cudaGetErrorString(e));
   return BSOLVE_OK;
+}
+
+// ---------------------------------------------- banded direct solver (f4) --
+extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b,
+                                   double *x, int32_t *info, int32_t *ipiv, void *stream) {
+  g_err.clear();
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (h->batch == 0) return BSOLVE_OK;
+  if (!values || !b || !x || !info)
+    return fail(BSOLVE_ERR_INVALID, "values, b, x and info must be non-NULL");
+  int rc;
+  const void *ptrs[] = {values, b, x, info, ipiv};
+  const char *names[] = {"values", "b", "x", "info", "ipiv"};
+  for (int i = 0; i < 5; ++i)
+    if ((rc = check_device_ptr(h, ptrs[i], names[i]))) return rc;
+  const int kb = std::max(h->kl, h->ku);
+  int cnt = 0;
+  const BVariant *tab = variants_banded(&cnt), *bv = nullptr;
+  for (int i = 0; i < cnt; ++i)  // smallest padded bandwidth that covers the pattern
+    if (tab[i].kb >= kb && tab[i].max_entries > h->W && (!bv || tab[i].kb < bv->kb)) bv = &tab[i];
+  if (!bv)
+    return fail(BSOLVE_ERR_UNSUPPORTED,
+                "banded solver: bandwidth kl = %d, ku = %d exceeds the largest instance", h->kl,
+                h->ku);
+  if ((long long)h->sys_stride >= (1LL << 23))
+    return fail(BSOLVE_ERR_UNSUPPORTED, "banded solver: %lld values per system exceed 2^23",
+                h->sys_stride);
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  auto done = [&](int code) {
+    if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+    return code;
+  };
+  const int n = h->n, W = h->W;
+  if (!h->d_bnd) {
+    // entry k of row r: its value index inside one system's block (CSR order
+    // or ELL slot k) and its band offset col - row; padding slots -> -1
+    std::vector<int32_t> bnd((size_t)W * n, -1);
+    for (int k = 0; k < W; ++k)
+      for (int r = 0; r < n; ++r) {
+        const int e = h->h_csr2ell[(size_t)k * n + r];
+        if (e < 0) continue;
+        const long long vidx = h->fmt == FMT_ELL ? (long long)k * n + r : e;
+        const int off = h->h_ell_col[(size_t)k * n + r] - r;
+        bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (off + 128));
+      }
+    if (cudaMalloc(&h->d_bnd, sizeof(int32_t) * bnd.size()) != cudaSuccess)
+      return done(fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed"));
+    if (cudaMemcpy(h->d_bnd, bnd.data(), sizeof(int32_t) * bnd.size(), cudaMemcpyHostToDevice) !=
+        cudaSuccess)
+      return done(fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed"));
+  }
+  if (bv->smem_bytes > 48 * 1024)
+    CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  bv->smem_bytes));
+  int occ = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)bv->fn, bv->nt,
+                                                         bv->smem_bytes));
+  if (occ < 1) return done(fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident"));
+  const int grid = (int)std::min<long long>((long long)occ * h->num_sms, h->batch);
+  const int Wb = 2 * bv->kb + 1;
+  const size_t need = sizeof(double) * (size_t)grid * ((size_t)n * Wb + n);
+  if (h->bws_bytes < need) {
+    cudaFree(h->d_bws);
+    h->d_bws = nullptr;
+    h->bws_bytes = 0;
+    if (cudaMalloc(&h->d_bws, need) != cudaSuccess) {
+      cudaGetLastError();
+      return done(fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need));
+    }
+    h->bws_bytes = need;
+  }
+  bband::BandParams P;
+  P.values = values;
+  P.b = b;
+  P.bnd = h->d_bnd;
+  P.x = x;
+  P.info = info;
+  P.ipiv = ipiv;
+  P.ws = h->d_bws;
+  P.sys_stride = h->sys_stride;
+  P.E = W;
+  P.n = n;
+  P.batch = h->batch;
+  bv->fn<<<grid, bv->nt, bv->smem_bytes, (cudaStream_t)stream>>>(P);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess)
+    return done(fail(BSOLVE_ERR_CUDA, "banded launch: %s", cudaGetErrorString(e)));
+  return done(BSOLVE_OK);
 }
 
 extern "C" int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz) {

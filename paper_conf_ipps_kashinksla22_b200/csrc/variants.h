@@ -8,8 +8,12 @@
 namespace bsolve {
 struct SolveParams;
 }
+namespace bband {
+struct BandParams;
+}
 
 typedef void (*solve_fn)(const bsolve::SolveParams);
+typedef void (*banded_fn)(const bband::BandParams);
 typedef void (*persist_fn)(const bsolve::SolveParams, unsigned long long *);
 
 // per-system-CTA kernels (bicgstab_kernel), k_generic.cu
@@ -43,6 +47,15 @@ struct LVariant {
   solve_fn fn;
 };
 
+// batched banded LU (dgbsv analogue), k_banded.cu
+struct BVariant {
+  int kb;          // padded bandwidth: serves patterns with kl, ku <= kb
+  int nt;          // threads per CTA
+  int max_entries; // loader lanes: rows with at most this many entries - 1
+  int smem_bytes;  // dynamic SMEM (row ring)
+  banded_fn fn;
+};
+
 const Variant *variants_generic(int *count);
 const PVariant *variants_persist(int *count);
 const CVariant *variants_cluster(int *count);
@@ -50,3 +63,4 @@ const CVariant *variants_cluster_tmem(int *count);
 const TVariant *variants_tmem(int *count);
 persist_fn variant_tmem_persist();
 const LVariant *variants_line(int *count);
+const BVariant *variants_banded(int *count);

@@ -1,0 +1,163 @@
+"""GPU parity of the batched banded LU solver (bsolve_banded_solve, the dgbsv
+analogue of SURVEY.md 8(f) f4) against the
+oracle's dgbtf2 + dgbtrs (oracle/oracle.c oracle_banded_solve_piv).
+
+Bar (f4 rows):
+  * ipiv (integer): bit-exact.  Both sides pick the pivot in fp64 from values
+    that agree to rounding; the test inputs have no near-ties.
+  * info (integer): equal.
+  * x: ||x_gpu - x_oracle|| / ||x_oracle|| <= FWD (kernel: fused multiply-add
+    and the multiplier folded as a_kj * (u_jc / u_jj), R25), with
+    FWD = 1e-12 on the well-conditioned XGC systems and a condition-scaled
+    bound on the pivoting-heavy random ones.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import xgcgen as X
+from paper_conf_ipps_kashinksla22_b200 import Solver
+
+pytestmark = pytest.mark.gpu
+
+
+def to_dev(a, dtype=torch.float64):
+    return torch.as_tensor(np.ascontiguousarray(a)).to(device="cuda", dtype=dtype)
+
+
+def gpu_banded(row_ptr, col_idx, csr_values, b, fmt="ell"):
+    batch = csr_values.shape[0]
+    S = Solver(row_ptr, col_idx, batch, format=fmt)
+    vals = S.ell_values(csr_values) if S.format == "ell" else csr_values
+    x, info, piv = S.banded_solve(to_dev(vals), to_dev(b), ipiv=True)
+    torch.cuda.synchronize()
+    out = x.cpu().numpy(), info.cpu().numpy(), piv.cpu().numpy()
+    S.close()
+    return out
+
+
+def oracle_banded(row_ptr, col_idx, csr_values, b):
+    xs, infos, pivs = [], [], []
+    for k in range(csr_values.shape[0]):
+        x, info, piv = O.banded_factor_solve(row_ptr, col_idx, csr_values[k], b[k])
+        xs.append(x)
+        infos.append(info)
+        pivs.append(piv)
+    return np.array(xs), np.array(infos), np.array(pivs)
+
+
+def check(row_ptr, col_idx, vals, b, fmt="ell", fwd=1e-12):
+    xg, ig, pg = gpu_banded(row_ptr, col_idx, vals, b, fmt)
+    xo, io, po = oracle_banded(row_ptr, col_idx, vals, b)
+    assert np.array_equal(ig, io), (ig, io)
+    assert np.array_equal(pg, po), np.argwhere(pg != po)[:5]
+    ok = io == 0
+    rel = np.linalg.norm(xg[ok] - xo[ok], axis=1) / np.linalg.norm(xo[ok], axis=1)
+    assert rel.max(initial=0.0) <= fwd, rel.max()
+    return xg, pg
+
+
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_xgc_pair(fmt):
+    """configs[0]: the ion + electron pair at 32 x 31 (kl = ku = 33, KB = 33)."""
+    B = X.make_batch(0, 2)
+    p = B.pattern
+    xg, pg = check(p.row_ptr, p.col_idx, B.values, B.b, fmt)
+    # the direct solution also satisfies the 1e-10 relative residual bar
+    for k in range(2):
+        r = B.b[k] - O.spmv(p.row_ptr, p.col_idx, B.values[k], xg[k])
+        assert np.linalg.norm(r) / np.linalg.norm(B.b[k]) <= 1e-13
+
+
+def test_xgc_batch_many_waves():
+    """configs[1] size (1280 systems): more systems than resident CTAs, so
+    every CTA of the persistent grid solves several (workspace reuse)."""
+    B = X.make_batch(0, 1280)
+    p = B.pattern
+    check(p.row_ptr, p.col_idx, B.values, B.b)
+
+
+@pytest.mark.parametrize("nx,ny", [(3, 3), (5, 4), (7, 5), (12, 9), (17, 6), (32, 31)])
+@pytest.mark.parametrize("fmt", ["ell", "csr"])
+def test_pivoting_random(nx, ny, fmt):
+    """Random 9-point values with tiny diagonals: most steps interchange rows,
+    exercising the swap path of every instance (KB = 4, 8, 16, 33) and n not a
+    multiple of the unroll (ragged last block)."""
+    pat = X.stencil_pattern(nx, ny)
+    rng = np.random.default_rng(nx * 1000 + ny)
+    batch = 40
+    v = rng.standard_normal((batch, pat.nnz))
+    diag = pat.col_idx == np.repeat(np.arange(pat.n), np.diff(pat.row_ptr))
+    v[:, diag] *= 1e-2
+    b = rng.standard_normal((batch, pat.n))
+    xo, io, po = oracle_banded(pat.row_ptr, pat.col_idx, v, b)
+    assert np.all(io == 0)
+    assert np.mean(po != np.arange(pat.n)) > 0.2
+    # condition-scaled bound: kappa_1 estimate of each system
+    kap = max(np.linalg.cond(X_dense(pat, v[k]), 1) for k in range(min(batch, 8)))
+    check(pat.row_ptr, pat.col_idx, v, b, fmt, fwd=max(1e-12, 1e-15 * kap * pat.n))
+
+
+def X_dense(pat, v):
+    A = np.zeros((pat.n, pat.n))
+    for i in range(pat.n):
+        for e in range(pat.row_ptr[i], pat.row_ptr[i + 1]):
+            A[i, pat.col_idx[e]] = v[e]
+    return A
+
+
+def test_tridiagonal_and_tiny():
+    """kl = ku = 1 (KB = 4 instance) at n = 1, 2, 3, 50; diagonal n = 1."""
+    for n in (1, 2, 3, 50):
+        rp = [0]
+        ci = []
+        for i in range(n):
+            for j in (i - 1, i, i + 1):
+                if 0 <= j < n:
+                    ci.append(j)
+            rp.append(len(ci))
+        rp, ci = np.array(rp, np.int32), np.array(ci, np.int32)
+        rng = np.random.default_rng(n)
+        v = rng.standard_normal((5, ci.size))
+        b = rng.standard_normal((5, n))
+        check(rp, ci, v, b, fwd=1e-10)
+
+
+def test_singular_info():
+    """A zero column j gives info = j+1 (LAPACK), same as the oracle; the
+    other systems of the batch are unaffected."""
+    pat = X.stencil_pattern(32, 31)
+    v = X.random_dd_values(pat.row_ptr, pat.col_idx, 3, seed=11).copy()
+    v[1, pat.col_idx == 500] = 0.0
+    b = X.random_rhs(3, pat.n, seed=2)
+    xg, ig, pg = gpu_banded(pat.row_ptr, pat.col_idx, v, b)
+    xo, io, po = oracle_banded(pat.row_ptr, pat.col_idx, v, b)
+    assert list(ig) == [0, 501, 0] and np.array_equal(ig, io)
+    assert np.array_equal(pg, po)
+    for k in (0, 2):
+        assert np.linalg.norm(xg[k] - xo[k]) / np.linalg.norm(xo[k]) <= 1e-12
+
+
+def test_large_grid_kb65():
+    """configs[4] grid 64 x 63 (n = 4032, kl = ku = 65: KB = 65 instance)."""
+    B = X.make_batch(0, 6, nx=64, ny=63)
+    p = B.pattern
+    check(p.row_ptr, p.col_idx, B.values, B.b)
+
+
+def test_bandwidth_too_large_is_unsupported():
+    """A pattern with kl > 65 has no instance: UNSUPPORTED, nothing launched."""
+    from paper_conf_ipps_kashinksla22_b200.bsolve import BsolveError, ERR_UNSUPPORTED
+    n = 100
+    rp, ci = [0], []
+    for i in range(n):
+        cols = sorted({i, (i + 70) % n})
+        ci += cols
+        rp.append(len(ci))
+    S = Solver(np.array(rp, np.int32), np.array(ci, np.int32), 2, format="csr")
+    v = torch.ones((2, len(ci)), dtype=torch.float64, device="cuda")
+    b = torch.ones((2, n), dtype=torch.float64, device="cuda")
+    with pytest.raises(BsolveError) as e:
+        S.banded_solve(v, b)
+    assert e.value.code == ERR_UNSUPPORTED

@@ -102,6 +102,47 @@ def test_banded_vs_lapack_gbsv_full_size():
         assert np.linalg.norm(x - ref) / np.linalg.norm(ref) <= 1e-12
 
 
+@pytest.mark.parametrize("nx,ny,scale", [(5, 4, 1e-3), (8, 6, 1e-2), (32, 31, 1e-3)])
+def test_banded_pivots_vs_lapack_dgbtrf(nx, ny, scale):
+    """P1 (f4 pivots): the row interchanges of the oracle's dgbtf2 equal those
+    of LAPACK dgbtrf (scipy.linalg.lapack) on matrices with tiny diagonals,
+    where most steps swap; x matches LAPACK's dgbtrs.  ipiv is what the GPU
+    banded solver is compared with bit for bit (PAPER.md:97-99 dgbsv)."""
+    from scipy.linalg import lapack
+    pat = X.stencil_pattern(nx, ny)
+    kl, ku = O.bandwidth(pat.row_ptr, pat.col_idx)
+    rng = np.random.default_rng(nx * 100 + ny)
+    for _ in range(3):
+        v = rng.standard_normal(pat.nnz)
+        diag = pat.col_idx == np.repeat(np.arange(pat.n), np.diff(pat.row_ptr))
+        v[diag] *= scale
+        b = rng.standard_normal(pat.n)
+        A = dense_of(pat.row_ptr, pat.col_idx, v, pat.n)
+        ab = np.zeros((2 * kl + ku + 1, pat.n))
+        for j in range(pat.n):
+            for i in range(max(0, j - ku), min(pat.n, j + kl + 1)):
+                ab[kl + ku + i - j, j] = A[i, j]
+        lu, piv, info = lapack.dgbtrf(ab, kl, ku)
+        assert info == 0
+        xr, info2 = lapack.dgbtrs(lu, kl, ku, b, piv)
+        x, oinfo, opiv = O.banded_factor_solve(pat.row_ptr, pat.col_idx, v, b)
+        assert oinfo == 0
+        assert np.array_equal(opiv, piv), np.nonzero(opiv != piv)
+        assert np.count_nonzero(opiv != np.arange(pat.n)) > pat.n // 4  # pivoting happened
+        np.testing.assert_allclose(x, xr, rtol=1e-9, atol=1e-9 * np.abs(xr).max())
+
+
+def test_banded_zero_pivot_info():
+    """LAPACK convention: info = j+1 for the first exactly-zero pivot column
+    (a zero column j makes every candidate of step j zero)."""
+    pat = X.stencil_pattern(4, 4)
+    v = X.random_dd_values(pat.row_ptr, pat.col_idx, 1, seed=3)[0].copy()
+    v[pat.col_idx == 6] = 0.0               # column 6 of A is zero
+    b = np.ones(pat.n)
+    _, info, piv = O.banded_factor_solve(pat.row_ptr, pat.col_idx, v, b)
+    assert info == 7 and piv[6] == 6
+
+
 def test_spmv_vs_dense():
     pat = X.stencil_pattern(7, 5)
     v = X.random_dd_values(pat.row_ptr, pat.col_idx, 1, seed=4)[0]
