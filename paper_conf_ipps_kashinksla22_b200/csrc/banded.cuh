@@ -14,12 +14,15 @@
 // B200 design:
 //  * the active window of the band -- rows j..j+KL, columns j..j+KL+KU -- is
 //    held in REGISTERS: thread t owns every column c = t (mod W) in turn, one
-//    double per window row; window row r sits in register slot r mod (KL+1).
-//    The step loop is unrolled by KL+1, so every slot index is static (no
-//    local memory) while the window slides one row/column per step.
+//    double per window row, v[k] = row j+k.  The elimination update writes
+//    row j+k into v[k-1], so the window slides by one row per step through
+//    the FMA destinations: every register index is static (no local memory)
+//    and the step loop stays rolled (small code: the instruction cache holds
+//    it, which an unrolled-by-(KL+1) loop of ~50k instructions did not).
 //  * thread W owns the right-hand side as one more column.
-//  * per step the pivot column's thread finds the pivot (tree argmax, first
-//    index on ties), publishes the pivot row index, 1/pivot and the column to
+//  * per step the pivot column's thread finds the pivot (first index of the
+//    largest |a_kj|: a cheap "is the diagonal the maximum" test, then a tree
+//    argmax only when it is not), publishes the pivot row index, 1/pivot and the column to
 //    SMEM (double-buffered, ONE __syncthreads per step); every thread then
 //    swaps (warp-uniform branch, rare) and applies
 //        a_kc -= a_kj * (u_jc / u_jj)                            k = 1..KL
@@ -28,9 +31,10 @@
 //  * rows enter the window KL+1 steps before they are pivot candidates: idle
 //    "loader" lanes cp.async the next rows' pattern entries (values in the
 //    handle's CSR or ELL layout, b) into a zeroed SMEM row ring D steps ahead.
-//  * U (row j: 1/u_jj then u_j,j+1..u_j,j+W-1) and y go to a per-CTA global
-//    workspace (HBM/L2) and are streamed back for the back substitution,
-//    which keeps one accumulator per thread for the rows j-W+1..j.
+//  * U (row j: 1/u_jj, u_j,j+1 .. u_j,j+W-1; coalesced stores) and y go to a
+//    per-CTA global workspace (HBM/L2).  The back substitution runs in ONE
+//    warp: lane l keeps the accumulators of the rows = l (mod 32) still in
+//    the band and x_j travels by shuffle (no CTA barrier per step).
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -40,11 +44,11 @@ namespace bband {
 struct BandParams {
   const double *values;   // [batch][sys_stride] in the handle's CSR or ELL layout
   const double *b;        // [batch][n]
-  const int32_t *bnd;     // [E][n]: (value index << 8) | (col - row + 128), -1 = none
+  const int32_t *bnd;     // [E][n]: (value index << 8) | (col mod W), -1 = none
   double *x;              // [batch][n] out
   int32_t *info;          // [batch] out: 0, or j+1 if u_jj == 0 (LAPACK convention)
   int32_t *ipiv;          // [batch][n] out or nullptr: row swapped with row j (0-based)
-  double *ws;             // per CTA: U [n][W] then y [n]
+  double *ws;             // per CTA: U [n][W] (row j: 1/u_jj, u_j,j+1 ..) then y [n]
   long long sys_stride;
   int E, n, batch;
 };
@@ -66,7 +70,8 @@ template <int KL, int KU>
 struct Geo {
   static constexpr int R = KL + 1;            // window rows = register slots per column
   static constexpr int W = KL + KU + 1;       // window columns (U row length)
-  static constexpr int NT = ((W + 2 + 31) / 32) * 32;  // + RHS thread + >= 1 loader
+  static constexpr int NTF = ((W + 2 + 31) / 32) * 32;  // factor warps: + RHS thread + >= 1 loader
+  static constexpr int NT = NTF + 32;                    // + the back-substitution warp
   static constexpr int D = R - 2 < 4 ? R - 2 : 4;      // row prefetch distance (steps)
   static constexpr int RB = W + 1;            // row ring stride (doubles)
   static constexpr int smem_bytes = R * RB * 8;
@@ -75,49 +80,169 @@ struct Geo {
 
 // Loader lane e (< E: pattern entry e of the row; == E: b) issues the cp.async
 // that brings row rr into ring slot `slot`: the entry of column c goes to
-// position c mod W, b to position W.  pk = P.bnd[e][rr], loaded a step ahead.
+// position c mod W (precomputed in pk's low byte), b to position W.
+// pk = P.bnd[e][rr], loaded one step ahead.
 template <int KL, int KU>
 __device__ __forceinline__ void load_entry(const BandParams &P, const double *val, const double *bb,
                                            double *ring, int slot, int rr, int e, int pk) {
   using G = Geo<KL, KU>;
   if (rr >= P.n || e > P.E) return;
   double *row = ring + slot * G::RB;
-  if (e == P.E) {
-    cp_async8(row + G::W, bb + rr);
-  } else if (pk >= 0) {
-    const int col = rr + (pk & 255) - 128;
-    cp_async8(row + col % G::W, val + (pk >> 8));
-  }
+  if (e == P.E) cp_async8(row + G::W, bb + rr);
+  else if (pk >= 0) cp_async8(row + (pk & 255), val + (pk >> 8));
 }
 __device__ __forceinline__ int load_pk(const BandParams &P, int rr, int e) {
   return (rr < P.n && e < P.E) ? __ldg(P.bnd + (size_t)e * P.n + rr) : -1;
 }
 
+// First index of the largest |a_k|, k = 0..N-1 (dgbtf2's IDAMAX): a tree
+// that keeps the left operand unless the right one is strictly larger.
+__device__ __forceinline__ void bar_factor(int nthreads) {  // named barrier 1: factor warps only
+  asm volatile("bar.sync 1, %0;" ::"r"(nthreads) : "memory");
+}
+__device__ __forceinline__ void mbar_init1(uint64_t *bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(saddr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
+  asm volatile("{\n.reg .b64 st;\nmbarrier.arrive.release.cta.shared::cta.b64 st, [%0];\n}" ::"r"(
+                   saddr(bar))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n.reg .pred p;\nW%=:\n"
+      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra W%=;\n}" ::"r"(saddr(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+template <int N>
+__device__ __forceinline__ int argmax_abs(const double (&a)[N]) {
+  double bv[N];
+  int bi[N];
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    bv[k] = a[k];
+    bi[k] = k;
+  }
+#pragma unroll
+  for (int s = 1; s < N; s *= 2)
+#pragma unroll
+    for (int k = 0; k + s < N; k += 2 * s)
+      if (fabs(bv[k + s]) > fabs(bv[k])) {
+        bv[k] = bv[k + s];
+        bi[k] = bi[k + s];
+      }
+  return bi[0];
+}
+
 template <int KL, int KU, int MINB>
 __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const BandParams P) {
   using G = Geo<KL, KU>;
-  constexpr int R = G::R, W = G::W, NT = G::NT, D = G::D, RB = G::RB;
+  constexpr int R = G::R, W = G::W, NTF = G::NTF, D = G::D, RB = G::RB;
+  constexpr int NA = (W + 31) / 32;  // back substitution: accumulators per lane
   extern __shared__ __align__(16) double ring[];  // [R][RB]
   constexpr int RP = (R + 1) & ~1;
   __shared__ __align__(16) double colbuf[2][RP];  // pivot column rows 1..KL (index k-1)
   __shared__ double s_rp[2];
   __shared__ int s_p[2];
-  __shared__ double s_xb[2];
   __shared__ int s_info;
+  // workspace hand-off factor warps -> back-substitution warp (2 buffers)
+  __shared__ __align__(8) uint64_t full_bar[2], empty_bar[2];
 
   const int t = threadIdx.x;
-  const bool owns = t <= W;        // column thread (t < W) or RHS thread (t == W)
-  const bool loader = t > W;
-  const int lidx = t - W - 1;  // loader lane = pattern entry (needs NT - W - 1 > E)
   const int n = P.n;
-  const int nsteps = ((n + R - 1) / R) * R;
-  double *U = P.ws + (size_t)blockIdx.x * ((size_t)n * W + n);
-  double *Y = U + (size_t)n * W;
+  const size_t ws_sys = (size_t)n * W + n;  // U [n][W] then y [n]
+  double *ws = P.ws + (size_t)blockIdx.x * 2 * ws_sys;
 
-  for (int i = t; i < R * RB; i += NT) ring[i] = 0.0;
+  if (t == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init1(&full_bar[i]);
+      mbar_init1(&empty_bar[i]);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  for (int i = t; i < R * RB; i += G::NT) ring[i] = 0.0;
   __syncthreads();
 
-  for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+  if (t >= NTF) {
+    // ======== back-substitution warp (dgbtrs U part, column order) =========
+    // lane l holds the accumulators of rows r0 - 32m (m < NA), r0 = the
+    // largest row <= j with r0 = l (mod 32).  Step j: the owner lane
+    // (l = j mod 32) forms x_j = y_j * (1/u_jj) and broadcasts it by shuffle;
+    // every other row i in the band gets y_i -= u_ij x_j.  u_ij is read from
+    // the row-major U (L1-cached: each lane walks its rows backwards).
+    const int l = t - NTF;
+    int k = 0;
+    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x, ++k) {
+      const int b = k & 1;
+      mbar_wait(&full_bar[b], (k >> 1) & 1);
+      const double *U = ws + b * ws_sys;
+      const double *Y = U + (size_t)n * W;
+      constexpr int PF = 8;  // U entries are loaded PF steps ahead
+      double a[NA], q[PF][NA];
+      const int r0 = (n - 1) - ((n - 1 - l) & 31);
+#pragma unroll
+      for (int m = 0; m < NA; ++m) a[m] = r0 - 32 * m >= 0 ? Y[r0 - 32 * m] : 0.0;
+      double ynext = r0 - 32 * NA >= 0 ? Y[r0 - 32 * NA] : 0.0;
+      auto uload = [&](int jj, int m) -> double {  // u_{i,jj}, i = the lane's m-th row at step jj
+        const int d = ((jj - l) & 31) + 32 * m;
+        const int i = jj - d;
+        return (jj >= 0 && i >= 0 && d < W) ? U[(size_t)i * W + d] : 0.0;
+      };
+#pragma unroll
+      for (int s = 0; s < PF; ++s)
+#pragma unroll
+        for (int m = 0; m < NA; ++m) q[s][m] = uload(n - 1 - s, m);
+      double *xs = P.x + sys * n;
+#pragma unroll 1
+      for (int jb0 = n - 1; jb0 >= 0; jb0 -= PF) {
+#pragma unroll
+        for (int s = 0; s < PF; ++s) {
+          const int j = jb0 - s;
+          double u[NA];
+#pragma unroll
+          for (int m = 0; m < NA; ++m) {
+            u[m] = q[s][m];
+            q[s][m] = uload(j - PF, m);
+          }
+          if (j >= 0) {  // uniform
+            const bool own = l == (j & 31);
+            const double xo = a[0] * u[0];  // owner: x_j = y_j / u_jj
+            const double x = __shfl_sync(0xffffffffu, xo, j & 31);
+            if (own) {
+              xs[j] = x;
+              u[0] = 0.0;
+            }
+#pragma unroll
+            for (int m = 0; m < NA; ++m) a[m] = fma(-u[m], x, a[m]);
+            if (own) {  // row j is done: the lane takes row j - 32 NA
+#pragma unroll
+              for (int m = 0; m + 1 < NA; ++m) a[m] = a[m + 1];
+              a[NA - 1] = ynext;
+              const int rn = j - 32 * (NA + 1);
+              ynext = rn >= 0 ? Y[rn] : 0.0;
+            }
+          }
+        }
+      }
+      __syncwarp();
+      if (l == 0) mbar_arrive1(&empty_bar[b]);  // buffer b may be overwritten
+    }
+    return;
+  }
+
+  // ======== factor warps: dgbtf2 + the L part of dgbtrs on b ================
+  const bool owns = t <= W;  // column thread (t < W) or RHS thread (t == W)
+  const bool loader = t > W;
+  const int lidx = t - W - 1;  // loader lane = pattern entry (needs NTF - W - 1 > E)
+  int k = 0;
+  for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x, ++k) {
+    const int b = k & 1;
+    if (k >= 2) mbar_wait(&empty_bar[b], ((k >> 1) - 1) & 1);  // back substitution k-2 done
+    double *U = ws + b * ws_sys;
+    double *Y = U + (size_t)n * W;
     const double *val = P.values + sys * P.sys_stride;
     const double *bb = P.b + sys * n;
     if (t == 0) s_info = 0;
@@ -128,14 +253,14 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
       cp_commit();
       cp_wait<0>();
     }
-    __syncthreads();
+    bar_factor(NTF);
     double v[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       v[r] = owns ? ring[r * RB + t] : 0.0;
       if (owns) ring[r * RB + t] = 0.0;
     }
-    __syncthreads();
+    bar_factor(NTF);
     // rows KL+1..KL+D into ring slots 0..D-1, one commit group per row
     int pk = -1;  // loader: pattern entry of the row the next step issues
     if (loader) {
@@ -146,145 +271,88 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
       }
       pk = load_pk(P, KL + 1 + D, lidx);
     }
-    int jm = 0;  // j mod W
-    // ---- factorisation + forward substitution (dgbtf2 / dgbtrs L part) -----
+    int pos = owns ? (t == W ? W : t) : -1;  // column j + pos (RHS: W)
+    int jr = 0;                              // j mod R: ring slot of row j+KL+1
+    double *Urow = U;                        // row j of U
+    // v[k] holds window row j+k of the thread's column; the update writes row
+    // j+k into v[k-1], so the window slides by register renaming
 #pragma unroll 1
-    for (int j0 = 0; j0 < nsteps; j0 += R) {
+    for (int j = 0; j < n; ++j) {
+      const int jb = j & 1;
+      if (pos == 0) {
+        // pivot: IDAMAX over rows j..j+KL.  Fast test first: the diagonal is
+        // the (first) largest iff |a_jj| >= |a_kj| for all k (ties keep k=0)
+        bool diag_max[4] = {true, true, true, true};
 #pragma unroll
-      for (int u = 0; u < R; ++u) {
-        const int j = j0 + u;
-        const int jb = j & 1;
-        int pos = t - jm;
-        if (pos < 0) pos += W;
-        if (t == W) pos = W;
-        if (t < W && pos == 0) {
-          // pivot: first index of max |a_kj|, k = 0..KL (tree keeps the left
-          // operand unless the right one is strictly larger)
-          double bv[R];
-          int bi[R];
+        for (int kk = 1; kk < R; ++kk)
+          diag_max[kk & 3] = diag_max[kk & 3] && (fabs(v[0]) >= fabs(v[kk]));
+        int p = 0;
+        if (!(diag_max[0] && diag_max[1] && diag_max[2] && diag_max[3])) p = argmax_abs<R>(v);
+        double pv = v[0];
+        double2 *cbw = reinterpret_cast<double2 *>(colbuf[jb]);
 #pragma unroll
-          for (int k = 0; k < R; ++k) {
-            bv[k] = v[(u + k) % R];
-            bi[k] = k;
-          }
-#pragma unroll
-          for (int s = 1; s < R; s *= 2)
-#pragma unroll
-            for (int k = 0; k + s < R; k += 2 * s)
-              if (fabs(bv[k + s]) > fabs(bv[k])) {
-                bv[k] = bv[k + s];
-                bi[k] = bi[k + s];
-              }
-          const int p = bi[0];
-          const double pv = bv[0];
-          const double rp = pv != 0.0 ? __drcp_rn(pv) : 0.0;
-#pragma unroll
-          for (int k = 1; k < R; ++k) colbuf[jb][k - 1] = v[(u + k) % R];
-          if (p != 0) colbuf[jb][p - 1] = v[u];
-          s_p[jb] = p;
-          s_rp[jb] = rp;
-          if (j < n) {
-            U[(size_t)j * W] = rp;
-            if (P.ipiv) P.ipiv[sys * n + j] = j + p;
-            if (pv == 0.0 && s_info == 0) s_info = j + 1;
-          }
-#pragma unroll
-          for (int k = 0; k < R; ++k) v[k] = 0.0;  // the thread takes column j + W next
+        for (int kk = 1; kk < R; kk += 2)
+          cbw[(kk - 1) / 2] = make_double2(v[kk], kk + 1 < R ? v[kk + 1] : 0.0);
+        if (p != 0) {
+          pv = colbuf[jb][p - 1];
+          colbuf[jb][p - 1] = v[0];  // row swap in the published column
         }
-        if (loader) {
-          load_entry<KL, KU>(P, val, bb, ring, (u + KL + 1 + D) % R, j + KL + 1 + D, lidx, pk);
-          pk = load_pk(P, j + KL + 2 + D, lidx);
-          cp_commit();
-          cp_wait<D>();
-        }
-        __syncthreads();
-        if (owns) {
-          const int p = s_p[jb];
-          const double rp = s_rp[jb];
-          if (p != 0) {  // row swap j <-> j+p (uniform branch)
-            const double a = v[u];
-            double bsel = a;
-#pragma unroll
-            for (int k = 1; k < R; ++k) bsel = (p == k) ? v[(u + k) % R] : bsel;
-#pragma unroll
-            for (int k = 1; k < R; ++k) v[(u + k) % R] = (p == k) ? a : v[(u + k) % R];
-            v[u] = bsel;
-          }
-          const double uc = v[u];
-          if (j < n) {
-            if (pos == W) Y[j] = uc;
-            else if (pos != 0) U[(size_t)j * W + pos] = uc;
-          }
-          const double w = uc * rp;
-          const double2 *cb = reinterpret_cast<const double2 *>(colbuf[jb]);
-#pragma unroll
-          for (int k = 1; k < R; k += 2) {
-            const double2 m = cb[(k - 1) / 2];
-            v[(u + k) % R] = fma(-m.x, w, v[(u + k) % R]);
-            if (k + 1 < R) v[(u + k + 1) % R] = fma(-m.y, w, v[(u + k + 1) % R]);
-          }
-          // row j leaves; row j+KL+1 enters slot u
-          v[u] = ring[u * RB + t];
-          ring[u * RB + t] = 0.0;
-        }
-        jm = (jm + 1 == W) ? 0 : jm + 1;
+        const double rp = pv != 0.0 ? __drcp_rn(pv) : 0.0;
+        s_p[jb] = p;
+        s_rp[jb] = rp;
+        Urow[0] = rp;
+        if (P.ipiv) P.ipiv[sys * n + j] = j + p;
+        if (pv == 0.0 && s_info == 0) s_info = j + 1;
       }
+      if (loader) {
+        int slot = jr + D;
+        if (slot >= R) slot -= R;
+        load_entry<KL, KU>(P, val, bb, ring, slot, j + KL + 1 + D, lidx, pk);
+        pk = load_pk(P, j + KL + 2 + D, lidx);
+        cp_commit();
+        cp_wait<D>();
+      }
+      bar_factor(NTF);
+      if (owns) {
+        const int p = s_p[jb];
+        const double rp = s_rp[jb];
+        if (p != 0) {  // row swap j <-> j+p (uniform branch)
+          const double a = v[0];
+          double bsel = a;
+#pragma unroll
+          for (int kk = 1; kk < R; ++kk) bsel = (p == kk) ? v[kk] : bsel;
+#pragma unroll
+          for (int kk = 1; kk < R; ++kk) v[kk] = (p == kk) ? a : v[kk];
+          v[0] = bsel;
+        }
+        const double uc = v[0];
+        if (pos == W) Y[j] = uc;
+        else if (pos != 0 && pos < n - j) Urow[pos] = uc;  // u_jc, c = j + pos
+        // the pivot thread's column equals the published one, so w = 1 turns
+        // its registers into exact zeros: it takes column j + W next
+        const double w = pos == 0 ? 1.0 : uc * rp;
+        const double2 *cb = reinterpret_cast<const double2 *>(colbuf[jb]);
+#pragma unroll
+        for (int kk = 1; kk < R; kk += 2) {
+          const double2 m = cb[(kk - 1) / 2];
+          v[kk - 1] = fma(-m.x, w, v[kk]);
+          if (kk + 1 < R) v[kk] = fma(-m.y, w, v[kk + 1]);
+        }
+        // row j leaves; row j+KL+1 (ring slot j mod R) enters as window row KL
+        v[KL] = ring[jr * RB + t];
+        ring[jr * RB + t] = 0.0;
+        if (t < W) pos = pos == 0 ? W - 1 : pos - 1;
+      }
+      jr = (jr + 1 == R) ? 0 : jr + 1;
+      Urow += W;
     }
     if (loader) cp_wait<0>();
-    __syncthreads();  // U, y (global) and s_info visible to the whole CTA
-    // ---- back substitution (dgbtrs U part, column order) --------------------
-    // thread t < W holds the accumulator of row i = the largest i <= j with
-    // i = t (mod W); at step j its U entry is U[i][j - i] (U[j][0] = 1/u_jj).
-    {
-      const bool act = t < W;
-      int d = (n - 1 - t) % W;  // j - i at j = n-1 (n-1-t may be < 0)
-      if (d < 0) d += W;
-      int i = act ? n - 1 - d : -1;
-      double acc = i >= 0 ? Y[i] : 0.0;
-      double ynext = i - W >= 0 ? Y[i - W] : 0.0;
-      // software pipeline: the U entries of the next PF steps are loaded ahead
-      constexpr int PF = 8;
-      double q[PF];
-      int dq = d, iq = i;
-#pragma unroll
-      for (int s = 0; s < PF; ++s) {
-        const int jj = n - 1 - s;
-        q[s] = (iq >= 0 && jj >= 0) ? U[(size_t)iq * W + (jj - iq)] : 0.0;
-        if (dq == 0) { dq = W - 1; iq -= W; } else { --dq; }
-      }
-#pragma unroll 1
-      for (int jb0 = n - 1; jb0 >= 0; jb0 -= PF) {
-#pragma unroll
-        for (int s = 0; s < PF; ++s) {
-          const int j = jb0 - s;
-          const double uij = q[s];
-          {  // refill: step j - PF
-            const int jj = j - PF;
-            q[s] = (iq >= 0 && jj >= 0) ? U[(size_t)iq * W + (jj - iq)] : 0.0;
-            if (dq == 0) { dq = W - 1; iq -= W; } else { --dq; }
-          }
-          if (act && j >= 0 && d == 0) {
-            const double xj = acc * uij;  // x_j = y_j / u_jj
-            P.x[sys * n + j] = xj;
-            s_xb[j & 1] = xj;
-          }
-          __syncthreads();
-          if (act && j >= 0) {
-            if (d == 0) {
-              i -= W;
-              d = W - 1;
-              acc = ynext;
-              ynext = i - W >= 0 ? Y[i - W] : 0.0;
-            } else {
-              if (i >= 0) acc = fma(-uij, s_xb[j & 1], acc);  // y_i -= u_ij x_j
-              --d;
-            }
-          }
-        }
-      }
+    bar_factor(NTF);  // every U / y store of this system issued; s_info final
+    if (t == 0) {
+      P.info[sys] = s_info;
+      __threadfence_block();
+      mbar_arrive1(&full_bar[b]);  // release: U, y of buffer b are complete
     }
-    if (t == 0) P.info[sys] = s_info;
-    __syncthreads();
   }
 }
 

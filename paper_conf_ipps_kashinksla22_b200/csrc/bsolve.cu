@@ -115,6 +115,7 @@ struct bsolve_plan {
   int8_t *h_st[kSlots] = {};
   // banded direct solver (bsolve_banded_solve, lazily set up)
   int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
+  int bnd_w = 0;              // window width the table's ring positions use
   double *d_bws = nullptr;    // per-CTA U + y workspace
   size_t bws_bytes = 0;
 };
@@ -1053,23 +1054,25 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
     return code;
   };
   const int n = h->n, W = h->W;
-  if (!h->d_bnd) {
+  const int Wb = 2 * bv->kb + 1;  // the instance's window width
+  if (!h->d_bnd || h->bnd_w != Wb) {
     // entry k of row r: its value index inside one system's block (CSR order
-    // or ELL slot k) and its band offset col - row; padding slots -> -1
+    // or ELL slot k) and the ring position (column mod Wb); padding -> -1
     std::vector<int32_t> bnd((size_t)W * n, -1);
     for (int k = 0; k < W; ++k)
       for (int r = 0; r < n; ++r) {
         const int e = h->h_csr2ell[(size_t)k * n + r];
         if (e < 0) continue;
         const long long vidx = h->fmt == FMT_ELL ? (long long)k * n + r : e;
-        const int off = h->h_ell_col[(size_t)k * n + r] - r;
-        bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (off + 128));
+        const int col = h->h_ell_col[(size_t)k * n + r];
+        bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (col % Wb));
       }
-    if (cudaMalloc(&h->d_bnd, sizeof(int32_t) * bnd.size()) != cudaSuccess)
+    if (!h->d_bnd && cudaMalloc(&h->d_bnd, sizeof(int32_t) * bnd.size()) != cudaSuccess)
       return done(fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed"));
     if (cudaMemcpy(h->d_bnd, bnd.data(), sizeof(int32_t) * bnd.size(), cudaMemcpyHostToDevice) !=
         cudaSuccess)
       return done(fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed"));
+    h->bnd_w = Wb;
   }
   if (bv->smem_bytes > 48 * 1024)
     CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1079,8 +1082,7 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
                                                          bv->smem_bytes));
   if (occ < 1) return done(fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident"));
   const int grid = (int)std::min<long long>((long long)occ * h->num_sms, h->batch);
-  const int Wb = 2 * bv->kb + 1;
-  const size_t need = sizeof(double) * (size_t)grid * ((size_t)n * Wb + n);
+  const size_t need = sizeof(double) * (size_t)grid * 2 * ((size_t)n * Wb + n);  // 2 buffers / CTA
   if (h->bws_bytes < need) {
     cudaFree(h->d_bws);
     h->d_bws = nullptr;
