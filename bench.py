@@ -51,8 +51,9 @@ def parse():
                     default="auto")
     ap.add_argument("--block-threads", type=int, default=0)
     ap.add_argument("--reg-slots", type=int, default=0)
-    ap.add_argument("--solver", choices=["bicgstab", "gmres"], default="bicgstab",
-                    help="Krylov solver (BiCGSTAB = the paper's Algorithm 1)")
+    ap.add_argument("--solver", choices=["bicgstab", "gmres", "banded"], default="bicgstab",
+                    help="BiCGSTAB = the paper's Algorithm 1; gmres = f3; banded = the "
+                         "dgbsv-analogue direct solver (SURVEY.md 8(f) f4)")
     ap.add_argument("--precond", choices=["jacobi", "none"], default="jacobi")
     ap.add_argument("--restart", type=int, default=7, help="GMRES restart length m")
     ap.add_argument("--tol", type=float, default=1e-10)
@@ -238,7 +239,8 @@ def run_reference(args, rank, world):
     if rank != 0:
         return
     per_rank = rank_slice_count(args, world)
-    cal = oracle_sample_rate(0, per_rank, args, target_s=min(5.0, args.cpu_seconds))
+    cal = oracle_sample_rate(0, per_rank, args, target_s=min(5.0, args.cpu_seconds),
+                             kind="banded" if args.solver == "banded" else "bicgstab")
     count = cal["_count"]
     import oracle as O
     pat, Bs = make_csr_sample(0, count, args)
@@ -246,7 +248,10 @@ def run_reference(args, rank, world):
     times = []
     for s in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        oracle_krylov(O, pat, Bs, args, cores)
+        if args.solver == "banded":
+            O.batch_banded(pat.row_ptr, pat.col_idx, Bs.values, Bs.b, threads=cores)
+        else:
+            oracle_krylov(O, pat, Bs, args, cores)
         dt = time.perf_counter() - t0
         if s >= args.warmup:
             times.append(dt)
@@ -260,7 +265,9 @@ def run_reference(args, rank, world):
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": f"{count} systems (g=0..{count - 1}) of the workload per step"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-        "note": "CPU oracle (oracle/oracle.c, Alg. 1) on the host cores; the paper has no "
+        "note": f"CPU oracle (oracle/oracle.c, "
+                f"{'banded LU' if args.solver == 'banded' else 'Alg. 1'}) on the host cores; "
+                "the paper has no "
                 "public code and this tier has no installable reference",
     }
     emit(line, args)
@@ -280,7 +287,8 @@ def config_dict(args, world, per_rank):
             "global_batch": args.batch * world if args.scaling == "weak" else args.batch, "n": n,
             "grid": f"{args.nx}x{args.ny}", "format": args.format, "placement": args.placement,
             "tol": args.tol, "stop": "rel_b", "maxiter": args.maxiter, "x0": "zero",
-            "solver": args.solver if args.solver == "bicgstab" else f"gmres({args.restart})",
+            "solver": (f"gmres({args.restart})" if args.solver == "gmres" else
+                       "banded LU (dgbsv analogue)" if args.solver == "banded" else args.solver),
             "precond": args.precond,
             "parallelism": f"batch-partitioned x{world} (one process per GPU, no solve-path "
                            f"collective)",
@@ -522,6 +530,138 @@ def run_ours(args, rank, world, local_rank):
         emit(line, args)
 
 
+# ------------------------------------------------------ banded (f4) arm --
+def run_banded(args, rank, world, local_rank):
+    """--solver banded: the batched banded LU + solve (bsolve_banded_solve,
+    the dgbsv analogue of SURVEY.md 8(f) f4) on the same workload.  A direct
+    solve meets the tol 1e-10 residual bar by construction (checked below)."""
+    import torch
+    from paper_conf_ipps_kashinksla22_b200 import Solver
+    from paper_conf_ipps_kashinksla22_b200.parallel import max_over_ranks, rank_slice
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    sl = rank_slice(args.batch, rank, world, args.scaling)
+    per_rank, g0 = sl.count, sl.g0
+    pat, vals_h, b_h = make_inputs(g0, per_rank, args, pinned=True)
+    n, nnz = pat.n, pat.nnz
+    S = Solver(pat.row_ptr, pat.col_idx, per_rank, format=args.format, device=local_rank)
+    vals = vals_h.to(dev)
+    b = b_h.to(dev)
+    x = torch.empty((per_rank, n), dtype=torch.float64, device=dev)
+    info_d = torch.empty(per_rank, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            import torch.distributed as dist
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(max(args.warmup, 0)):
+        S.banded_solve(vals, b, out=(x, info_d))
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launch = []
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ea.record(stream)
+            S.banded_solve(vals, b, out=(x, info_d))
+            eb.record(stream)
+            launch.append((ea, eb))
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    total_ms = max_over_ranks(ev0.elapsed_time(ev1), device=dev)
+    kern_ms = [a.elapsed_time(bb) for a, bb in launch]
+    kern_s = statistics.mean(kern_ms) * 1e-3
+    value = sl.total * args.steps / (total_ms * 1e-3)
+    info = S.info
+    kl, ku = info["kl"], info["ku"]
+    kb = next(k for k in (4, 8, 16, 33, 65) if k >= max(kl, ku))
+    Wb = 2 * kb + 1
+    # algorithmic FP64 work per system (DESIGN.md "Kernel f4"): dgbtf2's
+    # updates on the kl x (kl + ku) band window + the b column, and the two
+    # triangular solves: 2 n kl (kl + ku + 1) + 2 n (kl + ku + 1) flop
+    flops_sys = 2.0 * n * kl * (kl + ku + 1) + 2.0 * n * (kl + ku + 1)
+    fp64_peak = 64 * 2 * info["num_sms"] * 1965e6
+    hbm_sys = 8 * (vals.numel() / per_rank + 2 * n) + 4 + 2 * 8 * n * (Wb + 1)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:  # noqa: BLE001
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0)) * 1e9
+    roof = {"bound": "alu", "achieved": flops_sys * per_rank / kern_s / 1e12,
+            "peak": fp64_peak / 1e12, "unit": "TFLOP/s",
+            "frac": flops_sys * per_rank / kern_s / fp64_peak, "traffic": None,
+            "kernel": f"banded_lu_kernel<{kb},{kb}> (one launch per step)",
+            "algorithmic_flops_per_unit": flops_sys, "units_per_launch": per_rank,
+            "peak_source": "derived: 64 DFMA/clk/SM x 148 SMs x 1965 MHz (FP64 pipe)",
+            "kernel_ms_avg": kern_s * 1e3,
+            "hbm": {"achieved": hbm_sys * per_rank / kern_s / 1e9, "peak": hbm_peak / 1e9,
+                    "unit": "GB/s", "frac": hbm_sys * per_rank / kern_s / hbm_peak,
+                    "bytes_per_system": hbm_sys,
+                    "note": "values + b + x + info + the U/y workspace written and read back"}}
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic_banded.json")))
+        roof["hbm"]["traffic"] = tr["dram_bytes_per_launch"] * per_rank / tr["systems_per_launch"]
+        roof["traffic_source"] = tr["source"]
+    except Exception:  # noqa: BLE001
+        pass
+    # e2e: pinned host -> device inputs, the solve, device -> host x and info
+    e2e = None
+    if not args.no_e2e:
+        xh = torch.empty((per_rank, n), dtype=torch.float64, pin_memory=True)
+        ih = torch.empty(per_rank, dtype=torch.int32, pin_memory=True)
+        steps = max(1, min(args.steps, 3))
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(steps):
+            vals.copy_(vals_h, non_blocking=True)
+            b.copy_(b_h, non_blocking=True)
+            S.banded_solve(vals, b, out=(x, info_d))
+            xh.copy_(x, non_blocking=True)
+            ih.copy_(info_d, non_blocking=True)
+        torch.cuda.synchronize()
+        dt = max_over_ranks(time.perf_counter() - t0, device=dev)
+        e2e = {"value": sl.total * steps / dt, "unit": UNIT,
+               "h2d_bytes_per_step": int(vals_h.numel() * 8 + b_h.numel() * 8),
+               "d2h_bytes_per_step": int(per_rank * (8 * n + 4)), "steps": steps,
+               "api": "Solver.banded_solve (C ABI bsolve_banded_solve) + pinned copies"}
+    info_h = info_d.cpu().numpy()
+    xs = x[: min(per_rank, 2000)].cpu().numpy()
+    cpu, parity = None, None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cb = oracle_sample_rate(g0, per_rank, args, target_s=args.cpu_seconds, kind="banded")
+        o, cnt = cb.pop("_out"), cb.pop("_count")
+        Bs = cb.pop("_csr")
+        cnt = min(cnt, xs.shape[0])
+        import oracle as O
+        rel = np.linalg.norm(xs[:cnt] - o["x"][:cnt], axis=1) / np.linalg.norm(o["x"][:cnt], axis=1)
+        res = max(np.linalg.norm(Bs.b[i] - O.spmv(pat.row_ptr, pat.col_idx, Bs.values[i], xs[i]))
+                  / np.linalg.norm(Bs.b[i]) for i in range(min(cnt, 64)))
+        cpu = cb
+        parity = {"systems_checked": int(cnt), "oracle": "banded LU, dgbtf2 + dgbtrs order "
+                  "(oracle/oracle.c)", "max_rel_x_diff_vs_oracle": float(rel.max()),
+                  "max_true_rel_residual_gpu_first64": float(res)}
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_dict(args, world, per_rank), "roofline": roof, "cpu_baseline": cpu,
+        "e2e": e2e, "clocks": clk.summary(), "gpu_launches": args.steps,
+        "plan": {"kb": kb, "window": Wb, "kl": kl, "ku": ku},
+        "solve_stats": {"info_nonzero": int((info_h != 0).sum())}, "parity_sample": parity,
+        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms)},
+    }
+    if rank == 0:
+        emit(line, args)
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -536,7 +676,10 @@ def main():
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
-        run_ours(args, rank, world, local_rank)
+        if args.solver == "banded":
+            run_banded(args, rank, world, local_rank)
+        else:
+            run_ours(args, rank, world, local_rank)
     finally:
         if world > 1:
             import torch.distributed as dist

@@ -108,6 +108,21 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
                    saddr(bar))
                : "memory");
 }
+// try_wait with a back-off: the back-substitution warp waits most of the
+// time (the factorisation is the long pole) and must not steal issue slots
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+  uint32_t ok;
+  for (;;) {
+    asm volatile(
+        "{\n.reg .pred p;\nmbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
+        "selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(saddr(bar)), "r"(parity)
+        : "memory");
+    if (ok) return;
+    __nanosleep(1000);
+  }
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
   asm volatile(
       "{\n.reg .pred p;\nW%=:\n"
@@ -177,7 +192,7 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
     int k = 0;
     for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x, ++k) {
       const int b = k & 1;
-      mbar_wait(&full_bar[b], (k >> 1) & 1);
+      mbar_wait_sleep(&full_bar[b], (k >> 1) & 1);
       const double *U = ws + b * ws_sys;
       const double *Y = U + (size_t)n * W;
       constexpr int PF = 8;  // U entries are loaded PF steps ahead
@@ -337,6 +352,8 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
           const double2 m = cb[(kk - 1) / 2];
           v[kk - 1] = fma(-m.x, w, v[kk]);
           if (kk + 1 < R) v[kk] = fma(-m.y, w, v[kk + 1]);
+          // keep at most 6 multiplier pairs in flight (register pressure)
+          if ((kk - 1) % 12 == 10) asm volatile("" ::: "memory");
         }
         // row j leaves; row j+KL+1 (ring slot j mod R) enters as window row KL
         v[KL] = ring[jr * RB + t];
