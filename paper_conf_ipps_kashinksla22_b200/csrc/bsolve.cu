@@ -495,10 +495,13 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const int lg = genv ? atoi(genv) : 4;  // measured best: 7.33 vs 7.05 (G=2) M sys/s
     const char *rowsenv = getenv("BSOLVE_TMEM_LINE_ROWS");  // rows per thread: 8 or 4
     const int lr = rowsenv ? atoi(rowsenv) : 8;
+    const char *roundsenv = getenv("BSOLVE_ROUNDS");  // BiCGSTAB reduction rounds: 3 or 2
+    const int lrounds = roundsenv ? atoi(roundsenv) : 3;
     // first pass: the requested geometry; second pass: any variant for the grid
     for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
       const LVariant &cand = lv[i % lcnt];
       if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
+      if (!gm && cand.rounds != lrounds) continue;
       if (i < lcnt && (cand.g != lg || cand.r != lr)) continue;
       const int NX = cand.nx;
       const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};

@@ -8,15 +8,19 @@
 using namespace bsolve;
 
 #define LSMEM_(NX, R) ((R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 + 16)
-#define LV_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), \
+#define LV_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 3, \
                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB>}
+// two reduction rounds per iteration (deferred stop test 1, algebraic rho)
+#define LV2_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 2, \
+                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB, 2, 2>}
 // GMRES: + the Krylov basis and the triangular factor in SMEM
 #define LVG_(NX, R, G) {NX, R, G, SOLVER_GMRES,                                          \
-                        LSMEM_(NX, R) + (kMaxRestart * 1024 + kMaxRestart * kMaxRestart) * 8, \
+                        LSMEM_(NX, R) + (kMaxRestart * 1024 + kMaxRestart * kMaxRestart) * 8, 0, \
                         (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_GMRES>}
 static const LVariant kLVariants[] = {LV_(32, 8, 2),  LV_(32, 8, 4),  LV_(32, 4, 2),
                                       LV_(32, 4, 4),  LV_(31, 8, 4),  LV_(31, 4, 2),
-                                      LVG_(32, 8, 2), LVG_(31, 8, 2)};
+                                      LVG_(32, 8, 2), LVG_(31, 8, 2), LV2_(32, 8, 4),
+                                      LV2_(31, 8, 4)};
 
 const LVariant *variants_line(int *count) {
   *count = (int)(sizeof(kLVariants) / sizeof(kLVariants[0]));

@@ -44,6 +44,7 @@ struct LVariant {
   int nx, r, g;  // grid width, rows per thread (CTA = 1024 / r threads), TMEM load group
   int solver;    // SOLVER_BICGSTAB or SOLVER_GMRES
   int smem_bytes;  // dynamic SMEM of one CTA (gather planes + scratch + TMEM slot)
+  int rounds;      // BiCGSTAB reduction rounds per iteration (3, or 2: algebraic rho)
   solve_fn fn;
 };
 
