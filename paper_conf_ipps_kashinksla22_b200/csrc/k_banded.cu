@@ -12,7 +12,7 @@ using namespace bband;
 #define BV_(K, MINB)                                                              \
   {K, Geo<K, K>::NT, Geo<K, K>::NTF - Geo<K, K>::W - 1, Geo<K, K>::smem_bytes,    \
    (banded_fn)banded_lu_kernel<K, K, MINB>}
-static const BVariant kBVariants[] = {BV_(4, 8), BV_(8, 8), BV_(16, 5), BV_(33, 4), BV_(65, 1)};
+static const BVariant kBVariants[] = {BV_(4, 8), BV_(8, 8), BV_(16, 5), BV_(33, 5), BV_(65, 1)};
 
 const BVariant *variants_banded(int *count) {
   *count = (int)(sizeof(kBVariants) / sizeof(kBVariants[0]));
