@@ -117,8 +117,12 @@ enum {
 enum {
   BSOLVE_SYS_CONVERGED = 0, /* final TRUE ||b - A x||_2 < tau                 */
   BSOLVE_SYS_MAXITER = 1,   /* maxiter iterations done without convergence    */
-  BSOLVE_SYS_BREAKDOWN = 2  /* a BiCGSTAB denominator was 0 or non-finite;
+  BSOLVE_SYS_BREAKDOWN = 2, /* a BiCGSTAB denominator was 0 or non-finite;
                                x is the last finite iterate                   */
+  BSOLVE_SYS_DIRECT = 3     /* direct_fallback: the iterative solve did not
+                               converge (status 1 or 2) and x comes from the
+                               banded LU (bsolve_banded_solve); resnorm is
+                               its true residual, iters the iterative count   */
 };
 
 typedef struct bsolve_options {
@@ -139,6 +143,12 @@ typedef struct bsolve_options {
   int precond;             /* BSOLVE_PREC_*   (default JACOBI)                 */
   int restart;             /* GMRES: Krylov steps per restart cycle m,
                               1 <= m <= BSOLVE_MAX_RESTART (default 7)        */
+  int direct_fallback;     /* 1: after the iterative solve, every system whose
+                              status is not CONVERGED is re-solved by the
+                              banded LU in a second launch
+                              on the same stream and gets status DIRECT; a
+                              singular band keeps the iterative result.
+                              Needs status != NULL in bsolve_run (default 0) */
 } bsolve_options;
 
 typedef struct bsolve_info {

@@ -23,7 +23,7 @@ STOP_REL_B, STOP_ABS = 0, 1
 SOLVER_BICGSTAB, SOLVER_GMRES = 0, 1
 PREC_JACOBI, PREC_NONE = 0, 1
 MAX_RESTART = 7
-SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN = 0, 1, 2
+SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN, SYS_DIRECT = 0, 1, 2, 3
 
 _FMT = {"auto": FMT_AUTO, "csr": FMT_CSR, "ell": FMT_ELL}
 _PLACE = {"auto": PLACE_AUTO, "smem": PLACE_SMEM, "stream": PLACE_STREAM, "regs": PLACE_REGS,
@@ -43,7 +43,7 @@ class Options(C.Structure):
     _fields_ = [("format", C.c_int), ("placement", C.c_int), ("stop", C.c_int),
                 ("true_residual_check", C.c_int), ("device", C.c_int),
                 ("block_threads", C.c_int), ("reg_slots", C.c_int), ("solver", C.c_int),
-                ("precond", C.c_int), ("restart", C.c_int)]
+                ("precond", C.c_int), ("restart", C.c_int), ("direct_fallback", C.c_int)]
 
 
 class Info(C.Structure):
@@ -139,14 +139,16 @@ class Solver:
 
     Solver(row_ptr, col_idx, batch, format="ell", placement="auto",
            stop="rel_b", true_residual_check=True, device=None,
-           solver="bicgstab" | "gmres", precond="jacobi" | "none", restart=7)
+           solver="bicgstab" | "gmres", precond="jacobi" | "none", restart=7,
+           direct_fallback=False)
     .run(values, b, x0=None, tol=1e-10, maxiter=1000) -> (x, iters, resnorm, status)
     """
 
     def __init__(self, row_ptr, col_idx, batch: int, *, format: str = "ell",
                  placement: str = "auto", stop: str = "rel_b", true_residual_check: bool = True,
                  device: int | None = None, block_threads: int = 0, reg_slots: int = 0,
-                 solver: str = "bicgstab", precond: str = "jacobi", restart: int = MAX_RESTART):
+                 solver: str = "bicgstab", precond: str = "jacobi", restart: int = MAX_RESTART,
+                 direct_fallback: bool = False):
         L = lib()
         rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
         ci = np.ascontiguousarray(col_idx, dtype=np.int32)
@@ -164,6 +166,7 @@ class Solver:
         opt.solver = _SOLVER[solver]
         opt.precond = _PREC[precond]
         opt.restart = int(restart)
+        opt.direct_fallback = int(bool(direct_fallback))
         h = _P()
         check(L.bsolve_create(C.byref(h), self.n, self.batch, rp.ctypes.data, ci.ctypes.data,
                               C.byref(opt)))

@@ -46,8 +46,15 @@ struct BandParams {
   const double *b;        // [batch][n]
   const int32_t *bnd;     // [E][n]: (value index << 8) | (col mod W), -1 = none
   double *x;              // [batch][n] out
-  int32_t *info;          // [batch] out: 0, or j+1 if u_jj == 0 (LAPACK convention)
+  int32_t *info;          // [batch] out or nullptr: 0, or j+1 if u_jj == 0 (LAPACK)
   int32_t *ipiv;          // [batch][n] out or nullptr: row swapped with row j (0-based)
+  const int32_t *cols;    // [E][n] column of entry e of row r (residual in fallback mode)
+  int8_t *only;           // fallback mode: [batch] status of the iterative solve; systems
+                          // with 0 (converged) are skipped, the others get x = the direct
+                          // solution, resnorm = its true residual, only[i] = 3 (DIRECT);
+                          // a singular band (info > 0) leaves x, resnorm and status as
+                          // they were.  nullptr: solve every system.
+  double *resnorm;        // fallback mode: [batch] out
   double *ws;             // per CTA: U [n][W] (row j: 1/u_jj, u_j,j+1 ..) then y [n]
   long long sys_stride;
   int E, n, batch;
@@ -165,6 +172,7 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
   __shared__ int s_info;
   // workspace hand-off factor warps -> back-substitution warp (2 buffers)
   __shared__ __align__(8) uint64_t full_bar[2], empty_bar[2];
+  __shared__ int s_info_buf[2];  // info of the system in workspace buffer b
 
   const int t = threadIdx.x;
   const int n = P.n;
@@ -190,9 +198,11 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
     // the row-major U (L1-cached: each lane walks its rows backwards).
     const int l = t - NTF;
     int k = 0;
-    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x, ++k) {
+    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+      if (P.only && P.only[sys] == 0) continue;  // converged iteratively (same test as below)
       const int b = k & 1;
       mbar_wait_sleep(&full_bar[b], (k >> 1) & 1);
+      const bool skip = P.only && s_info_buf[b] != 0;  // singular: keep the iterative result
       const double *U = ws + b * ws_sys;
       const double *Y = U + (size_t)n * W;
       constexpr int PF = 8;  // U entries are loaded PF steps ahead
@@ -212,7 +222,7 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
         for (int m = 0; m < NA; ++m) q[s][m] = uload(n - 1 - s, m);
       double *xs = P.x + sys * n;
 #pragma unroll 1
-      for (int jb0 = n - 1; jb0 >= 0; jb0 -= PF) {
+      for (int jb0 = skip ? -1 : n - 1; jb0 >= 0; jb0 -= PF) {
 #pragma unroll
         for (int s = 0; s < PF; ++s) {
           const int j = jb0 - s;
@@ -244,6 +254,28 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
       }
       __syncwarp();
       if (l == 0) mbar_arrive1(&empty_bar[b]);  // buffer b may be overwritten
+      if (P.only && !skip) {
+        // true residual ||b - A x||_2 of the direct solution (plain sum of
+        // squares per lane, then a butterfly), x re-read from L2
+        const double *val = P.values + sys * P.sys_stride;
+        const double *bb = P.b + sys * n;
+        double ss = 0.0;
+        for (int r = l; r < n; r += 32) {
+          double acc = __ldg(bb + r);
+          for (int e = 0; e < P.E; ++e) {
+            const int pk = __ldg(P.bnd + (size_t)e * n + r);
+            if (pk >= 0) acc -= __ldg(val + (pk >> 8)) * __ldcg(xs + __ldg(P.cols + (size_t)e * n + r));
+          }
+          ss += acc * acc;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+        if (l == 0) {
+          P.resnorm[sys] = sqrt(ss);
+          P.only[sys] = 3;  // BSOLVE_SYS_DIRECT
+        }
+      }
+      ++k;
     }
     return;
   }
@@ -253,7 +285,8 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
   const bool loader = t > W;
   const int lidx = t - W - 1;  // loader lane = pattern entry (needs NTF - W - 1 > E)
   int k = 0;
-  for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x, ++k) {
+  for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+    if (P.only && P.only[sys] == 0) continue;  // converged iteratively
     const int b = k & 1;
     if (k >= 2) mbar_wait(&empty_bar[b], ((k >> 1) - 1) & 1);  // back substitution k-2 done
     double *U = ws + b * ws_sys;
@@ -366,10 +399,12 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
     if (loader) cp_wait<0>();
     bar_factor(NTF);  // every U / y store of this system issued; s_info final
     if (t == 0) {
-      P.info[sys] = s_info;
+      if (P.info) P.info[sys] = s_info;
+      s_info_buf[b] = s_info;
       __threadfence_block();
       mbar_arrive1(&full_bar[b]);  // release: U, y of buffer b are complete
     }
+    ++k;
   }
 }
 

@@ -116,6 +116,7 @@ struct bsolve_plan {
   // banded direct solver (bsolve_banded_solve, lazily set up)
   int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
   int bnd_w = 0;              // window width the table's ring positions use
+  int direct_fallback = 0;    // bsolve_options.direct_fallback
   double *d_bws = nullptr;    // per-CTA U + y workspace
   size_t bws_bytes = 0;
 };
@@ -132,6 +133,7 @@ extern "C" void bsolve_default_options(bsolve_options *o) {
   o->solver = BSOLVE_SOLVER_BICGSTAB;
   o->precond = BSOLVE_PREC_JACOBI;
   o->restart = BSOLVE_MAX_RESTART;
+  o->direct_fallback = 0;
 }
 
 static void free_plan(bsolve_plan *h) {
@@ -340,6 +342,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   h->solver = opt.solver;
   h->precond = opt.precond;
   h->restart = opt.solver == BSOLVE_SOLVER_GMRES ? opt.restart : 0;
+  h->direct_fallback = opt.direct_fallback ? 1 : 0;
   h->sys_stride = h->fmt == FMT_ELL ? (long long)W * n : nnz;
 
   // bandwidth (for bsolve_info; the banded structure is not used by the solve)
@@ -801,6 +804,10 @@ static int check_run_args(bsolve_handle h, const double *values, const double *b
   return BSOLVE_OK;
 }
 
+static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
+                         int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
+                         int8_t *only, double *resnorm);
+
 static int launch_solve(bsolve_handle h, const double *values, const double *b, const double *x0,
                         double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
                         int8_t *status, int count, cudaStream_t stream) {
@@ -865,6 +872,8 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));
+  if (h->direct_fallback)  // non-converged systems -> banded LU
+    return launch_banded(h, values, b, x, nullptr, nullptr, count, stream, status, resnorm);
   return BSOLVE_OK;
 }
 
@@ -891,6 +900,9 @@ extern "C" int bsolve_run(bsolve_handle h, const double *values, const double *b
   int rc = check_run_args(h, values, b, tol, maxiter, x, iters, resnorm);
   if (rc) return rc;
   if (h->batch == 0) return BSOLVE_OK;
+  if (h->direct_fallback && !status)
+    return fail(BSOLVE_ERR_INVALID, "direct_fallback needs the status array (it selects the "
+                                    "systems the banded solver re-solves)");
   const void *ptrs[] = {values, b, x0, x, iters, resnorm, status};
   const char *names[] = {"values", "b", "x0", "x", "iters", "resnorm", "status"};
   for (int i = 0; i < 7; ++i)
@@ -1025,18 +1037,15 @@ extern "C" int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, doub
 }
 
 // ---------------------------------------------- banded direct solver (f4) --
-extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b,
-                                   double *x, int32_t *info, int32_t *ipiv, void *stream) {
-  g_err.clear();
-  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
-  if (h->batch == 0) return BSOLVE_OK;
-  if (!values || !b || !x || !info)
-    return fail(BSOLVE_ERR_INVALID, "values, b, x and info must be non-NULL");
-  int rc;
-  const void *ptrs[] = {values, b, x, info, ipiv};
-  const char *names[] = {"values", "b", "x", "info", "ipiv"};
-  for (int i = 0; i < 5; ++i)
-    if ((rc = check_device_ptr(h, ptrs[i], names[i]))) return rc;
+// Enqueue the banded LU kernel over `count` systems.  Fallback mode
+// (only != NULL): systems with only[i] == BSOLVE_SYS_CONVERGED are skipped;
+// for the others x is replaced by the direct solution (unless the band is
+// singular), resnorm[i] by its true residual and status[i] by
+// BSOLVE_SYS_DIRECT (only and status_out are the same array).
+static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
+                         int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
+                         int8_t *only, double *resnorm) {
+  if (count <= 0) return BSOLVE_OK;
   const int kb = std::max(h->kl, h->ku);
   int cnt = 0;
   const BVariant *tab = variants_banded(&cnt), *bv = nullptr;
@@ -1049,13 +1058,6 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
   if ((long long)h->sys_stride >= (1LL << 23))
     return fail(BSOLVE_ERR_UNSUPPORTED, "banded solver: %lld values per system exceed 2^23",
                 h->sys_stride);
-  int prev = -1;
-  cudaGetDevice(&prev);
-  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
-  auto done = [&](int code) {
-    if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
-    return code;
-  };
   const int n = h->n, W = h->W;
   const int Wb = 2 * bv->kb + 1;  // the instance's window width
   if (!h->d_bnd || h->bnd_w != Wb) {
@@ -1071,10 +1073,10 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
         bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (col % Wb));
       }
     if (!h->d_bnd && cudaMalloc(&h->d_bnd, sizeof(int32_t) * bnd.size()) != cudaSuccess)
-      return done(fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed"));
+      return fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed");
     if (cudaMemcpy(h->d_bnd, bnd.data(), sizeof(int32_t) * bnd.size(), cudaMemcpyHostToDevice) !=
         cudaSuccess)
-      return done(fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed"));
+      return fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed");
     h->bnd_w = Wb;
   }
   if (bv->smem_bytes > 48 * 1024)
@@ -1083,8 +1085,8 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
   int occ = 0;
   CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)bv->fn, bv->nt,
                                                          bv->smem_bytes));
-  if (occ < 1) return done(fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident"));
-  const int grid = (int)std::min<long long>((long long)occ * h->num_sms, h->batch);
+  if (occ < 1) return fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident");
+  const int grid = (int)std::min<long long>((long long)occ * h->num_sms, count);
   const size_t need = sizeof(double) * (size_t)grid * 2 * ((size_t)n * Wb + n);  // 2 buffers / CTA
   if (h->bws_bytes < need) {
     cudaFree(h->d_bws);
@@ -1092,7 +1094,7 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
     h->bws_bytes = 0;
     if (cudaMalloc(&h->d_bws, need) != cudaSuccess) {
       cudaGetLastError();
-      return done(fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need));
+      return fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need);
     }
     h->bws_bytes = need;
   }
@@ -1100,19 +1102,42 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
   P.values = values;
   P.b = b;
   P.bnd = h->d_bnd;
+  P.cols = h->d_ell_col;
   P.x = x;
   P.info = info;
   P.ipiv = ipiv;
+  P.only = only;
+  P.resnorm = resnorm;
   P.ws = h->d_bws;
   P.sys_stride = h->sys_stride;
   P.E = W;
   P.n = n;
-  P.batch = h->batch;
-  bv->fn<<<grid, bv->nt, bv->smem_bytes, (cudaStream_t)stream>>>(P);
+  P.batch = count;
+  bv->fn<<<grid, bv->nt, bv->smem_bytes, stream>>>(P);
   cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess)
-    return done(fail(BSOLVE_ERR_CUDA, "banded launch: %s", cudaGetErrorString(e)));
-  return done(BSOLVE_OK);
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "banded launch: %s", cudaGetErrorString(e));
+  return BSOLVE_OK;
+}
+
+extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b,
+                                   double *x, int32_t *info, int32_t *ipiv, void *stream) {
+  g_err.clear();
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (h->batch == 0) return BSOLVE_OK;
+  if (!values || !b || !x || !info)
+    return fail(BSOLVE_ERR_INVALID, "values, b, x and info must be non-NULL");
+  int rc;
+  const void *ptrs[] = {values, b, x, info, ipiv};
+  const char *names[] = {"values", "b", "x", "info", "ipiv"};
+  for (int i = 0; i < 5; ++i)
+    if ((rc = check_device_ptr(h, ptrs[i], names[i]))) return rc;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  rc = launch_banded(h, values, b, x, info, ipiv, h->batch, (cudaStream_t)stream, nullptr,
+                     nullptr);
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  return rc;
 }
 
 extern "C" int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz) {

@@ -202,3 +202,41 @@ def test_ell_map_slot0_diagonal_and_stencil_offsets():
     rp, ci = X.random_pattern(200, 9, seed=7)
     W, cols, src = pkg.ell_layout(rp, ci)
     assert np.all(cols[:200] == np.arange(200)) and np.all(src[:200] >= 0)
+
+
+def _header_struct_fields(name):
+    txt = re.sub(r"/\*.*?\*/", "", open(HEADER).read(), flags=re.S)
+    body = re.search(r"typedef struct " + name + r" \{(.*?)\}", txt, flags=re.S).group(1)
+    fields = []
+    for decl in body.split(";"):
+        decl = decl.strip()
+        if decl:
+            fields += [f.strip() for f in decl.split(None, 1)[1].split(",")]
+    return fields
+
+
+def test_binding_structs_match_the_header():
+    """The ctypes mirrors of bsolve_options / bsolve_info list the header's
+    int fields in the header's order (a mismatch would shift every option)."""
+    assert [f for f, _ in B.Options._fields_] == _header_struct_fields("bsolve_options")
+    assert [f for f, _ in B.Info._fields_] == _header_struct_fields("bsolve_info")
+
+
+def test_direct_fallback_needs_status():
+    """direct_fallback selects the systems to re-solve from status[]: a NULL
+    status is rejected before any CUDA call."""
+    rp = np.array([0, 1], np.int32)
+    ci = np.array([0], np.int32)
+    L = B.lib()
+    opt = B.Options()
+    L.bsolve_default_options(C.byref(opt))
+    assert opt.direct_fallback == 0
+    opt.direct_fallback = 1
+    h = B._P()
+    rc = L.bsolve_create(C.byref(h), 1, 1, rp.ctypes.data, ci.ctypes.data, C.byref(opt))
+    if rc != B.OK:  # no GPU in this container: create fails at the device query
+        pytest.skip("bsolve_create needs a CUDA device")
+    d = C.c_void_p(1)
+    rc = L.bsolve_run(h, d, d, None, 1e-10, 10, d, d, d, None, None)
+    L.bsolve_destroy(h)
+    assert rc == B.ERR_INVALID

@@ -161,3 +161,53 @@ def test_bandwidth_too_large_is_unsupported():
     with pytest.raises(BsolveError) as e:
         S.banded_solve(v, b)
     assert e.value.code == ERR_UNSUPPORTED
+
+
+# ------------------------------------------- direct fallback in bsolve_run --
+def _run(p, vals, b, **kw):
+    maxiter = kw.pop("maxiter", 1000)
+    S = Solver(p.row_ptr, p.col_idx, vals.shape[0], **kw)
+    ev = to_dev(S.ell_values(vals))
+    x, it, res, st = S.run(ev, to_dev(b), maxiter=maxiter)
+    torch.cuda.synchronize()
+    out = x.cpu().numpy(), it.cpu().numpy(), res.cpu().numpy(), st.cpu().numpy()
+    return S, out
+
+
+def test_direct_fallback_replaces_non_converged():
+    """maxiter = 6: ions converge (status 0, untouched), electrons do not
+    (status 1) and are re-solved by the banded LU: status DIRECT (3), x = the
+    oracle's banded solution, resnorm = its true residual, iters kept."""
+    B = X.make_batch(0, 300)
+    p = B.pattern
+    _, (x0, it0, r0, s0) = _run(p, B.values, B.b, maxiter=6)
+    assert np.any(s0 == 0) and np.any(s0 == 1)
+    _, (x1, it1, r1, s1) = _run(p, B.values, B.b, maxiter=6, direct_fallback=True)
+    conv = s0 == 0
+    assert np.array_equal(s1[conv], s0[conv]) and np.array_equal(x1[conv], x0[conv])
+    assert np.array_equal(r1[conv], r0[conv])
+    assert np.all(s1[~conv] == 3) and np.array_equal(it1, it0)
+    xo, io, _ = oracle_banded(p.row_ptr, p.col_idx, B.values[~conv], B.b[~conv])
+    assert np.all(io == 0)
+    rel = np.linalg.norm(x1[~conv] - xo, axis=1) / np.linalg.norm(xo, axis=1)
+    assert rel.max() <= 1e-12
+    bn = np.linalg.norm(B.b[~conv], axis=1)
+    tr = np.array([np.linalg.norm(B.b[k] - O.spmv(p.row_ptr, p.col_idx, B.values[k], x1[k]))
+                   for k in np.nonzero(~conv)[0]])
+    assert np.all(r1[~conv] <= 1e-13 * bn) and np.allclose(r1[~conv], tr, rtol=0.5, atol=1e-14 * bn.max())
+
+
+def test_direct_fallback_singular_keeps_iterative_result_and_host_path():
+    """A singular band cannot be solved directly: that system keeps its
+    iterative x, resnorm and status; run_host gives the same outputs."""
+    pat = X.stencil_pattern(32, 31)
+    v = X.random_dd_values(pat.row_ptr, pat.col_idx, 4, seed=11).copy()
+    v[2, pat.col_idx == 500] = 0.0          # column 500 of A_2 is zero: singular
+    b = X.random_rhs(4, pat.n, seed=2)
+    _, (x0, it0, r0, s0) = _run(pat, v, b, maxiter=2)
+    S, (x1, it1, r1, s1) = _run(pat, v, b, maxiter=2, direct_fallback=True)
+    assert s0[2] != 0 and s1[2] == s0[2] and np.array_equal(x1[2], x0[2]) and r1[2] == r0[2]
+    others = [0, 1, 3]
+    assert np.all(s1[others] == 3)
+    xh, ih, rh, sh = S.run_host(S.ell_values(v), b, maxiter=2)
+    assert np.array_equal(sh, s1) and np.array_equal(xh, x1) and np.array_equal(rh, r1)
