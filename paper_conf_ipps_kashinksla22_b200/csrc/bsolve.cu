@@ -593,6 +593,28 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     // (opt-in via BSOLVE_TMEM_PERSIST=1: measured no faster than the per-system
     // launch, 6.89 vs 6.91 M sys/s -- the co-resident CTA already hides a
     // CTA's start-up)
+    // line-tiled plan, persistent with TMA prefetch of the next system
+    // (BSOLVE_LINE_PERSIST=1; 16-byte aligned system blocks, 8 rows/thread)
+    const char *lpenv = getenv("BSOLVE_LINE_PERSIST");
+    if (h->line_nx && lpenv && atoi(lpenv) == 1 && h->r == 8 && n % 2 == 0 &&
+        (h->sys_stride * 8) % 16 == 0) {
+      int sb = 0;
+      persist_fn f = variant_line_persist(h->line_nx, &sb, h->smem_vals, h->n_pad);
+      if (f && sb <= smem_optin &&
+          cudaFuncSetAttribute((const void *)f, cudaFuncAttributeMaxDynamicSharedMemorySize, sb) ==
+              cudaSuccess) {
+        cudaFuncSetAttribute((const void *)f, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             cudaSharedmemCarveoutMaxShared);
+        h->var_tmem_p = f;
+        h->smem_bytes_tmem_p = sb;
+        h->grid_tmem_p = 2 * h->num_sms;
+        if (cudaMalloc(&h->d_ctr, 2 * sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMemset(h->d_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
+          return fail_free(fail(BSOLVE_ERR_NOMEM, "work counter allocation failed"));
+      } else {
+        cudaGetLastError();
+      }
+    }
     const char *penv = getenv("BSOLVE_TMEM_PERSIST");
     const bool persist = (penv && atoi(penv) == 1) && !h->line_nx && h->nt == 128 && h->r == 8 &&
                          n % 2 == 0 && (h->sys_stride * 8) % 16 == 0;
@@ -841,7 +863,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)
-    if (h->var_tmem_p && aligned && !h->line_nx) {
+    if (h->var_tmem_p && aligned) {  // persistent (strided or line-tiled plan)
       const int grid = (int)std::min<long long>(h->grid_tmem_p, count);
       h->var_tmem_p<<<grid, h->nt, h->smem_bytes_tmem_p, stream>>>(P, h->d_ctr);
     } else {

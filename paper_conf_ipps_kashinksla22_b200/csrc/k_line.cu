@@ -26,3 +26,16 @@ const LVariant *variants_line(int *count) {
   *count = (int)(sizeof(kLVariants) / sizeof(kLVariants[0]));
   return kLVariants;
 }
+
+// persistent line-tiled kernel (TMA prefetch of the next system), 8 rows x 128 threads
+persist_fn variant_line_persist(int nx, int *smem_bytes, int smem_vals, int n_pad) {
+  if (nx == 32) {
+    *smem_bytes = line_persist_smem<32, 8, 4>(smem_vals, n_pad);
+    return (persist_fn)bicgstab_tmem_line_persist_kernel<32, 8, 4>;
+  }
+  if (nx == 31) {
+    *smem_bytes = line_persist_smem<31, 8, 4>(smem_vals, n_pad);
+    return (persist_fn)bicgstab_tmem_line_persist_kernel<31, 8, 4>;
+  }
+  return nullptr;
+}

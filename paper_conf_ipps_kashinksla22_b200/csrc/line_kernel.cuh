@@ -261,4 +261,132 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s), "n"(128));
 }
 
+// Persistent variant of the line-tiled TMEM kernel: 2 CTAs per SM loop over
+// systems claimed from a self-resetting work counter (dynamic, so ion and
+// electron systems balance).  While a CTA iterates on system i, a TMA bulk
+// copy stages system i+1's values, b and x0 into SMEM; at the switch the
+// threads move them SMEM -> registers / TMEM (tens of cycles instead of an
+// HBM round trip on the critical path).
+//   SMEM: [values staging: smem_vals] [b: n_pad] [x0: n_pad] [gather planes]
+//         [reduction scratch: 16 * NWARP] [mbarrier] [next system] [TMEM base]
+template <int NX, int R, int G>
+__host__ __device__ constexpr int line_persist_smem(int smem_vals, int n_pad) {
+  return (smem_vals + 2 * n_pad + R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 +
+         32;
+}
+
+template <int NX, int R, int G>
+__global__ void __launch_bounds__(1024 / R, 2)
+    bicgstab_tmem_line_persist_kernel(const SolveParams P, unsigned long long *ctr) {
+  constexpr int NT = 1024 / R, NWARP = NT / 32;
+  static_assert(R == 8, "8 rows per thread (one warp per TMEM lane quarter)");
+  using L = LineGeom<NX, NT, R>;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sval = reinterpret_cast<double *>(smem_raw);
+  double *sb = sval + P.smem_vals;
+  double *sx0 = sb + P.n_pad;
+  double *sg = sx0 + P.n_pad;
+  double *sred = sg + R * L::S;
+  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
+  volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 2);
+
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long batch = P.batch;
+  const int row0 = R * tid;
+  const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
+  const uint32_t nbytes = static_cast<uint32_t>(n * 8);
+  auto issue = [&](long long s) {  // one thread: TMA of system s into the staging buffers
+    mbar_arrive_expect_tx(mbar, vbytes + nbytes + (P.x0 ? nbytes : 0u));
+    const unsigned char *src = reinterpret_cast<const unsigned char *>(P.values + s * P.sys_stride);
+    constexpr uint32_t CH = 32768;
+    for (uint32_t off = 0; off < vbytes; off += CH)
+      tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off, src + off,
+                   vbytes - off < CH ? vbytes - off : CH, mbar);
+    tma_bulk_g2s(sb, P.b + s * n, nbytes, mbar);
+    if (P.x0) tma_bulk_g2s(sx0, P.x0 + s * n, nbytes, mbar);
+  };
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(128));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  for (int i = tid; i < R * (L::S - NT); i += NT) {  // zero guard columns once
+    const int pl = i / (L::S - NT), q = i % (L::S - NT);
+    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
+  }
+  bool act[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
+  if (tid == 32) {
+    mbar_init(mbar, 1);
+    fence_mbar_init();
+    const long long first = static_cast<long long>(atomicAdd(ctr, 1ull));
+    *s_next = first;
+    if (first < batch) issue(first);
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
+  long long cur = *s_next;
+  uint32_t phase = 0;
+  LineComm<NX, NT, R> comm(sg, sred, act);
+  while (cur < batch) {
+    mbar_wait_parity(mbar, phase);
+    phase ^= 1u;
+    double x[R], r[R], d[R], a0[R], bv[R];
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      a0[j] = act[j] ? sval[row0 + j] : 0.0;
+      d[j] = jacobi_inv(P.precond, a0[j]);
+      bv[j] = act[j] ? sb[row0 + j] : 0.0;
+      r[j] = bv[j];
+      x[j] = (act[j] && P.x0) ? sx0[row0 + j] : 0.0;
+    }
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      uint32_t w[16];
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const int k = P.c2s[c];
+        const double v = (act[j] && k >= 0) ? sval[(long long)k * n + row0 + j] : 0.0;
+        w[2 * c] = static_cast<uint32_t>(__double2loint(v));
+        w[2 * c + 1] = static_cast<uint32_t>(__double2hiint(v));
+      }
+      tmem_st16(tlane + 16 * j, w);
+    }
+    tmem_wait_st();
+    __syncthreads();  // every thread is done with the staging buffers
+    if (tid == 32) {
+      const long long nxt = static_cast<long long>(atomicAdd(ctr, 1ull));
+      *s_next = nxt;
+      if (nxt < batch) {
+        fence_proxy_async_smem();  // generic reads above before the async-proxy writes
+        issue(nxt);
+      }
+    }
+    auto spmv = [&](const double(&own)[R], double(&y)[R]) {
+      line_spmv<NX, NT, R, G>(tlane, comm.gq, a0, own, y);
+    };
+    bicgstab_core<R, NT, true, 3>(P, cur, x, r, d, act, bv, comm, spmv);
+    cur = *s_next;  // written before the core's first barrier
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s), "n"(128));
+  if (tid == 0) {
+    __threadfence();
+    const unsigned long long done = atomicAdd(ctr + 1, 1ull);
+    if (done == gridDim.x - 1) {
+      atomicExch(ctr, 0ull);
+      atomicExch(ctr + 1, 0ull);
+    }
+  }
+}
+
 }  // namespace bsolve

@@ -63,5 +63,6 @@ const CVariant *variants_cluster(int *count);
 const CVariant *variants_cluster_tmem(int *count);
 const TVariant *variants_tmem(int *count);
 persist_fn variant_tmem_persist();
+persist_fn variant_line_persist(int nx, int *smem_bytes, int smem_vals, int n_pad);
 const LVariant *variants_line(int *count);
 const BVariant *variants_banded(int *count);
