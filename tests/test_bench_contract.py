@@ -36,3 +36,14 @@ def test_reference_arm_nonzero_rank_is_silent():
     lines = run(["--impl", "reference", "--steps", "1", "--warmup", "0", "--batch", "64"],
                 env={"RANK": "1", "WORLD_SIZE": "2", "LOCAL_RANK": "1"})
     assert lines == []
+
+
+def test_reference_arm_banded_solver():
+    """--solver banded --impl reference times the oracle's banded LU (the
+    dgbsv analogue's CPU reference) with the same contract keys."""
+    lines = run(["--impl", "reference", "--solver", "banded", "--steps", "1", "--warmup", "1",
+                 "--batch", "200", "--cpu-seconds", "0.3"])
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["value"] > 0
+    assert d["config"]["solver"].startswith("banded") and "banded LU" in d["note"]
