@@ -80,7 +80,7 @@ struct Geo {
   static constexpr int NTF = ((W + 2 + 31) / 32) * 32;  // factor warps: + RHS thread + >= 1 loader
   static constexpr int NT = NTF + 32;                    // + the back-substitution warp
   static constexpr int D = R - 2 < 4 ? R - 2 : 4;      // row prefetch distance (steps)
-  static constexpr int RB = W + 1;            // row ring stride (doubles)
+  static constexpr int RB = W + 2;            // row ring stride: W columns, b, a dummy slot
   static constexpr int smem_bytes = R * RB * 8;
   static_assert(D >= 1, "KL must be >= 2");
 };
@@ -319,7 +319,8 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
       }
       pk = load_pk(P, KL + 1 + D, lidx);
     }
-    int pos = owns ? (t == W ? W : t) : -1;  // column j + pos (RHS: W)
+    int pos = owns ? (t == W ? W : t) : -1;  // column j + pos (RHS: W; loaders -1)
+    const int rcol = owns ? t : W + 1;       // ring column read (loaders: dummy slot)
     int jr = 0;                              // j mod R: ring slot of row j+KL+1
     double *Urow = U;                        // row j of U
     // v[k] holds window row j+k of the thread's column; the update writes row
@@ -361,7 +362,7 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
         cp_wait<D>();
       }
       bar_factor(NTF);
-      if (owns) {
+      {  // every factor thread (loader lanes hold zeros and use the dummy slot)
         const int p = s_p[jb];
         const double rp = s_rp[jb];
         if (p != 0) {  // row swap j <-> j+p (uniform branch)
@@ -374,8 +375,9 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
           v[0] = bsel;
         }
         const double uc = v[0];
-        if (pos == W) Y[j] = uc;
-        else if (pos != 0 && pos < n - j) Urow[pos] = uc;  // u_jc, c = j + pos
+        // u_jc (c = j + pos) or y_j: one predicated store, no branch
+        double *dst = pos == W ? Y + j : Urow + pos;
+        if (pos == W || (pos >= 1 && pos < n - j)) *dst = uc;
         // the pivot thread's column equals the published one, so w = 1 turns
         // its registers into exact zeros: it takes column j + W next
         const double w = pos == 0 ? 1.0 : uc * rp;
@@ -389,9 +391,9 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
           if ((kk - 1) % 12 == 10) asm volatile("" ::: "memory");
         }
         // row j leaves; row j+KL+1 (ring slot j mod R) enters as window row KL
-        v[KL] = ring[jr * RB + t];
-        ring[jr * RB + t] = 0.0;
-        if (t < W) pos = pos == 0 ? W - 1 : pos - 1;
+        v[KL] = ring[jr * RB + rcol];
+        ring[jr * RB + rcol] = 0.0;
+        pos = t < W ? (pos == 0 ? W - 1 : pos - 1) : pos;
       }
       jr = (jr + 1 == R) ? 0 : jr + 1;
       Urow += W;
