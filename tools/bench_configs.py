@@ -76,7 +76,9 @@ def c0(out):
     S, v, b = solver_inputs(B)
     o = S.alloc_outputs()
     ms, _ = timed(lambda: S.run(v, b, out=o), reps=20, warm=5)
+    msb, _ = timed(lambda: S.banded_solve(v, b), reps=20, warm=5)
     emit({"config": "c0 pair (batch 2)", "us_per_batch": ms * 1e3,
+          "us_per_batch_banded_lu": msb * 1e3,
           "iters": o[1].cpu().tolist(), "plan": S.info}, out)
 
 
@@ -88,6 +90,7 @@ def c1(out, batch=1280):
         S, v, b = solver_inputs(B)
         o = S.alloc_outputs()
         ms0, _ = timed(lambda: S.run(v, b, out=o))
+        msb, _ = timed(lambda: S.banded_solve(v, b))
         it0 = o[1].cpu().numpy()
         if xprev is None:
             msw, itw = ms0, it0
@@ -101,7 +104,7 @@ def c1(out, batch=1280):
         tot_zero += ms0
         tot_warm += msw
         emit({"config": f"c1 picard p={pcd} (batch {batch})", "ms_zero_guess": ms0,
-              "ms_warm_start": msw, "sys_per_s_warm": batch / (msw * 1e-3),
+              "ms_warm_start": msw, "ms_banded_lu": msb, "sys_per_s_warm": batch / (msw * 1e-3),
               "iters_zero": {"ion": float(it0[0::2].mean()), "electron": float(it0[1::2].mean())},
               "iters_warm": {"ion": float(itw[0::2].mean()), "electron": float(itw[1::2].mean())},
               "paper_table3": {"ion": [5, 4, 3, 2, 2][pcd], "electron": [30, 28, 20, 16, 12][pcd]}},
@@ -116,8 +119,8 @@ def c2(out, exps=(10, 12, 14, 16, 17)):
     for e in exps:
         batch = 1 << e
         B = X.make_batch(0, batch, pattern=pat)
-        for fmt in ("ell", "csr"):
-            for placement in ("smem", "stream"):
+        for fmt, placements in (("ell", ("auto", "smem", "stream")), ("csr", ("smem", "stream"))):
+            for placement in placements:
                 S, v, b = solver_inputs(B, fmt=fmt, placement=placement)
                 o = S.alloc_outputs()
                 ms, _ = timed(lambda: S.run(v, b, out=o), reps=3, warm=1)
@@ -127,6 +130,11 @@ def c2(out, exps=(10, 12, 14, 16, 17)):
                       "us_per_system": ms * 1e3 / batch, "iters_mean": float(its.mean()),
                       "kernel_mode": S.info["kernel_mode"],
                       "block_threads": S.info["block_threads"]}, out)
+                if placement == "auto":
+                    msb, _ = timed(lambda: S.banded_solve(v, b), reps=3, warm=1)
+                    emit({"config": "c2 sweep", "batch": batch, "format": fmt,
+                          "placement": "banded LU", "ms": msb, "sys_per_s": batch / (msb * 1e-3)},
+                         out)
                 del S, v, o
         del B
         torch.cuda.empty_cache()
