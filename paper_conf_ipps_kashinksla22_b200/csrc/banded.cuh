@@ -115,20 +115,21 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
                    saddr(bar))
                : "memory");
 }
-// try_wait with a back-off: the back-substitution warp waits most of the
-// time (the factorisation is the long pole) and must not steal issue slots
+// try_wait with a suspend-time hint: the back-substitution warp waits most
+// of the time (the factorisation is the long pole); the hint lets the
+// hardware park the warp until the phase flips instead of spinning on issue
+// slots the factor warps need (a __nanosleep back-off still woke ~20 times
+// per elimination step)
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
   uint32_t ok;
-  for (;;) {
+  do {
     asm volatile(
-        "{\n.reg .pred p;\nmbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
+        "{\n.reg .pred p;\nmbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2, %3;\n"
         "selp.u32 %0, 1, 0, p;\n}"
         : "=r"(ok)
-        : "r"(saddr(bar)), "r"(parity)
+        : "r"(saddr(bar)), "r"(parity), "r"(1000000u)
         : "memory");
-    if (ok) return;
-    __nanosleep(1000);
-  }
+  } while (!ok);
 }
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
   asm volatile(
