@@ -160,51 +160,17 @@ __device__ __forceinline__ int argmax_abs(const double (&a)[N]) {
   return bi[0];
 }
 
-template <int KL, int KU, int MINB>
-__global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const BandParams P) {
-  using G = Geo<KL, KU>;
-  constexpr int R = G::R, W = G::W, NTF = G::NTF, D = G::D, RB = G::RB;
-  constexpr int NA = (W + 31) / 32;  // back substitution: accumulators per lane
-  extern __shared__ __align__(16) double ring[];  // [R][RB]
-  constexpr int RP = (R + 1) & ~1;
-  __shared__ __align__(16) double colbuf[2][RP];  // pivot column rows 1..KL (index k-1)
-  __shared__ double s_rp[2];
-  __shared__ int s_p[2];
-  __shared__ int s_info;
-  // workspace hand-off factor warps -> back-substitution warp (2 buffers)
-  __shared__ __align__(8) uint64_t full_bar[2], empty_bar[2];
-  __shared__ int s_info_buf[2];  // info of the system in workspace buffer b
-
-  const int t = threadIdx.x;
+// Back substitution of one system by one warp (dgbtrs U part, column order):
+// lane l holds the accumulators of rows r0 - 32m (m < NA), r0 = the largest
+// row <= j with r0 = l (mod 32).  Step j: the owner lane (l = j mod 32) forms
+// x_j = y_j * (1/u_jj) and broadcasts it by shuffle; every other row i in
+// the band gets y_i -= u_ij x_j.  u_ij is read from the row-major U
+// (L1-cached: each lane walks its rows backwards), PF steps ahead.
+template <int W>
+__device__ __forceinline__ void backsub_system(const BandParams &P, const double *U,
+                                               long long sys, int l, bool skip) {
+  constexpr int NA = (W + 31) / 32;
   const int n = P.n;
-  const size_t ws_sys = (size_t)n * W + n;  // U [n][W] then y [n]
-  double *ws = P.ws + (size_t)blockIdx.x * 2 * ws_sys;
-
-  if (t == 0) {
-    for (int i = 0; i < 2; ++i) {
-      mbar_init1(&full_bar[i]);
-      mbar_init1(&empty_bar[i]);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  for (int i = t; i < R * RB; i += G::NT) ring[i] = 0.0;
-  __syncthreads();
-
-  if (t >= NTF) {
-    // ======== back-substitution warp (dgbtrs U part, column order) =========
-    // lane l holds the accumulators of rows r0 - 32m (m < NA), r0 = the
-    // largest row <= j with r0 = l (mod 32).  Step j: the owner lane
-    // (l = j mod 32) forms x_j = y_j * (1/u_jj) and broadcasts it by shuffle;
-    // every other row i in the band gets y_i -= u_ij x_j.  u_ij is read from
-    // the row-major U (L1-cached: each lane walks its rows backwards).
-    const int l = t - NTF;
-    int k = 0;
-    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
-      if (P.only && P.only[sys] == 0) continue;  // converged iteratively (same test as below)
-      const int b = k & 1;
-      mbar_wait_sleep(&full_bar[b], (k >> 1) & 1);
-      const bool skip = P.only && s_info_buf[b] != 0;  // singular: keep the iterative result
-      const double *U = ws + b * ws_sys;
       const double *Y = U + (size_t)n * W;
       constexpr int PF = 8;  // U entries are loaded PF steps ahead
       double a[NA], q[PF][NA];
@@ -253,9 +219,15 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
           }
         }
       }
-      __syncwarp();
-      if (l == 0) mbar_arrive1(&empty_bar[b]);  // buffer b may be overwritten
-      if (P.only && !skip) {
+  __syncwarp();
+}
+
+// Fallback mode: true residual ||b - A x||_2 of the direct solution, status
+// DIRECT (one warp; x re-read from L2).
+__device__ __forceinline__ void fallback_residual(const BandParams &P, long long sys, int l) {
+  const int n = P.n;
+  double *xs = P.x + sys * n;
+      {
         // true residual ||b - A x||_2 of the direct solution (plain sum of
         // squares per lane, then a butterfly), x re-read from L2
         const double *val = P.values + sys * P.sys_stride;
@@ -276,6 +248,59 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
           P.only[sys] = 3;  // BSOLVE_SYS_DIRECT
         }
       }
+}
+
+// SPLIT = false: factor warps + the back-substitution warp in one kernel
+// (per-CTA double-buffered workspace, mbarrier hand-off).  SPLIT = true: the
+// factor warps only (NTF threads: more CTAs per SM); U and y of system i go to
+// workspace slot i and banded_backsub_kernel finishes the systems afterwards.
+template <int KL, int KU, int MINB, bool SPLIT = false>
+__global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MINB)
+    banded_lu_kernel(const BandParams P) {
+  using G = Geo<KL, KU>;
+  constexpr int R = G::R, W = G::W, NTF = G::NTF, D = G::D, RB = G::RB;
+  extern __shared__ __align__(16) double ring[];  // [R][RB]
+  constexpr int RP = (R + 1) & ~1;
+  __shared__ __align__(16) double colbuf[2][RP];  // pivot column rows 1..KL (index k-1)
+  __shared__ double s_rp[2];
+  __shared__ int s_p[2];
+  __shared__ int s_info;
+  // workspace hand-off factor warps -> back-substitution warp (2 buffers)
+  __shared__ __align__(8) uint64_t full_bar[2], empty_bar[2];
+  __shared__ int s_info_buf[2];  // info of the system in workspace buffer b
+
+  const int t = threadIdx.x;
+  const int n = P.n;
+  const size_t ws_sys = (size_t)n * W + n;  // U [n][W] then y [n]
+  double *ws = P.ws + (SPLIT ? 0 : (size_t)blockIdx.x * 2 * ws_sys);
+
+  if (!SPLIT && t == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init1(&full_bar[i]);
+      mbar_init1(&empty_bar[i]);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  for (int i = t; i < R * RB; i += (SPLIT ? NTF : G::NT)) ring[i] = 0.0;
+  __syncthreads();
+
+  if (!SPLIT && t >= NTF) {
+    // ======== back-substitution warp (dgbtrs U part, column order) =========
+    // lane l holds the accumulators of rows r0 - 32m (m < NA), r0 = the
+    // largest row <= j with r0 = l (mod 32).  Step j: the owner lane
+    // (l = j mod 32) forms x_j = y_j * (1/u_jj) and broadcasts it by shuffle;
+    // every other row i in the band gets y_i -= u_ij x_j.  u_ij is read from
+    // the row-major U (L1-cached: each lane walks its rows backwards).
+    const int l = t - NTF;
+    int k = 0;
+    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+      if (P.only && P.only[sys] == 0) continue;  // converged iteratively (same test as below)
+      const int b = k & 1;
+      mbar_wait_sleep(&full_bar[b], (k >> 1) & 1);
+      const bool skip = P.only && s_info_buf[b] != 0;  // singular: keep the iterative result
+      backsub_system<W>(P, ws + b * ws_sys, sys, l, skip);
+      if (l == 0) mbar_arrive1(&empty_bar[b]);  // buffer b may be overwritten
+      if (P.only && !skip) fallback_residual(P, sys, l);
       ++k;
     }
     return;
@@ -289,8 +314,8 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
   for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
     if (P.only && P.only[sys] == 0) continue;  // converged iteratively
     const int b = k & 1;
-    if (k >= 2) mbar_wait(&empty_bar[b], ((k >> 1) - 1) & 1);  // back substitution k-2 done
-    double *U = ws + b * ws_sys;
+    if (!SPLIT && k >= 2) mbar_wait(&empty_bar[b], ((k >> 1) - 1) & 1);  // back subst. k-2 done
+    double *U = SPLIT ? ws + (size_t)sys * ws_sys : ws + b * ws_sys;
     double *Y = U + (size_t)n * W;
     const double *val = P.values + sys * P.sys_stride;
     const double *bb = P.b + sys * n;
@@ -403,12 +428,87 @@ __global__ void __launch_bounds__(Geo<KL, KU>::NT, MINB) banded_lu_kernel(const 
     bar_factor(NTF);  // every U / y store of this system issued; s_info final
     if (t == 0) {
       if (P.info) P.info[sys] = s_info;
-      s_info_buf[b] = s_info;
-      __threadfence_block();
-      mbar_arrive1(&full_bar[b]);  // release: U, y of buffer b are complete
+      if (!SPLIT) {
+        s_info_buf[b] = s_info;
+        __threadfence_block();
+        mbar_arrive1(&full_bar[b]);  // release: U, y of buffer b are complete
+      }
     }
     ++k;
   }
 }
 
+// Split mode, second launch: one warp per system, ROW-oriented back
+// substitution on the row-major U that the factor kernel wrote with
+// coalesced stores:  x_j = (y_j - sum_d u_j,j+d x_j+d) / u_jj, the sum split
+// over the lanes (d = l, l+32, l+64 ..) and closed by a butterfly; each step
+// reads one contiguous U row (prefetched PF steps ahead).  x is kept in a
+// per-warp SMEM array (zero beyond n).  Many warps per SM hide the per-step
+// reduction latency; P.info holds the factorisation's info (fallback mode:
+// singular systems keep their iterative result).
+template <int KL, int KU>
+__global__ void __launch_bounds__(128) banded_backsub_kernel(const BandParams P) {
+  constexpr int W = Geo<KL, KU>::W;
+  constexpr int NA = (W + 31) / 32;
+  constexpr int PF = 8;
+  extern __shared__ __align__(16) double xsm[];  // [4 warps][n + W]
+  const int l = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  const int n = P.n;
+  double *xw = xsm + (size_t)wi * (n + W);
+  const size_t ws_sys = (size_t)n * W + n;
+  const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
+  for (long long sys = (long long)blockIdx.x * (blockDim.x >> 5) + wi; sys < P.batch; sys += nw) {
+    if (P.only && (P.only[sys] == 0 || P.info[sys] != 0)) continue;  // converged / singular
+    const double *U = P.ws + (size_t)sys * ws_sys;
+    const double *Y = U + (size_t)n * W;
+    for (int i = l; i < W; i += 32) xw[n + i] = 0.0;  // x beyond n is zero
+    __syncwarp();
+    auto uload = [&](int jj, int m) -> double {  // u_jj,jj+d, d = l + 32 m (d = 0: 1/u_jj)
+      const int d = l + 32 * m;
+      return (jj >= 0 && d < W) ? U[(size_t)jj * W + d] : 0.0;
+    };
+    double q[PF][NA], yq[PF];
+#pragma unroll
+    for (int s = 0; s < PF; ++s) {
+#pragma unroll
+      for (int m = 0; m < NA; ++m) q[s][m] = uload(n - 1 - s, m);
+      yq[s] = n - 1 - s >= 0 ? Y[n - 1 - s] : 0.0;
+    }
+    double *xs = P.x + sys * n;
+#pragma unroll 1
+    for (int jb0 = n - 1; jb0 >= 0; jb0 -= PF) {
+#pragma unroll
+      for (int s = 0; s < PF; ++s) {
+        const int j = jb0 - s;
+        double u[NA];
+#pragma unroll
+        for (int m = 0; m < NA; ++m) {
+          u[m] = q[s][m];
+          q[s][m] = uload(j - PF, m);
+        }
+        const double yj = yq[s];
+        yq[s] = j - PF >= 0 ? Y[j - PF] : 0.0;
+        if (j >= 0) {  // uniform
+          double part = 0.0;
+#pragma unroll
+          for (int m = 0; m < NA; ++m) {
+            const int d = l + 32 * m;
+            if (d >= 1 && d < W) part = fma(u[m], xw[j + d], part);
+          }
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+          const double rp = __shfl_sync(0xffffffffu, u[0], 0);  // lane 0 holds d = 0
+          const double xj = (yj - part) * rp;
+          if (l == 0) {
+            xw[j] = xj;
+            xs[j] = xj;
+          }
+          __syncwarp();
+        }
+      }
+    }
+    if (P.only) fallback_residual(P, sys, l);
+    __syncwarp();
+  }
+}
 }  // namespace bband

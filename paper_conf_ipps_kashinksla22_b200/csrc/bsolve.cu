@@ -117,6 +117,8 @@ struct bsolve_plan {
   int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
   int bnd_w = 0;              // window width the table's ring positions use
   int direct_fallback = 0;    // bsolve_options.direct_fallback
+  int32_t *d_binfo = nullptr; // split banded solve in fallback mode: per-chunk info
+  long long binfo_len = 0;
   double *d_bws = nullptr;    // per-CTA U + y workspace
   size_t bws_bytes = 0;
 };
@@ -148,6 +150,7 @@ static void free_plan(bsolve_plan *h) {
   cudaFree(h->d_ctr);
   cudaFree(h->d_bnd);
   cudaFree(h->d_bws);
+  cudaFree(h->d_binfo);
   for (int s = 0; s < bsolve_plan::kSlots; ++s) {
     if (h->hs[s]) cudaStreamDestroy(h->hs[s]);
     cudaFree(h->h_val[s]);
@@ -1101,25 +1104,6 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
       return fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed");
     h->bnd_w = Wb;
   }
-  if (bv->smem_bytes > 48 * 1024)
-    CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  bv->smem_bytes));
-  int occ = 0;
-  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)bv->fn, bv->nt,
-                                                         bv->smem_bytes));
-  if (occ < 1) return fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident");
-  const int grid = (int)std::min<long long>((long long)occ * h->num_sms, count);
-  const size_t need = sizeof(double) * (size_t)grid * 2 * ((size_t)n * Wb + n);  // 2 buffers / CTA
-  if (h->bws_bytes < need) {
-    cudaFree(h->d_bws);
-    h->d_bws = nullptr;
-    h->bws_bytes = 0;
-    if (cudaMalloc(&h->d_bws, need) != cudaSuccess) {
-      cudaGetLastError();
-      return fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need);
-    }
-    h->bws_bytes = need;
-  }
   bband::BandParams P;
   P.values = values;
   P.b = b;
@@ -1130,12 +1114,82 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
   P.ipiv = ipiv;
   P.only = only;
   P.resnorm = resnorm;
-  P.ws = h->d_bws;
   P.sys_stride = h->sys_stride;
   P.E = W;
   P.n = n;
-  P.batch = count;
-  bv->fn<<<grid, bv->nt, bv->smem_bytes, stream>>>(P);
+  const size_t ws_sys = (size_t)n * Wb + n;  // doubles of U + y per system
+  // Split mode (default; BSOLVE_BANDED_SPLIT=0 selects the fused kernel):
+  // factor-only CTAs (more per SM) write U, y per system into a chunk
+  // workspace, then one warp per system back-substitutes; chunks of systems
+  // keep the workspace bounded.
+  const char *senv = getenv("BSOLVE_BANDED_SPLIT");
+  const bool split = !(senv && atoi(senv) == 0);
+  banded_fn fact = split ? bv->fn_split : bv->fn;
+  const int nt = split ? bv->nt_split : bv->nt;
+  if (bv->smem_bytes > 48 * 1024)
+    CUDA_TRY(cudaFuncSetAttribute((const void *)fact, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  bv->smem_bytes));
+  int occ = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)fact, nt,
+                                                         bv->smem_bytes));
+  if (occ < 1) return fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident");
+  const long long resident = (long long)occ * h->num_sms;
+  long long chunk = count;
+  size_t need;
+  if (split) {
+    // at most ~8 GB of workspace, at least one full wave of CTAs
+    chunk = std::max<long long>(resident, (long long)((8ull << 30) / (8 * ws_sys)));
+    chunk = std::min<long long>(chunk, count);
+    need = sizeof(double) * (size_t)chunk * ws_sys;
+  } else {
+    need = sizeof(double) * (size_t)std::min<long long>(resident, count) * 2 * ws_sys;
+  }
+  if (h->bws_bytes < need) {
+    cudaFree(h->d_bws);
+    h->d_bws = nullptr;
+    h->bws_bytes = 0;
+    if (cudaMalloc(&h->d_bws, need) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need);
+    }
+    h->bws_bytes = need;
+  }
+  P.ws = h->d_bws;
+  if (split && only && !info) {  // fallback mode: the back substitution needs info
+    if (h->binfo_len < chunk) {
+      cudaFree(h->d_binfo);
+      h->d_binfo = nullptr;
+      h->binfo_len = 0;
+      if (cudaMalloc(&h->d_binfo, sizeof(int32_t) * chunk) != cudaSuccess)
+        return fail(BSOLVE_ERR_NOMEM, "banded solver: info buffer allocation failed");
+      h->binfo_len = chunk;
+    }
+  }
+  if (!split) {
+    P.batch = count;
+    const int grid = (int)std::min<long long>(resident, count);
+    fact<<<grid, nt, bv->smem_bytes, stream>>>(P);
+  } else {
+    for (long long c0 = 0; c0 < count; c0 += chunk) {
+      const long long cnt = std::min<long long>(chunk, count - c0);
+      bband::BandParams Q = P;
+      Q.values = values + c0 * h->sys_stride;
+      Q.b = b + c0 * n;
+      Q.x = x + c0 * n;
+      Q.info = info ? info + c0 : (only ? h->d_binfo : nullptr);
+      Q.ipiv = ipiv ? ipiv + c0 * n : nullptr;
+      Q.only = only ? only + c0 : nullptr;
+      Q.resnorm = resnorm ? resnorm + c0 : nullptr;
+      Q.batch = cnt;
+      fact<<<(int)std::min<long long>(resident, cnt), nt, bv->smem_bytes, stream>>>(Q);
+      const int gb = (int)std::min<long long>((cnt + 3) / 4, (long long)h->num_sms * 16);
+      const int sbs = 4 * (n + Wb) * (int)sizeof(double);  // per-warp x arrays
+      if (sbs > 48 * 1024)
+        CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn_backsub,
+                                      cudaFuncAttributeMaxDynamicSharedMemorySize, sbs));
+      bv->fn_backsub<<<gb, 128, sbs, stream>>>(Q);
+    }
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "banded launch: %s", cudaGetErrorString(e));
   return BSOLVE_OK;

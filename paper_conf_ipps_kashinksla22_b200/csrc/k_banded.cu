@@ -9,10 +9,13 @@
 
 using namespace bband;
 
-#define BV_(K, MINB)                                                              \
+#define BV_(K, MINB, MINB_SPLIT)                                                  \
   {K, Geo<K, K>::NT, Geo<K, K>::NTF - Geo<K, K>::W - 1, Geo<K, K>::smem_bytes,    \
-   (banded_fn)banded_lu_kernel<K, K, MINB>}
-static const BVariant kBVariants[] = {BV_(4, 8), BV_(8, 8), BV_(16, 5), BV_(33, 5), BV_(65, 1)};
+   (banded_fn)banded_lu_kernel<K, K, MINB>, Geo<K, K>::NTF,                       \
+   (banded_fn)banded_lu_kernel<K, K, MINB_SPLIT, true>,                          \
+   (banded_fn)banded_backsub_kernel<K, K>}
+static const BVariant kBVariants[] = {BV_(4, 8, 8), BV_(8, 8, 8), BV_(16, 5, 8),
+                                      BV_(33, 5, 8), BV_(65, 1, 1)};
 
 const BVariant *variants_banded(int *count) {
   *count = (int)(sizeof(kBVariants) / sizeof(kBVariants[0]));

@@ -54,7 +54,10 @@ struct BVariant {
   int nt;          // threads per CTA
   int max_entries; // loader lanes: rows with at most this many entries - 1
   int smem_bytes;  // dynamic SMEM (row ring)
-  banded_fn fn;
+  banded_fn fn;    // factor + back-substitution warps in one kernel
+  int nt_split;    // split mode: factor-only CTA size
+  banded_fn fn_split;    // split mode: factorisation (U, y to a per-system workspace)
+  banded_fn fn_backsub;  // split mode: one warp per system back substitution
 };
 
 const Variant *variants_generic(int *count);
