@@ -1138,7 +1138,8 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
   size_t need;
   if (split) {
     // at most ~8 GB of workspace, at least one full wave of CTAs
-    chunk = std::max<long long>(resident, (long long)((8ull << 30) / (8 * ws_sys)));
+    // (a whole number of resident-CTA waves: no partial last wave per chunk)
+    chunk = std::max<long long>(1, (long long)((8ull << 30) / (8 * ws_sys)) / resident) * resident;
     chunk = std::min<long long>(chunk, count);
     need = sizeof(double) * (size_t)chunk * ws_sys;
   } else {
