@@ -598,7 +598,7 @@ def run_banded(args, rank, world, local_rank):
     roof = {"bound": "alu", "achieved": flops_sys * per_rank / kern_s / 1e12,
             "peak": fp64_peak / 1e12, "unit": "TFLOP/s",
             "frac": flops_sys * per_rank / kern_s / fp64_peak, "traffic": None,
-            "kernel": f"banded_lu_kernel<{kb},{kb}> (one launch per step)",
+            "kernel": f"banded_lu_kernel<{kb},{kb},.,true> + banded_backsub_kernel (per chunk)",
             "algorithmic_flops_per_unit": flops_sys, "units_per_launch": per_rank,
             "peak_source": "derived: 64 DFMA/clk/SM x 148 SMs x 1965 MHz (FP64 pipe)",
             "kernel_ms_avg": kern_s * 1e3,
@@ -609,6 +609,7 @@ def run_banded(args, rank, world, local_rank):
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic_banded.json")))
         roof["hbm"]["traffic"] = tr["dram_bytes_per_launch"] * per_rank / tr["systems_per_launch"]
+        roof["hbm"]["traffic_note"] = tr.get("note", "")
         roof["traffic_source"] = tr["source"]
     except Exception:  # noqa: BLE001
         pass
@@ -653,8 +654,11 @@ def run_banded(args, rank, world, local_rank):
         "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
         "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": config_dict(args, world, per_rank), "roofline": roof, "cpu_baseline": cpu,
-        "e2e": e2e, "clocks": clk.summary(), "gpu_launches": args.steps,
-        "plan": {"kb": kb, "window": Wb, "kl": kl, "ku": ku},
+        "e2e": e2e, "clocks": clk.summary(),
+        "gpu_launches": args.steps * S.query()["banded_launches"],
+        "plan": {"kb": kb, "window": Wb, "kl": kl, "ku": ku,
+                 "launches_per_step": S.query()["banded_launches"],
+                 "mode": "split: factor kernel + back-substitution kernel per chunk of systems"},
         "solve_stats": {"info_nonzero": int((info_h != 0).sum())}, "parity_sample": parity,
         "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms)},
     }

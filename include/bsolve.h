@@ -170,6 +170,9 @@ typedef struct bsolve_info {
                               consecutive grid rows (DESIGN.md Kernels 10)   */
   int cluster;             /* CTAs per system (PLACE_CLUSTER), else 0        */
   int solver, precond, restart; /* resolved BSOLVE_SOLVER_*, BSOLVE_PREC_*, m  */
+  int banded_launches;     /* kernel launches of the last bsolve_banded_solve
+                              (or direct-fallback) call: 2 per system chunk in
+                              the split mode, 1 fused; 0 before the first   */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

@@ -39,6 +39,10 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+#ifndef BBAND_LDS64
+#define BBAND_LDS64 0  // 1: 8-byte multiplier loads (same SMEM wavefronts, measured 0.895 vs 0.903)
+#endif
+
 namespace bband {
 
 struct BandParams {
@@ -407,6 +411,16 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
         // the pivot thread's column equals the published one, so w = 1 turns
         // its registers into exact zeros: it takes column j + W next
         const double w = pos == 0 ? 1.0 : uc * rp;
+#if BBAND_LDS64
+        // 8-byte broadcast loads of the multipliers: one SMEM wavefront each
+        // (a 16-byte broadcast load costs as many wavefronts as a full one)
+        const double *cb = colbuf[jb];
+#pragma unroll
+        for (int kk = 1; kk < R; ++kk) {
+          v[kk - 1] = fma(-cb[kk - 1], w, v[kk]);
+          if ((kk - 1) % 12 == 11) asm volatile("" ::: "memory");
+        }
+#else
         const double2 *cb = reinterpret_cast<const double2 *>(colbuf[jb]);
 #pragma unroll
         for (int kk = 1; kk < R; kk += 2) {
@@ -416,6 +430,7 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
           // keep at most 6 multiplier pairs in flight (register pressure)
           if ((kk - 1) % 12 == 10) asm volatile("" ::: "memory");
         }
+#endif
         // row j leaves; row j+KL+1 (ring slot j mod R) enters as window row KL
         v[KL] = ring[jr * RB + rcol];
         ring[jr * RB + rcol] = 0.0;

@@ -117,6 +117,7 @@ struct bsolve_plan {
   int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
   int bnd_w = 0;              // window width the table's ring positions use
   int direct_fallback = 0;    // bsolve_options.direct_fallback
+  int banded_launches = 0;    // kernel launches of the last banded call
   int32_t *d_binfo = nullptr; // split banded solve in fallback mode: per-chunk info
   long long binfo_len = 0;
   double *d_bws = nullptr;    // per-CTA U + y workspace
@@ -806,6 +807,7 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->solver = h->solver;
   info->precond = h->precond;
   info->restart = h->restart;
+  info->banded_launches = h->banded_launches;
   return BSOLVE_OK;
 }
 
@@ -1166,6 +1168,7 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
       h->binfo_len = chunk;
     }
   }
+  h->banded_launches = split ? (int)(2 * ((count + chunk - 1) / chunk)) : 1;
   if (!split) {
     P.batch = count;
     const int grid = (int)std::min<long long>(resident, count);
