@@ -355,6 +355,19 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->kl = std::max(h->kl, i - col_idx[e]);
       h->ku = std::max(h->ku, col_idx[e] - i);
     }
+  if (h->direct_fallback) {  // the banded kernels must cover the pattern (fail early)
+    int cnt = 0;
+    const BVariant *tab = variants_banded(&cnt);
+    bool ok = false;
+    for (int i = 0; i < cnt; ++i)
+      ok = ok || (tab[i].kb >= std::max(h->kl, h->ku) && tab[i].max_entries > W);
+    if (!ok) {
+      const int kl = h->kl, ku = h->ku;
+      delete h;
+      return fail(BSOLVE_ERR_UNSUPPORTED,
+                  "direct_fallback: bandwidth kl = %d, ku = %d exceeds the banded solver", kl, ku);
+    }
+  }
   // ELL slot map (conflict-free gathers, see build_ell_map)
   std::vector<int32_t> ell_diag;
   build_ell_map(n, row_ptr, col_idx, W, h->h_ell_col, h->h_csr2ell, ell_diag);

@@ -240,3 +240,22 @@ def test_direct_fallback_needs_status():
     rc = L.bsolve_run(h, d, d, None, 1e-10, 10, d, d, d, None, None)
     L.bsolve_destroy(h)
     assert rc == B.ERR_INVALID
+
+
+def test_direct_fallback_wide_band_rejected_before_cuda():
+    """direct_fallback needs a banded-kernel instance for the pattern: a band
+    wider than 65 is UNSUPPORTED at create time, before any CUDA call."""
+    n = 100
+    rp, ci = [0], []
+    for i in range(n):
+        ci += sorted({i, (i + 70) % n})
+        rp.append(len(ci))
+    rp, ci = np.array(rp, np.int32), np.array(ci, np.int32)
+    L = B.lib()
+    opt = B.Options()
+    L.bsolve_default_options(C.byref(opt))
+    opt.direct_fallback = 1
+    h = B._P()
+    assert L.bsolve_create(C.byref(h), n, 2, rp.ctypes.data, ci.ctypes.data, C.byref(opt)) == \
+        B.ERR_UNSUPPORTED
+    assert "direct_fallback" in L.bsolve_last_error().decode()

@@ -211,3 +211,18 @@ def test_direct_fallback_singular_keeps_iterative_result_and_host_path():
     assert np.all(s1[others] == 3)
     xh, ih, rh, sh = S.run_host(S.ell_values(v), b, maxiter=2)
     assert np.array_equal(sh, s1) and np.array_equal(xh, x1) and np.array_equal(rh, r1)
+
+
+def test_direct_fallback_rejects_wide_band_at_create():
+    """direct_fallback on a pattern the banded kernels cannot cover fails in
+    bsolve_create (UNSUPPORTED), not later inside bsolve_run."""
+    from paper_conf_ipps_kashinksla22_b200.bsolve import BsolveError, ERR_UNSUPPORTED
+    n = 100
+    rp, ci = [0], []
+    for i in range(n):
+        ci += sorted({i, (i + 70) % n})
+        rp.append(len(ci))
+    with pytest.raises(BsolveError) as e:
+        Solver(np.array(rp, np.int32), np.array(ci, np.int32), 2, format="csr",
+               direct_fallback=True)
+    assert e.value.code == ERR_UNSUPPORTED
