@@ -446,12 +446,43 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       const char *ctenv = getenv("BSOLVE_CLUSTER_TMEM");
       const bool ctmem = opt.reg_slots == 0 && !(ctenv && atoi(ctenv) == 0);
       h->cvar = nullptr;
-      if (ctmem) {
+      // line-tiled TMEM cluster kernel for a 2D grid of a compiled width:
+      // opt-in (BSOLVE_CLUSTER_LINE=1), measured 0.88 vs 0.92 M sys/s for the
+      // strided-row kernel at n = 4032 (its halo rows are sent by 9 threads
+      // with 8 st.async each; 255 registers with spills)
+      const char *clenv = getenv("BSOLVE_CLUSTER_LINE");
+      int line_smem = 0;
+      if (ctmem && clenv && atoi(clenv) == 1) {
+        int cnt = 0;
+        const CVariant *t = variants_cluster_line(&cnt, &line_smem);
+        for (int i = 0; i < cnt && !h->cvar; ++i) {
+          if (t[i].c != c) continue;
+          const int NX = t[i].kreg;
+          const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
+          int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
+          bool ok = true;
+          for (int k = 1; k < W && ok; ++k) {
+            bool real = false;
+            for (int rr = 0; rr < n && !real; ++rr) real = h->h_csr2ell[(size_t)k * n + rr] >= 0;
+            if (!real) continue;
+            const int o = h->doff[k] / 8;
+            int cc = 0;
+            while (cc < 8 && canon[cc] != o) ++cc;
+            if (cc == 8 || c2s[cc] >= 0) ok = false;
+            else c2s[cc] = k;
+          }
+          if (!ok) continue;
+          h->cvar = &t[i];
+          h->line_nx = NX;
+          for (int cc = 0; cc < 8; ++cc) h->c2s[cc] = c2s[cc];
+        }
+      }
+      if (ctmem && !h->cvar) {
         int cnt = 0;
         const CVariant *t = variants_cluster_tmem(&cnt);
         for (int i = 0; i < cnt; ++i)
           if (t[i].c == c) h->cvar = &t[i];
-      } else {
+      } else if (!ctmem) {
         h->cvar = find_cvariant(c, kr, 3);
       }
       if (!h->cvar)
@@ -464,7 +495,8 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->n_pad = (n + 1) & ~1;
       h->smem_vals = 9 * rpc;
       // + 4 mbarriers + the TMEM base address slot
-      h->smem_bytes = (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 5 * 8;
+      h->smem_bytes = h->line_nx ? line_smem
+                                 : (9 * rpc + rpc + 2 * h->guard) * 8 + 16 * c * 4 * 8 + 5 * 8;
       if (h->smem_bytes > smem_optin)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster plan needs %d B of SMEM",
                               h->smem_bytes));

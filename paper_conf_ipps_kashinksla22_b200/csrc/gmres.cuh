@@ -182,7 +182,7 @@ __device__ __forceinline__ void gmres_core(const SolveParams &P, long long sys, 
     }
     if (brk) { st = SYS_BREAKDOWN; break; }
     // ---- y = R^-1 g (every thread, R from SMEM); x += M^-1 V y --------------
-    comm.sync();  // thread 0's writes of R visible
+    comm.barrier();  // thread 0's writes of R visible (CTA only)
     double y[M];
 #pragma unroll
     for (int i = M - 1; i >= 0; --i) {

@@ -39,3 +39,13 @@ persist_fn variant_line_persist(int nx, int *smem_bytes, int smem_vals, int n_pa
   }
   return nullptr;
 }
+
+// line-tiled TMEM plan on a cluster of C CTAs (n > 1024), NX = 64 (63 x 64 grid)
+#define LCV_(NX, C) {C, NX, 3, (solve_fn)bicgstab_tmem_line_cluster_kernel<NX, C>}
+static const CVariant kLCVariants[] = {LCV_(64, 2), LCV_(64, 3), LCV_(64, 4), LCV_(64, 5),
+                                       LCV_(64, 6), LCV_(64, 7), LCV_(64, 8)};
+const CVariant *variants_cluster_line(int *count, int *smem_bytes) {
+  *count = (int)(sizeof(kLCVariants) / sizeof(kLCVariants[0]));
+  *smem_bytes = line_cluster_smem<64, 8>();
+  return kLCVariants;
+}

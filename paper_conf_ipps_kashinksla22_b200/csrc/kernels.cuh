@@ -367,6 +367,7 @@ struct CtaComm {
     if (act[j]) sg[threadIdx.x + j * NT] = v;
   }
   __device__ __forceinline__ void sync() { __syncthreads(); }
+  __device__ __forceinline__ void barrier() { __syncthreads(); }  // CTA only, no halo
   template <int K>
   __device__ __forceinline__ void sum(double (&v)[K]) {
     block_sum<K, NT / 32>(v, sred, buf, threadIdx.x & 31, threadIdx.x >> 5);
@@ -648,7 +649,10 @@ __device__ __forceinline__ void bicgstab_core(const SolveParams &P, long long sy
 
   if (final_res < 0.0) {
     // final TRUE residual ||b - A x|| (always reported, R4)
-    comm.sync();  // previous gather readers done before overwriting
+    // previous gather readers of this CTA done before the publish overwrites
+    // (a CTA barrier: no halo is in flight -- for the cluster plans the last
+    // reduction already ordered every CTA's previous SpMV before this point)
+    comm.barrier();
     double q[R];
     final_res = sqrt(true_residual(q));
   }
@@ -1283,6 +1287,8 @@ struct ClusterComm {
   // complete this CTA's halo mbarrier.  (Two consecutive publishes are always
   // separated by a reduction that depends on every CTA's SpMV, so a halo is
   // never overwritten while it is still being gathered.)
+  // CTA barrier without a halo exchange (no publish preceded it)
+  __device__ __forceinline__ void barrier() { __syncthreads(); }
   __device__ __forceinline__ void sync() {
     if (threadIdx.x == 0) mbar_arrive_expect_tx(hbar, static_cast<uint32_t>(halo_bytes));
     __syncthreads();

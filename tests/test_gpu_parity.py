@@ -574,3 +574,35 @@ def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
     o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
+
+
+@pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4)])
+def test_cluster_line_kernel(nx, ny, C, monkeypatch):
+    """Opt-in line-tiled TMEM cluster kernel (BSOLVE_CLUSTER_LINE=1): the
+    plane guards carry the neighbours' halo rows (st.async + mbarrier); same
+    parity bar, warm start included."""
+    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", "1")
+    B = X.make_batch(0, 12, nx=nx, ny=ny)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
+    assert g["info"]["cluster"] == C and g["info"]["kernel_mode"] == 4
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-3)
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
+
+
+@pytest.mark.parametrize("line", ["0", "1"])
+def test_cluster_maxiter_exhausted(line, monkeypatch):
+    """Cluster plans (strided and line-tiled) when maxiter runs out: the final
+    true-residual check must not wait for a halo nobody sent (regression: the
+    pre-publish barrier used the halo-waiting sync and hung)."""
+    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", line)
+    B = X.make_batch(0, 6, nx=64, ny=63)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=4)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=4)
+    assert g["info"]["cluster"] == 4
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
+    assert np.any(g["status"] == 1)
