@@ -272,6 +272,14 @@ int bsolve_ell_layout(int n, const int32_t *row_ptr, const int32_t *col_idx, int
 int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b, double *x,
                         int32_t *info, int32_t *ipiv, void *stream);
 
+/* bsolve_banded_solve with HOST buffers (values, b as for bsolve_run_host;
+ * x: batch * n doubles out; info: batch int32 out).  The batch streams through
+ * the device in chunks on the handle's 3 internal streams, copies of one chunk
+ * overlapping the solve of another (pinned memory needed for the overlap).
+ * Synchronous.  Errors as bsolve_banded_solve. */
+int bsolve_banded_solve_host(bsolve_handle h, const double *values, const double *b, double *x,
+                             int32_t *info);
+
 /* Release the handle and its device memory.  NULL-safe; returns BSOLVE_OK. */
 int bsolve_destroy(bsolve_handle h);
 

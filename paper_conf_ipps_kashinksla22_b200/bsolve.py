@@ -79,6 +79,7 @@ def lib():
             L.bsolve_query.argtypes = [_P, C.POINTER(Info)]
             L.bsolve_ell_map.argtypes = [_P, _P, _P]
             L.bsolve_banded_solve.argtypes = [_P, _P, _P, _P, _P, _P, _P]
+            L.bsolve_banded_solve_host.argtypes = [_P, _P, _P, _P, _P]
             L.bsolve_ell_layout.argtypes = [C.c_int, _P, _P, C.POINTER(C.c_int32), _P, _P]
             L.bsolve_destroy.argtypes = [_P]
             L.bsolve_last_error.argtypes = []
@@ -87,7 +88,7 @@ def lib():
                                                       C.POINTER(C.c_double)]
             for f in ("bsolve_create", "bsolve_run", "bsolve_run_host", "bsolve_spmv",
                       "bsolve_csr_to_ell", "bsolve_query", "bsolve_ell_map", "bsolve_destroy",
-                      "bsolve_ell_layout", "bsolve_banded_solve",
+                      "bsolve_ell_layout", "bsolve_banded_solve", "bsolve_banded_solve_host",
                       "bsolve_probe_smem_bandwidth"):
                 getattr(L, f).restype = C.c_int
             _lib = L
@@ -291,6 +292,19 @@ class Solver:
                                     int(maxiter), _np_ptr(x), _np_ptr(it), _np_ptr(res),
                                     _np_ptr(st)))
         return x, it, res, st
+
+    def banded_solve_host(self, values, b, out=None):
+        """Synchronous banded LU solve from HOST arrays (chunked H2D / solve /
+        D2H pipeline; pinned memory overlaps best): returns (x, info)."""
+        v = np.ascontiguousarray(values, dtype=np.float64)
+        bb = np.ascontiguousarray(b, dtype=np.float64)
+        assert v.size == self.batch * self.values_per_system and bb.size == self.batch * self.n
+        if out is None:
+            out = (np.empty((self.batch, self.n)), np.empty(self.batch, np.int32))
+        x, info = out
+        check(lib().bsolve_banded_solve_host(self._h, _np_ptr(v), _np_ptr(bb), _np_ptr(x),
+                                             _np_ptr(info)))
+        return x, info
 
 
 def _np_ptr(a):

@@ -113,6 +113,9 @@ struct bsolve_plan {
          *h_res[kSlots] = {};
   int32_t *h_it[kSlots] = {};
   int8_t *h_st[kSlots] = {};
+  double *h_bws[kSlots] = {};       // banded workspace per pipeline slot
+  size_t h_bws_bytes[kSlots] = {};
+  int32_t *h_it_b[kSlots] = {};     // banded info per pipeline slot (fallback mode)
   // banded direct solver (bsolve_banded_solve, lazily set up)
   int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
   int bnd_w = 0;              // window width the table's ring positions use
@@ -161,6 +164,8 @@ static void free_plan(bsolve_plan *h) {
     cudaFree(h->h_res[s]);
     cudaFree(h->h_it[s]);
     cudaFree(h->h_st[s]);
+    cudaFree(h->h_bws[s]);
+    cudaFree(h->h_it_b[s]);
   }
   if (cur >= 0) cudaSetDevice(cur);
   delete h;
@@ -878,11 +883,11 @@ static int check_run_args(bsolve_handle h, const double *values, const double *b
 
 static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
                          int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
-                         int8_t *only, double *resnorm);
+                         int8_t *only, double *resnorm, int slot = -1);
 
 static int launch_solve(bsolve_handle h, const double *values, const double *b, const double *x0,
                         double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
-                        int8_t *status, int count, cudaStream_t stream) {
+                        int8_t *status, int count, cudaStream_t stream, int slot = -1) {
   if (count <= 0) return BSOLVE_OK;
   SolveParams P;
   P.values = values;
@@ -945,7 +950,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));
   if (h->direct_fallback)  // non-converged systems -> banded LU
-    return launch_banded(h, values, b, x, nullptr, nullptr, count, stream, status, resnorm);
+    return launch_banded(h, values, b, x, nullptr, nullptr, count, stream, status, resnorm, slot);
   return BSOLVE_OK;
 }
 
@@ -988,6 +993,36 @@ extern "C" int bsolve_run(bsolve_handle h, const double *values, const double *b
   return rc;
 }
 
+// Lazily set up the host-buffer pipeline (bsolve_run_host,
+// bsolve_banded_solve_host): 3 non-blocking streams, each with device
+// buffers for one chunk of ~64 MB of values (whole waves of resident CTAs).
+static int ensure_host_pipeline(bsolve_handle h) {
+  if (h->h_chunk != 0) return BSOLVE_OK;
+  const int n = h->n;
+  const long long ss = h->sys_stride;
+  const long long wave = (long long)h->num_sms * h->ctas_per_sm;
+  long long c = std::max<long long>(wave, (64ll << 20) / (ss * 8));
+  c = (c + wave - 1) / wave * wave;
+  c = std::min<long long>(c, h->batch);
+  const int chunk = (int)std::max<long long>(c, 1);
+  for (int s = 0; s < bsolve_plan::kSlots; ++s) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&h->hs[s], cudaStreamNonBlocking));
+    const size_t c_ = (size_t)chunk;
+    if (cudaMalloc(&h->h_val[s], c_ * ss * 8) != cudaSuccess ||
+        cudaMalloc(&h->h_b[s], c_ * n * 8) != cudaSuccess ||
+        cudaMalloc(&h->h_x0[s], c_ * n * 8) != cudaSuccess ||
+        cudaMalloc(&h->h_x[s], c_ * n * 8) != cudaSuccess ||
+        cudaMalloc(&h->h_res[s], c_ * 8) != cudaSuccess ||
+        cudaMalloc(&h->h_it[s], c_ * 4) != cudaSuccess ||
+        cudaMalloc(&h->h_st[s], c_) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(BSOLVE_ERR_NOMEM, "device allocation for the host pipeline failed");
+    }
+  }
+  h->h_chunk = chunk;
+  return BSOLVE_OK;
+}
+
 extern "C" int bsolve_run_host(bsolve_handle h, const double *values, const double *b,
                                const double *x0, double tol, int maxiter, double *x, int32_t *iters,
                                double *resnorm, int8_t *status) {
@@ -1000,28 +1035,7 @@ extern "C" int bsolve_run_host(bsolve_handle h, const double *values, const doub
   if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
   const int n = h->n;
   const long long ss = h->sys_stride;
-  if (h->h_chunk == 0) {
-    // ~64 MB of values per chunk, rounded to whole waves of resident CTAs
-    const long long wave = (long long)h->num_sms * h->ctas_per_sm;
-    long long c = std::max<long long>(wave, (64ll << 20) / (ss * 8));
-    c = (c + wave - 1) / wave * wave;
-    c = std::min<long long>(c, h->batch);
-    h->h_chunk = (int)std::max<long long>(c, 1);
-    for (int s = 0; s < bsolve_plan::kSlots; ++s) {
-      CUDA_TRY(cudaStreamCreateWithFlags(&h->hs[s], cudaStreamNonBlocking));
-      const size_t c_ = (size_t)h->h_chunk;
-      if (cudaMalloc(&h->h_val[s], c_ * ss * 8) != cudaSuccess ||
-          cudaMalloc(&h->h_b[s], c_ * n * 8) != cudaSuccess ||
-          cudaMalloc(&h->h_x0[s], c_ * n * 8) != cudaSuccess ||
-          cudaMalloc(&h->h_x[s], c_ * n * 8) != cudaSuccess ||
-          cudaMalloc(&h->h_res[s], c_ * 8) != cudaSuccess ||
-          cudaMalloc(&h->h_it[s], c_ * 4) != cudaSuccess ||
-          cudaMalloc(&h->h_st[s], c_) != cudaSuccess) {
-        cudaGetLastError();
-        return fail(BSOLVE_ERR_NOMEM, "device allocation for the host pipeline failed");
-      }
-    }
-  }
+  if ((rc = ensure_host_pipeline(h))) return rc;
   const int C = h->h_chunk;
   int k = 0;
   for (long long s0 = 0; s0 < h->batch; s0 += C, ++k) {
@@ -1035,7 +1049,7 @@ extern "C" int bsolve_run_host(bsolve_handle h, const double *values, const doub
       CUDA_TRY(cudaMemcpyAsync(h->h_x0[sl], x0 + s0 * n, (size_t)cnt * n * 8,
                                cudaMemcpyHostToDevice, st));
     rc = launch_solve(h, h->h_val[sl], h->h_b[sl], x0 ? h->h_x0[sl] : nullptr, tol, maxiter,
-                      h->h_x[sl], h->h_it[sl], h->h_res[sl], h->h_st[sl], cnt, st);
+                      h->h_x[sl], h->h_it[sl], h->h_res[sl], h->h_st[sl], cnt, st, sl);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(x + s0 * n, h->h_x[sl], (size_t)cnt * n * 8, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(cudaMemcpyAsync(iters + s0, h->h_it[sl], (size_t)cnt * 4, cudaMemcpyDeviceToHost, st));
@@ -1116,7 +1130,7 @@ extern "C" int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, doub
 // BSOLVE_SYS_DIRECT (only and status_out are the same array).
 static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
                          int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
-                         int8_t *only, double *resnorm) {
+                         int8_t *only, double *resnorm, int slot) {
   if (count <= 0) return BSOLVE_OK;
   const int kb = std::max(h->kl, h->ku);
   int cnt = 0;
@@ -1192,17 +1206,26 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
   } else {
     need = sizeof(double) * (size_t)std::min<long long>(resident, count) * 2 * ws_sys;
   }
-  if (h->bws_bytes < need) {
-    cudaFree(h->d_bws);
-    h->d_bws = nullptr;
-    h->bws_bytes = 0;
-    if (cudaMalloc(&h->d_bws, need) != cudaSuccess) {
+  // workspace: the handle's, or host-pipeline slot `slot`'s (concurrent streams)
+  double *&wsp = slot >= 0 ? h->h_bws[slot] : h->d_bws;
+  size_t &wsb = slot >= 0 ? h->h_bws_bytes[slot] : h->bws_bytes;
+  if (wsb < need) {
+    cudaFree(wsp);
+    wsp = nullptr;
+    wsb = 0;
+    if (cudaMalloc(&wsp, need) != cudaSuccess) {
       cudaGetLastError();
       return fail(BSOLVE_ERR_NOMEM, "banded solver: %zu B workspace allocation failed", need);
     }
-    h->bws_bytes = need;
+    wsb = need;
   }
-  P.ws = h->d_bws;
+  P.ws = wsp;
+  if (split && only && !info && slot >= 0) {  // host pipeline, fallback mode: per-slot info
+    if (!h->h_it_b[slot] &&
+        cudaMalloc(&h->h_it_b[slot], sizeof(int32_t) * (size_t)h->h_chunk) != cudaSuccess)
+      return fail(BSOLVE_ERR_NOMEM, "banded solver: info buffer allocation failed");
+    info = h->h_it_b[slot];
+  }
   if (split && only && !info) {  // fallback mode: the back substitution needs info
     if (h->binfo_len < chunk) {
       cudaFree(h->d_binfo);
@@ -1263,6 +1286,40 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
                      nullptr);
   if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
   return rc;
+}
+
+extern "C" int bsolve_banded_solve_host(bsolve_handle h, const double *values, const double *b,
+                                        double *x, int32_t *info) {
+  g_err.clear();
+  if (!h) return fail(BSOLVE_ERR_INVALID, "handle is NULL");
+  if (h->batch == 0) return BSOLVE_OK;
+  if (!values || !b || !x || !info)
+    return fail(BSOLVE_ERR_INVALID, "values, b, x and info must be non-NULL");
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
+  int rc = ensure_host_pipeline(h);
+  if (rc) return rc;
+  const int n = h->n;
+  const long long ss = h->sys_stride;
+  const int C = h->h_chunk;
+  int k = 0;
+  for (long long s0 = 0; s0 < h->batch; s0 += C, ++k) {
+    const int cnt = (int)std::min<long long>(C, h->batch - s0);
+    const int sl = k % bsolve_plan::kSlots;
+    cudaStream_t st = h->hs[sl];
+    CUDA_TRY(cudaMemcpyAsync(h->h_val[sl], values + s0 * ss, (size_t)cnt * ss * 8,
+                             cudaMemcpyHostToDevice, st));
+    CUDA_TRY(cudaMemcpyAsync(h->h_b[sl], b + s0 * n, (size_t)cnt * n * 8, cudaMemcpyHostToDevice, st));
+    rc = launch_banded(h, h->h_val[sl], h->h_b[sl], h->h_x[sl], h->h_it[sl], nullptr, cnt, st,
+                       nullptr, nullptr, sl);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(x + s0 * n, h->h_x[sl], (size_t)cnt * n * 8, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaMemcpyAsync(info + s0, h->h_it[sl], (size_t)cnt * 4, cudaMemcpyDeviceToHost, st));
+  }
+  for (int s = 0; s < bsolve_plan::kSlots; ++s) CUDA_TRY(cudaStreamSynchronize(h->hs[s]));
+  if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
+  return BSOLVE_OK;
 }
 
 extern "C" int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz) {

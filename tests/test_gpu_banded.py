@@ -226,3 +226,23 @@ def test_direct_fallback_rejects_wide_band_at_create():
         Solver(np.array(rp, np.int32), np.array(ci, np.int32), 2, format="csr",
                direct_fallback=True)
     assert e.value.code == ERR_UNSUPPORTED
+
+
+def test_host_pipeline_banded_and_fallback_many_chunks():
+    """bsolve_banded_solve_host (3 streams, one workspace per pipeline slot)
+    equals the device path bit for bit over several chunks; run_host with
+    direct_fallback (banded re-solves on concurrent streams) equals run."""
+    B = X.make_batch(0, 3000)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 3000)
+    ev = S.ell_values(B.values)
+    xd, infod = S.banded_solve(to_dev(ev), to_dev(B.b))
+    xh, infoh = S.banded_solve_host(ev, B.b)
+    torch.cuda.synchronize()
+    assert np.array_equal(xh, xd.cpu().numpy()) and np.array_equal(infoh, infod.cpu().numpy())
+    F = Solver(p.row_ptr, p.col_idx, 3000, direct_fallback=True)
+    x1, it1, r1, s1 = F.run(to_dev(ev), to_dev(B.b), maxiter=6)
+    torch.cuda.synchronize()
+    x2, it2, r2, s2 = F.run_host(ev, B.b, maxiter=6)
+    assert np.any(s2 == 3) and np.array_equal(s2, s1.cpu().numpy())
+    assert np.array_equal(x2, x1.cpu().numpy()) and np.array_equal(r2, r1.cpu().numpy())
