@@ -915,6 +915,13 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   for (int c = 0; c < 8; ++c) P.c2s[c] = h->c2s[c];
   P.precond = h->precond;
   P.restart = h->restart;
+  // line plan: each CTA asks L2 for the system that will start about one
+  // residency later (CTAs dispatch in blockIdx order, 2 per SM), so its
+  // start-up loads hit L2 instead of HBM (BSOLVE_L2_PREFETCH=0 disables)
+  {
+    const char *pe = getenv("BSOLVE_L2_PREFETCH");
+    P.pf_ahead = (h->line_nx && !(pe && atoi(pe) == 0)) ? 2 * h->num_sms : 0;
+  }
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)

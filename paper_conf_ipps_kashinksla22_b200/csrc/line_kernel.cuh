@@ -186,6 +186,19 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
     const int pl = i / (L::S - NT), q = i % (L::S - NT);
     sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
   }
+  // L2 prefetch (TMA bulk prefetch) of a system that starts later
+  if (tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {
+    const long long ns = sys + P.pf_ahead;
+    const uint32_t vb = static_cast<uint32_t>(P.sys_stride * 8) & ~15u;
+    const void *va = P.values + ns * P.sys_stride;
+    const void *ba = P.b + ns * n;
+    if (((reinterpret_cast<uintptr_t>(va) | reinterpret_cast<uintptr_t>(ba)) & 15u) == 0) {
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(va), "r"(vb) : "memory");
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
+                   "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                   : "memory");
+    }
+  }
 
   // ---- this thread's rows: b, x0, diagonal and the 8 off-diagonal values ----
   bool act[R];
