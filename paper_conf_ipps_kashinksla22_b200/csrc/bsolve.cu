@@ -920,7 +920,8 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   // start-up loads hit L2 instead of HBM (BSOLVE_L2_PREFETCH=0 disables)
   {
     const char *pe = getenv("BSOLVE_L2_PREFETCH");
-    P.pf_ahead = (h->line_nx && !(pe && atoi(pe) == 0)) ? 2 * h->num_sms : 0;
+    const int k = pe ? atoi(pe) : 2;  // systems ahead, in units of #SMs
+    P.pf_ahead = (h->line_nx && k > 0) ? k * h->num_sms : 0;
   }
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
