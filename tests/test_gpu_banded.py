@@ -246,3 +246,15 @@ def test_host_pipeline_banded_and_fallback_many_chunks():
     x2, it2, r2, s2 = F.run_host(ev, B.b, maxiter=6)
     assert np.any(s2 == 3) and np.array_equal(s2, s1.cpu().numpy())
     assert np.array_equal(x2, x1.cpu().numpy()) and np.array_equal(r2, r1.cpu().numpy())
+
+
+def test_direct_fallback_with_gmres():
+    """direct_fallback also covers the GMRES(m) solver's non-converged systems."""
+    B = X.make_batch(0, 64)
+    p = B.pattern
+    _, (x0, it0, r0, s0) = _run(p, B.values, B.b, maxiter=5, solver="gmres")
+    _, (x1, it1, r1, s1) = _run(p, B.values, B.b, maxiter=5, solver="gmres", direct_fallback=True)
+    bad = s0 != 0
+    assert np.any(bad) and np.all(s1[bad] == 3) and np.array_equal(x1[~bad], x0[~bad])
+    xo, _, _ = oracle_banded(p.row_ptr, p.col_idx, B.values[bad], B.b[bad])
+    assert np.max(np.linalg.norm(x1[bad] - xo, axis=1) / np.linalg.norm(xo, axis=1)) <= 1e-12
