@@ -462,10 +462,10 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
 // reduction latency; P.info holds the factorisation's info (fallback mode:
 // singular systems keep their iterative result).
 template <int KL, int KU>
-__global__ void __launch_bounds__(128) banded_backsub_kernel(const BandParams P) {
+__global__ void __launch_bounds__(128, 6) banded_backsub_kernel(const BandParams P) {
   constexpr int W = Geo<KL, KU>::W;
   constexpr int NA = (W + 31) / 32;
-  constexpr int PF = 8;
+  constexpr int PF = 4;
   extern __shared__ __align__(16) double xsm[];  // [4 warps][n + W]
   const int l = threadIdx.x & 31, wi = threadIdx.x >> 5;
   const int n = P.n;
