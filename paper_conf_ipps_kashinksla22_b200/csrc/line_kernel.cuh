@@ -197,6 +197,11 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
       asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
                    "r"(static_cast<uint32_t>(n * 8) & ~15u)
                    : "memory");
+      const void *xa = P.x0 ? P.x0 + ns * n : nullptr;  // warm start (Picard) guess
+      if (xa && (reinterpret_cast<uintptr_t>(xa) & 15u) == 0)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(xa),
+                     "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                     : "memory");
     }
   }
 
