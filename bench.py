@@ -524,7 +524,8 @@ def run_ours(args, rank, world, local_rank):
                         "max_true_rel_residual_rank0": float(np.max(
                             res_h / np.linalg.norm(b_h.numpy(), axis=1)))},
         "parity_sample": parity,
-        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms)},
+        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms),
+                      "std": statistics.pstdev(kern_ms), "n": len(kern_ms)},
     }
     if rank == 0:
         emit(line, args)
@@ -662,7 +663,8 @@ def run_banded(args, rank, world, local_rank):
                  "launches_per_step": launches_per_step,
                  "mode": "split: factor kernel + back-substitution kernel per chunk of systems"},
         "solve_stats": {"info_nonzero": int((info_h != 0).sum())}, "parity_sample": parity,
-        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms)},
+        "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms),
+                      "std": statistics.pstdev(kern_ms), "n": len(kern_ms)},
     }
     if rank == 0:
         emit(line, args)
