@@ -100,9 +100,10 @@ def check(rc: int):
         raise BsolveError(rc, lib().bsolve_last_error().decode(errors="replace"))
 
 
-def _stream_ptr(stream):
+def _stream_ptr(stream, device=None):
+    """cudaStream_t of `stream`, default: the current stream of the handle's device."""
     import torch
-    s = torch.cuda.current_stream() if stream is None else stream
+    s = torch.cuda.current_stream(device) if stream is None else stream
     return s.cuda_stream
 
 
@@ -218,6 +219,8 @@ class Solver:
             raise TypeError(f"{name} must be contiguous {dtype}")
         if t.numel() != int(np.prod(shape)):
             raise ValueError(f"{name} has {t.numel()} elements, expected {shape}")
+        if t.device.index != self.device:
+            raise ValueError(f"{name} lives on cuda:{t.device.index}, the handle on cuda:{self.device}")
 
     def alloc_outputs(self):
         import torch
@@ -239,15 +242,18 @@ class Solver:
         check(lib().bsolve_run(self._h, values.data_ptr(), b.data_ptr(),
                                None if x0 is None else x0.data_ptr(), float(tol), int(maxiter),
                                x.data_ptr(), it.data_ptr(), res.data_ptr(),
-                               None if st is None else st.data_ptr(), _stream_ptr(stream)))
+                               None if st is None else st.data_ptr(), _stream_ptr(stream, self.device)))
         return x, it, res, st
 
     def spmv(self, values, x, out=None, stream=None):
         import torch
-        batch = x.shape[0]
+        batch = int(x.shape[0]) if x.dim() > 0 else 0
+        self._dev_check(x, "x", (batch, self.n), torch.float64)
+        self._dev_check(values, "values", (batch, self.values_per_system), torch.float64)
         y = torch.empty_like(x) if out is None else out
+        self._dev_check(y, "out", (batch, self.n), torch.float64)
         check(lib().bsolve_spmv(self._h, values.data_ptr(), x.data_ptr(), y.data_ptr(), int(batch),
-                                _stream_ptr(stream)))
+                                _stream_ptr(stream, self.device)))
         return y
 
     def banded_solve(self, values, b, out=None, ipiv: bool = False, stream=None):
@@ -265,16 +271,18 @@ class Solver:
         piv = torch.empty((self.batch, self.n), dtype=torch.int32, device=dev) if ipiv else None
         check(lib().bsolve_banded_solve(self._h, values.data_ptr(), b.data_ptr(), x.data_ptr(),
                                         info.data_ptr(), None if piv is None else piv.data_ptr(),
-                                        _stream_ptr(stream)))
+                                        _stream_ptr(stream, self.device)))
         return (x, info, piv) if ipiv else (x, info)
 
     def csr_to_ell(self, csr_values, out=None, stream=None):
         import torch
-        batch = csr_values.shape[0]
+        batch = int(csr_values.shape[0]) if csr_values.dim() > 0 else 0
+        self._dev_check(csr_values, "csr_values", (batch, self.nnz), torch.float64)
         y = (torch.empty((batch, self.width * self.n), dtype=torch.float64,
                          device=csr_values.device) if out is None else out)
+        self._dev_check(y, "out", (batch, self.width * self.n), torch.float64)
         check(lib().bsolve_csr_to_ell(self._h, csr_values.data_ptr(), y.data_ptr(), int(batch),
-                                      _stream_ptr(stream)))
+                                      _stream_ptr(stream, self.device)))
         return y
 
     # -------------------------------------------------------------- host --

@@ -60,6 +60,9 @@ struct BandParams {
                           // they were.  nullptr: solve every system.
   double *resnorm;        // fallback mode: [batch] out
   double *ws;             // per CTA: U [n][W] (row j: 1/u_jj, u_j,j+1 ..) then y [n]
+  const int32_t *list;    // fallback mode: indices of the systems to solve (compacted
+                          // on the device by fallback_compact_kernel), nullptr: all
+  const int32_t *list_len;  // device: number of entries in `list`
   long long sys_stride;
   int E, n, batch;
 };
@@ -297,7 +300,9 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
     // the row-major U (L1-cached: each lane walks its rows backwards).
     const int l = t - NTF;
     int k = 0;
-    for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+    const long long cnt = P.list ? *P.list_len : P.batch;
+    for (long long it = blockIdx.x; it < cnt; it += gridDim.x) {
+      const long long sys = P.list ? P.list[it] : it;
       if (P.only && P.only[sys] == 0) continue;  // converged iteratively (same test as below)
       const int b = k & 1;
       mbar_wait_sleep(&full_bar[b], (k >> 1) & 1);
@@ -315,7 +320,9 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
   const bool loader = t > W;
   const int lidx = t - W - 1;  // loader lane = pattern entry (needs NTF - W - 1 > E)
   int k = 0;
-  for (long long sys = blockIdx.x; sys < P.batch; sys += gridDim.x) {
+  const long long cnt = P.list ? *P.list_len : P.batch;
+  for (long long it = blockIdx.x; it < cnt; it += gridDim.x) {
+    const long long sys = P.list ? P.list[it] : it;
     if (P.only && P.only[sys] == 0) continue;  // converged iteratively
     const int b = k & 1;
     if (!SPLIT && k >= 2) mbar_wait(&empty_bar[b], ((k >> 1) - 1) & 1);  // back subst. k-2 done
@@ -479,8 +486,10 @@ __global__ void __launch_bounds__(128, 6) banded_backsub_kernel(const BandParams
     for (int i = l; i < W; i += 32) xw[n + i] = 0.0;  // x beyond n is zero
     __syncwarp();
     auto uload = [&](int jj, int m) -> double {  // u_jj,jj+d, d = l + 32 m (d = 0: 1/u_jj)
+      // entries of columns >= n are never written by the factor kernel (the
+      // workspace is not cleared): never read them, x beyond n is zero anyway
       const int d = l + 32 * m;
-      return (jj >= 0 && d < W) ? U[(size_t)jj * W + d] : 0.0;
+      return (jj >= 0 && d < W && jj + d < n) ? U[(size_t)jj * W + d] : 0.0;
     };
     double q[PF][NA], yq[PF];
 #pragma unroll
@@ -524,6 +533,25 @@ __global__ void __launch_bounds__(128, 6) banded_backsub_kernel(const BandParams
     }
     if (P.only) fallback_residual(P, sys, l);
     __syncwarp();
+  }
+}
+// Fallback mode, first launch: list the systems whose iterative status is not
+// CONVERGED (their order in the list is irrelevant: every system is solved
+// independently, bit for bit the same wherever it lands).  *len must be 0 on
+// entry (cudaMemsetAsync on the same stream).
+static __global__ void __launch_bounds__(256) fallback_compact_kernel(const int8_t *status, long long batch,
+                                                               int32_t *list, int32_t *len) {
+  const int lane = threadIdx.x & 31;
+  // warp-uniform trip count: the ballot needs all 32 lanes
+  for (long long i0 = blockIdx.x * 256LL + (threadIdx.x & ~31); i0 < batch; i0 += gridDim.x * 256LL) {
+    const long long i = i0 + lane;
+    const bool need = i < batch && status[i] != 0;
+    const unsigned m = __ballot_sync(0xffffffffu, need);
+    if (m == 0) continue;
+    int base = 0;
+    if (lane == __ffs(m) - 1) base = atomicAdd(len, __popc(m));
+    base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
+    if (need) list[base + __popc(m & ((1u << lane) - 1))] = static_cast<int32_t>(i);
   }
 }
 }  // namespace bband

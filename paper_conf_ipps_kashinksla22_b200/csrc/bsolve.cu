@@ -115,17 +115,31 @@ struct bsolve_plan {
   int8_t *h_st[kSlots] = {};
   double *h_bws[kSlots] = {};       // banded workspace per pipeline slot
   size_t h_bws_bytes[kSlots] = {};
-  int32_t *h_it_b[kSlots] = {};     // banded info per pipeline slot (fallback mode)
+  double *h_fbws[kSlots] = {};      // direct fallback per pipeline slot: workspace,
+  int32_t *h_fbl[kSlots] = {};      //   compacted system list (chunk entries),
+  int32_t *h_fbn[kSlots] = {};      //   list length
   // banded direct solver (bsolve_banded_solve, lazily set up)
-  int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col - row + 128)
+  int32_t *d_bnd = nullptr;   // [W][n] packed (value index << 8) | (col mod window width)
+  int32_t *d_bcol = nullptr;  // [W][n] column of ELL slot k of row r (fallback residual)
   int bnd_w = 0;              // window width the table's ring positions use
+  const BVariant *bvar = nullptr;  // banded instance covering the pattern (setup_banded)
+  int smem_optin = 0;         // device limit on dynamic SMEM per CTA
   int direct_fallback = 0;    // bsolve_options.direct_fallback
   int banded_launches = 0;    // kernel launches of the last banded call
-  int32_t *d_binfo = nullptr; // split banded solve in fallback mode: per-chunk info
-  long long binfo_len = 0;
-  double *d_bws = nullptr;    // per-CTA U + y workspace
+  double *d_bws = nullptr;    // split banded solve: per-system U + y workspace (one chunk)
   size_t bws_bytes = 0;
+  // direct fallback (allocated by bsolve_create, so bsolve_run stays asynchronous):
+  // fused-kernel workspace for fb_grid CTAs, the compacted list of non-converged
+  // systems and its length
+  int fb_grid = 0;
+  double *d_fbws = nullptr;
+  int32_t *d_fbl = nullptr, *d_fbn = nullptr;
 };
+
+static int setup_banded(bsolve_handle h);
+static size_t banded_ws_sys(bsolve_handle h);
+static int alloc_fallback(bsolve_handle h, int grid, long long list_len, double **ws,
+                          int32_t **list, int32_t **len);
 
 extern "C" void bsolve_default_options(bsolve_options *o) {
   if (!o) return;
@@ -153,8 +167,11 @@ static void free_plan(bsolve_plan *h) {
   cudaFree(h->d_src);
   cudaFree(h->d_ctr);
   cudaFree(h->d_bnd);
+  cudaFree(h->d_bcol);
   cudaFree(h->d_bws);
-  cudaFree(h->d_binfo);
+  cudaFree(h->d_fbws);
+  cudaFree(h->d_fbl);
+  cudaFree(h->d_fbn);
   for (int s = 0; s < bsolve_plan::kSlots; ++s) {
     if (h->hs[s]) cudaStreamDestroy(h->hs[s]);
     cudaFree(h->h_val[s]);
@@ -165,7 +182,9 @@ static void free_plan(bsolve_plan *h) {
     cudaFree(h->h_it[s]);
     cudaFree(h->h_st[s]);
     cudaFree(h->h_bws[s]);
-    cudaFree(h->h_it_b[s]);
+    cudaFree(h->h_fbws[s]);
+    cudaFree(h->h_fbl[s]);
+    cudaFree(h->h_fbn[s]);
   }
   if (cur >= 0) cudaSetDevice(cur);
   delete h;
@@ -428,6 +447,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     return fail_free(fail(BSOLVE_ERR_CUDA, "cudaGetDeviceProperties: %s", cudaGetErrorString(ce)));
   h->num_sms = prop.multiProcessorCount;
   const int smem_optin = (int)prop.sharedMemPerBlockOptin;
+  h->smem_optin = smem_optin;
 
   // ---- cluster plan: one system per cluster of C CTAs x 1024 rows ---------
   // (DESIGN.md "Kernels" 8).  Auto for 9-point stencils with n > 1024.
@@ -817,6 +837,22 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
           cudaSuccess ||
       cudaMemcpy(h->d_diag, diag.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail_free(fail(BSOLVE_ERR_CUDA, "copy of the pattern to the device failed"));
+  if (h->direct_fallback) {
+    // banded tables + fallback buffers now, so bsolve_run never allocates:
+    // the fused banded kernel on at most one wave of resident CTAs, its
+    // workspace capped at 256 MB (failures are rare; the grid bounds memory)
+    int rc = setup_banded(h);
+    if (rc) return fail_free(rc);
+    int occ = 0;
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)h->bvar->fn,
+                                                       h->bvar->nt, h->bvar->smem_bytes);
+    if (ce != cudaSuccess || occ < 1)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "direct_fallback: banded kernel cannot be resident"));
+    const long long cap = std::max<long long>(1, (256ll << 20) / (16ll * (long long)banded_ws_sys(h)));
+    h->fb_grid = (int)std::min<long long>((long long)occ * h->num_sms, cap);
+    rc = alloc_fallback(h, h->fb_grid, batch, &h->d_fbws, &h->d_fbl, &h->d_fbn);
+    if (rc) return fail_free(rc);
+  }
   if (prev >= 0) cudaSetDevice(prev);
   *out = h;
   return BSOLVE_OK;
@@ -881,9 +917,12 @@ static int check_run_args(bsolve_handle h, const double *values, const double *b
   return BSOLVE_OK;
 }
 
+static int launch_fallback(bsolve_handle h, const double *values, const double *b, double *x,
+                           int8_t *status, double *resnorm, long long count, cudaStream_t stream,
+                           int slot);
 static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
                          int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
-                         int8_t *only, double *resnorm, int slot = -1);
+                         int slot = -1);
 
 static int launch_solve(bsolve_handle h, const double *values, const double *b, const double *x0,
                         double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
@@ -958,7 +997,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "solve launch: %s", cudaGetErrorString(e));
   if (h->direct_fallback)  // non-converged systems -> banded LU
-    return launch_banded(h, values, b, x, nullptr, nullptr, count, stream, status, resnorm, slot);
+    return launch_fallback(h, values, b, x, status, resnorm, count, stream, slot);
   return BSOLVE_OK;
 }
 
@@ -1025,6 +1064,11 @@ static int ensure_host_pipeline(bsolve_handle h) {
         cudaMalloc(&h->h_st[s], c_) != cudaSuccess) {
       cudaGetLastError();
       return fail(BSOLVE_ERR_NOMEM, "device allocation for the host pipeline failed");
+    }
+    if (h->direct_fallback) {  // each slot's stream runs its own fallback (smaller grid)
+      const int rc = alloc_fallback(h, std::max(1, h->fb_grid / bsolve_plan::kSlots), chunk,
+                                    &h->h_fbws[s], &h->h_fbl[s], &h->h_fbn[s]);
+      if (rc) return rc;
     }
   }
   h->h_chunk = chunk;
@@ -1131,15 +1175,12 @@ extern "C" int bsolve_csr_to_ell(bsolve_handle h, const double *csr_values, doub
 }
 
 // ---------------------------------------------- banded direct solver (f4) --
-// Enqueue the banded LU kernel over `count` systems.  Fallback mode
-// (only != NULL): systems with only[i] == BSOLVE_SYS_CONVERGED are skipped;
-// for the others x is replaced by the direct solution (unless the band is
-// singular), resnorm[i] by its true residual and status[i] by
-// BSOLVE_SYS_DIRECT (only and status_out are the same array).
-static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
-                         int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
-                         int8_t *only, double *resnorm, int slot) {
-  if (count <= 0) return BSOLVE_OK;
+// Pick the banded instance that covers the pattern and upload its tables
+// (pattern entry -> value index + ring position; the ELL column of every
+// slot for the fallback's residual).  Synchronous host work: bsolve_create
+// runs it when direct_fallback is set, bsolve_banded_solve on its first call.
+static int setup_banded(bsolve_handle h) {
+  if (h->bvar) return BSOLVE_OK;
   const int kb = std::max(h->kl, h->ku);
   int cnt = 0;
   const BVariant *tab = variants_banded(&cnt), *bv = nullptr;
@@ -1154,50 +1195,134 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
                 h->sys_stride);
   const int n = h->n, W = h->W;
   const int Wb = 2 * bv->kb + 1;  // the instance's window width
-  if (!h->d_bnd || h->bnd_w != Wb) {
-    // entry k of row r: its value index inside one system's block (CSR order
-    // or ELL slot k) and the ring position (column mod Wb); padding -> -1
-    std::vector<int32_t> bnd((size_t)W * n, -1);
-    for (int k = 0; k < W; ++k)
-      for (int r = 0; r < n; ++r) {
-        const int e = h->h_csr2ell[(size_t)k * n + r];
-        if (e < 0) continue;
-        const long long vidx = h->fmt == FMT_ELL ? (long long)k * n + r : e;
-        const int col = h->h_ell_col[(size_t)k * n + r];
-        bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (col % Wb));
-      }
-    if (!h->d_bnd && cudaMalloc(&h->d_bnd, sizeof(int32_t) * bnd.size()) != cudaSuccess)
-      return fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed");
-    if (cudaMemcpy(h->d_bnd, bnd.data(), sizeof(int32_t) * bnd.size(), cudaMemcpyHostToDevice) !=
-        cudaSuccess)
-      return fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed");
-    h->bnd_w = Wb;
+  // entry k of row r: its value index inside one system's block (CSR order
+  // or ELL slot k) and the ring position (column mod Wb); padding -> -1
+  std::vector<int32_t> bnd((size_t)W * n, -1);
+  for (int k = 0; k < W; ++k)
+    for (int r = 0; r < n; ++r) {
+      const int e = h->h_csr2ell[(size_t)k * n + r];
+      if (e < 0) continue;
+      const long long vidx = h->fmt == FMT_ELL ? (long long)k * n + r : e;
+      const int col = h->h_ell_col[(size_t)k * n + r];
+      bnd[(size_t)k * n + r] = (int32_t)((vidx << 8) | (col % Wb));
+    }
+  const size_t tb = sizeof(int32_t) * bnd.size();
+  if (cudaMalloc(&h->d_bnd, tb) != cudaSuccess || cudaMalloc(&h->d_bcol, tb) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BSOLVE_ERR_NOMEM, "banded solver: pattern table allocation failed");
   }
+  if (cudaMemcpy(h->d_bnd, bnd.data(), tb, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(h->d_bcol, h->h_ell_col.data(), tb, cudaMemcpyHostToDevice) != cudaSuccess)
+    return fail(BSOLVE_ERR_CUDA, "banded solver: pattern table copy failed");
+  if (bv->smem_bytes > 48 * 1024) {
+    CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  bv->smem_bytes));
+    CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn_split,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, bv->smem_bytes));
+  }
+  h->bnd_w = Wb;
+  h->bvar = bv;
+  return BSOLVE_OK;
+}
+
+static size_t banded_ws_sys(bsolve_handle h) {  // doubles of U + y per system
+  return (size_t)h->n * h->bnd_w + h->n;
+}
+
+// Direct fallback buffers (the fused kernel's double-buffered per-CTA
+// workspace for `grid` CTAs, the compacted list, its length).
+static int alloc_fallback(bsolve_handle h, int grid, long long list_len, double **ws,
+                          int32_t **list, int32_t **len) {
+  if (cudaMalloc(ws, sizeof(double) * (size_t)grid * 2 * banded_ws_sys(h)) != cudaSuccess ||
+      cudaMalloc(list, sizeof(int32_t) * (size_t)std::max<long long>(1, list_len)) != cudaSuccess ||
+      cudaMalloc(len, sizeof(int32_t)) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BSOLVE_ERR_NOMEM, "direct_fallback: workspace allocation failed");
+  }
+  return BSOLVE_OK;
+}
+
+// direct_fallback (R27): after the iterative launch, list the
+// systems whose status is not CONVERGED on the device, then ONE fused banded
+// launch (factor warps + back-substitution warp, per-CTA double-buffered
+// workspace) solves only those.  No allocation, no host synchronisation:
+// 3 asynchronous operations (memset of the counter, compaction, solve); with
+// no failed system the solve kernel exits at once.
+static int launch_fallback(bsolve_handle h, const double *values, const double *b, double *x,
+                           int8_t *status, double *resnorm, long long count, cudaStream_t stream,
+                           int slot) {
+  const BVariant *bv = h->bvar;
+  double *ws = slot >= 0 ? h->h_fbws[slot] : h->d_fbws;
+  int32_t *list = slot >= 0 ? h->h_fbl[slot] : h->d_fbl;
+  int32_t *len = slot >= 0 ? h->h_fbn[slot] : h->d_fbn;
+  if (!bv || !ws || !list || !len)
+    return fail(BSOLVE_ERR_INVALID, "direct_fallback buffers are missing (handle not set up)");
+  CUDA_TRY(cudaMemsetAsync(len, 0, sizeof(int32_t), stream));
+  const int cgrid = (int)std::min<long long>((count + 255) / 256, (long long)h->num_sms * 4);
+  bband::fallback_compact_kernel<<<cgrid, 256, 0, stream>>>(status, count, list, len);
   bband::BandParams P;
   P.values = values;
   P.b = b;
   P.bnd = h->d_bnd;
-  P.cols = h->d_ell_col;
+  P.cols = h->d_bcol;
+  P.x = x;
+  P.info = nullptr;
+  P.ipiv = nullptr;
+  P.only = status;
+  P.resnorm = resnorm;
+  P.ws = ws;
+  P.list = list;
+  P.list_len = len;
+  P.sys_stride = h->sys_stride;
+  P.E = h->W;
+  P.n = h->n;
+  P.batch = (int)count;
+  const int grid = slot >= 0 ? std::max(1, h->fb_grid / bsolve_plan::kSlots) : h->fb_grid;
+  bv->fn<<<grid, bv->nt, bv->smem_bytes, stream>>>(P);
+  h->banded_launches = 2;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "fallback launch: %s", cudaGetErrorString(e));
+  return BSOLVE_OK;
+}
+
+// Standalone banded solve of `count` systems (bsolve_banded_solve[_host]).
+// Split mode (default; BSOLVE_BANDED_SPLIT=0 selects the fused kernel):
+// factor-only CTAs (more per SM) write U, y per system into a chunk
+// workspace, then one warp per system back-substitutes; chunks of systems
+// keep the workspace bounded.
+static int launch_banded(bsolve_handle h, const double *values, const double *b, double *x,
+                         int32_t *info, int32_t *ipiv, long long count, cudaStream_t stream,
+                         int slot) {
+  if (count <= 0) return BSOLVE_OK;
+  int rc = setup_banded(h);
+  if (rc) return rc;
+  const BVariant *bv = h->bvar;
+  const int n = h->n;
+  const int Wb = h->bnd_w;
+  bband::BandParams P;
+  P.values = values;
+  P.b = b;
+  P.bnd = h->d_bnd;
+  P.cols = h->d_bcol;
   P.x = x;
   P.info = info;
   P.ipiv = ipiv;
-  P.only = only;
-  P.resnorm = resnorm;
+  P.only = nullptr;
+  P.resnorm = nullptr;
+  P.list = nullptr;
+  P.list_len = nullptr;
   P.sys_stride = h->sys_stride;
-  P.E = W;
+  P.E = h->W;
   P.n = n;
-  const size_t ws_sys = (size_t)n * Wb + n;  // doubles of U + y per system
-  // Split mode (default; BSOLVE_BANDED_SPLIT=0 selects the fused kernel):
-  // factor-only CTAs (more per SM) write U, y per system into a chunk
-  // workspace, then one warp per system back-substitutes; chunks of systems
-  // keep the workspace bounded.
+  const size_t ws_sys = banded_ws_sys(h);
+  // the back substitution keeps x of each of its warps in SMEM: as many
+  // warps per CTA (<= 4) as the device's SMEM allows, else the fused kernel
+  const int bs_warps =
+      (int)std::min<long long>(4, (long long)h->smem_optin / ((long long)(n + Wb) * 8));
   const char *senv = getenv("BSOLVE_BANDED_SPLIT");
-  const bool split = !(senv && atoi(senv) == 0);
+  const bool split = !(senv && atoi(senv) == 0) && bs_warps >= 1;
   banded_fn fact = split ? bv->fn_split : bv->fn;
   const int nt = split ? bv->nt_split : bv->nt;
-  if (bv->smem_bytes > 48 * 1024)
-    CUDA_TRY(cudaFuncSetAttribute((const void *)fact, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  bv->smem_bytes));
   int occ = 0;
   CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)fact, nt,
                                                          bv->smem_bytes));
@@ -1228,46 +1353,29 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
     wsb = need;
   }
   P.ws = wsp;
-  if (split && only && !info && slot >= 0) {  // host pipeline, fallback mode: per-slot info
-    if (!h->h_it_b[slot] &&
-        cudaMalloc(&h->h_it_b[slot], sizeof(int32_t) * (size_t)h->h_chunk) != cudaSuccess)
-      return fail(BSOLVE_ERR_NOMEM, "banded solver: info buffer allocation failed");
-    info = h->h_it_b[slot];
-  }
-  if (split && only && !info) {  // fallback mode: the back substitution needs info
-    if (h->binfo_len < chunk) {
-      cudaFree(h->d_binfo);
-      h->d_binfo = nullptr;
-      h->binfo_len = 0;
-      if (cudaMalloc(&h->d_binfo, sizeof(int32_t) * chunk) != cudaSuccess)
-        return fail(BSOLVE_ERR_NOMEM, "banded solver: info buffer allocation failed");
-      h->binfo_len = chunk;
-    }
-  }
   h->banded_launches = split ? (int)(2 * ((count + chunk - 1) / chunk)) : 1;
   if (!split) {
     P.batch = count;
     const int grid = (int)std::min<long long>(resident, count);
     fact<<<grid, nt, bv->smem_bytes, stream>>>(P);
   } else {
+    const int sbs = bs_warps * (n + Wb) * (int)sizeof(double);  // per-warp x arrays
+    if (sbs > 48 * 1024)
+      CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn_backsub,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, sbs));
     for (long long c0 = 0; c0 < count; c0 += chunk) {
       const long long cnt = std::min<long long>(chunk, count - c0);
       bband::BandParams Q = P;
       Q.values = values + c0 * h->sys_stride;
       Q.b = b + c0 * n;
       Q.x = x + c0 * n;
-      Q.info = info ? info + c0 : (only ? h->d_binfo : nullptr);
+      Q.info = info ? info + c0 : nullptr;
       Q.ipiv = ipiv ? ipiv + c0 * n : nullptr;
-      Q.only = only ? only + c0 : nullptr;
-      Q.resnorm = resnorm ? resnorm + c0 : nullptr;
       Q.batch = cnt;
       fact<<<(int)std::min<long long>(resident, cnt), nt, bv->smem_bytes, stream>>>(Q);
-      const int gb = (int)std::min<long long>((cnt + 3) / 4, (long long)h->num_sms * 16);
-      const int sbs = 4 * (n + Wb) * (int)sizeof(double);  // per-warp x arrays
-      if (sbs > 48 * 1024)
-        CUDA_TRY(cudaFuncSetAttribute((const void *)bv->fn_backsub,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, sbs));
-      bv->fn_backsub<<<gb, 128, sbs, stream>>>(Q);
+      const int gb =
+          (int)std::min<long long>((cnt + bs_warps - 1) / bs_warps, (long long)h->num_sms * 16);
+      bv->fn_backsub<<<gb, 32 * bs_warps, sbs, stream>>>(Q);
     }
   }
   cudaError_t e = cudaGetLastError();
@@ -1290,8 +1398,7 @@ extern "C" int bsolve_banded_solve(bsolve_handle h, const double *values, const 
   int prev = -1;
   cudaGetDevice(&prev);
   if (prev != h->device) CUDA_TRY(cudaSetDevice(h->device));
-  rc = launch_banded(h, values, b, x, info, ipiv, h->batch, (cudaStream_t)stream, nullptr,
-                     nullptr);
+  rc = launch_banded(h, values, b, x, info, ipiv, h->batch, (cudaStream_t)stream);
   if (prev >= 0 && prev != h->device) cudaSetDevice(prev);
   return rc;
 }
@@ -1319,8 +1426,7 @@ extern "C" int bsolve_banded_solve_host(bsolve_handle h, const double *values, c
     CUDA_TRY(cudaMemcpyAsync(h->h_val[sl], values + s0 * ss, (size_t)cnt * ss * 8,
                              cudaMemcpyHostToDevice, st));
     CUDA_TRY(cudaMemcpyAsync(h->h_b[sl], b + s0 * n, (size_t)cnt * n * 8, cudaMemcpyHostToDevice, st));
-    rc = launch_banded(h, h->h_val[sl], h->h_b[sl], h->h_x[sl], h->h_it[sl], nullptr, cnt, st,
-                       nullptr, nullptr, sl);
+    rc = launch_banded(h, h->h_val[sl], h->h_b[sl], h->h_x[sl], h->h_it[sl], nullptr, cnt, st, sl);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(x + s0 * n, h->h_x[sl], (size_t)cnt * n * 8, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(cudaMemcpyAsync(info + s0, h->h_it[sl], (size_t)cnt * 4, cudaMemcpyDeviceToHost, st));

@@ -258,3 +258,46 @@ def test_direct_fallback_with_gmres():
     assert np.any(bad) and np.all(s1[bad] == 3) and np.array_equal(x1[~bad], x0[~bad])
     xo, _, _ = oracle_banded(p.row_ptr, p.col_idx, B.values[bad], B.b[bad])
     assert np.max(np.linalg.norm(x1[bad] - xo, axis=1) / np.linalg.norm(xo, axis=1)) <= 1e-12
+
+
+def test_direct_fallback_csr_resnorm_is_true_residual():
+    """CSR values + direct_fallback: the DIRECT systems' resnorm is the true
+    ||b - A x|| (the residual reads each value with its own column: ADVICE r1)."""
+    B = X.make_batch(0, 64)
+    p = B.pattern
+    S = Solver(p.row_ptr, p.col_idx, 64, format="csr", direct_fallback=True)
+    x, it, res, st = S.run(to_dev(B.values), to_dev(B.b), maxiter=6)
+    torch.cuda.synchronize()
+    x, res, st = x.cpu().numpy(), res.cpu().numpy(), st.cpu().numpy()
+    assert np.any(st == 3) and np.any(st == 0)
+    for k in np.nonzero(st == 3)[0]:
+        tr = np.linalg.norm(B.b[k] - O.spmv(p.row_ptr, p.col_idx, B.values[k], x[k]))
+        bn = np.linalg.norm(B.b[k])
+        assert res[k] <= 1e-13 * bn and abs(res[k] - tr) <= 0.5 * tr + 1e-15 * bn, (k, res[k], tr)
+    assert S.query()["banded_launches"] == 2  # compaction + one fused solve launch
+
+
+def test_direct_fallback_no_failures_is_cheap():
+    """All systems converge: the fallback launches still run (compaction +
+    an immediately-exiting solve) and change nothing, bit for bit."""
+    B = X.make_batch(0, 600)
+    p = B.pattern
+    _, (x0, it0, r0, s0) = _run(p, B.values, B.b)
+    _, (x1, it1, r1, s1) = _run(p, B.values, B.b, direct_fallback=True)
+    assert np.all(s0 == 0)
+    for a, b in ((x0, x1), (it0, it1), (r0, r1), (s0, s1)):
+        assert np.array_equal(a, b)
+
+
+def test_banded_large_grid_backsub_smem():
+    """64 x 127 grid (n = 8128, kb = 65): the split back substitution sizes its
+    per-warp x arrays to the device's SMEM limit."""
+    pat = X.stencil_pattern(64, 127)
+    B = X.make_batch(0, 3, pattern=pat)
+    S = Solver(pat.row_ptr, pat.col_idx, 3)
+    x, info = S.banded_solve(to_dev(S.ell_values(B.values)), to_dev(B.b))
+    torch.cuda.synchronize()
+    x, info = x.cpu().numpy(), info.cpu().numpy()
+    assert np.all(info == 0)
+    xo, io, _ = oracle_banded(pat.row_ptr, pat.col_idx, B.values, B.b)
+    assert np.max(np.linalg.norm(x - xo, axis=1) / np.linalg.norm(xo, axis=1)) <= 1e-12

@@ -13,8 +13,13 @@ import oracle as O  # noqa: E402  (test infrastructure: checks the results)
 import xgcgen as X  # noqa: E402
 from paper_conf_ipps_kashinksla22_b200 import Solver  # noqa: E402
 
+# (name, grid, Solver options[, developer env knobs read by bsolve_create])
 CASES = [
-    ("tmem values (default 992)", dict(nx=32, ny=31), dict()),
+    ("line-tiled tmem (bench default)", dict(nx=32, ny=31), dict()),
+    ("line-tiled tmem, grid 31x32", dict(nx=31, ny=32), dict()),
+    ("line-tiled GMRES(7)", dict(nx=32, ny=31), dict(solver="gmres")),
+    ("line-tiled + direct fallback", dict(nx=32, ny=31), dict(direct_fallback=True)),
+    ("strided tmem (line off)", dict(nx=32, ny=31), dict(), {"BSOLVE_TMEM_LINE": "0"}),
     ("tmem values, unaligned block (5x5)", dict(nx=5, ny=5), dict(placement="tmem")),
     ("hybrid 128x8 DIA, 4 reg slots", dict(nx=32, ny=31), dict(block_threads=128, reg_slots=4)),
     ("smem 256x4 DIA", dict(nx=32, ny=31), dict(block_threads=256)),
@@ -23,6 +28,7 @@ CASES = [
     ("persistent regs", dict(nx=32, ny=31), dict(placement="regs")),
     ("cluster C=4 (n=4032)", dict(nx=64, ny=63), dict()),
     ("cluster C=3 (n=2112)", dict(nx=64, ny=33), dict()),
+    ("line-tiled cluster C=4 (n=4032)", dict(nx=64, ny=63), dict(), {"BSOLVE_CLUSTER_LINE": "1"}),
 ]
 
 
@@ -59,13 +65,26 @@ def banded_cases():
 
 def main():
     batch = int(os.environ.get("SAN_BATCH", "3"))
-    bad = banded_cases()
+    only = os.environ.get("SAN_CASES")
+    bad = banded_cases() if not only or "banded" in only else 0
     if os.environ.get("SAN_ONLY_BANDED"):
         sys.exit(1 if bad else 0)
-    for name, grid, opts in CASES:
+    # SAN_CASES: comma-separated substrings of case names ("banded": the f4 cases)
+    for case in CASES:
+        name, grid, opts = case[:3]
+        if only and not any(k in name for k in only.split(",")):
+            continue
+        env = case[3] if len(case) > 3 else {}
+        saved = {k: os.environ.get(k) for k in env}
+        os.environ.update(env)
         pat = X.stencil_pattern(**grid)
         B = X.make_batch(0, batch, pattern=pat)
         S = Solver(pat.row_ptr, pat.col_idx, batch, **opts)
+        for k, v in saved.items():  # knobs are read at create time only
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
         vals = S.ell_values(B.values) if S.format == "ell" else B.values
         x, it, res, st = S.run(torch.from_numpy(vals).cuda(), torch.from_numpy(B.b).cuda())
         torch.cuda.synchronize()
