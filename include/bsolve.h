@@ -158,7 +158,7 @@ typedef struct bsolve_info {
   int block_threads;       /* CTA size used by the solve kernel               */
   int rows_per_thread;     /* rows each thread owns                           */
   int smem_bytes;          /* dynamic shared memory per CTA                   */
-  int ctas_per_sm;         /* resident CTAs per SM (occupancy calculator)     */
+  int ctas_per_sm;         /* resident CTAs per SM                            */
   int num_sms;             /* SMs on the device                               */
   int grid;                /* CTAs launched per bsolve_run (REGS: persistent) */
   int kl, ku;              /* lower / upper bandwidth of the pattern          */
@@ -172,7 +172,13 @@ typedef struct bsolve_info {
   int solver, precond, restart; /* resolved BSOLVE_SOLVER_*, BSOLVE_PREC_*, m  */
   int banded_launches;     /* kernel launches of the last bsolve_banded_solve
                               (or direct-fallback) call: 2 per system chunk in
-                              the split mode, 1 fused; 0 before the first   */
+                              the split mode, 1 fused; 2 for a direct
+                              fallback (compaction + fused solve); 0 before
+                              the first                                      */
+  int regs_per_thread;     /* registers of the solve kernel (TMEM plans), else 0 */
+  int occupancy_api;       /* cudaOccupancyMaxActiveBlocksPerMultiprocessor for
+                              it (TMEM plans; ctas_per_sm is computed from the
+                              register, SMEM, thread and TMEM-column limits) */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

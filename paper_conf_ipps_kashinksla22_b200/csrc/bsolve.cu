@@ -86,6 +86,8 @@ struct bsolve_plan {
   int solver = 0, precond = 0, restart = 0;
   int fmt = 0, place = 0, stop = 0, trc = 1, device = 0;
   int nt = 0, r = 0, smem_bytes = 0, smem_vals = 0, n_pad = 0, ctas_per_sm = 0, num_sms = 0;
+  int occ_api = 0;         // cudaOccupancyMaxActiveBlocksPerMultiprocessor (TMEM plans)
+  int regs = 0;            // registers per thread of the solve kernel
   int kl = 0, ku = 0;
   int kfmt = 0;            // kernel storage mode: FMT_CSR / FMT_ELL / FMT_DIA
   int guard = 0;           // DIA: zero doubles around the gather body
@@ -96,6 +98,7 @@ struct bsolve_plan {
   const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
   solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
   int line_nx = 0;                   // > 0: line-tiled TMEM kernel for an NX-wide 9-point grid
+  int line_ctas = 0;                 // its resident CTAs per SM (launch bounds)
   int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};  // its canonical offset -> ELL slot map
   persist_fn var_tmem_p = nullptr;   // persistent TMEM kernel (aligned buffers)
   int smem_bytes_tmem_p = 0, grid_tmem_p = 0;
@@ -572,14 +575,25 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const int lg = genv ? atoi(genv) : 4;  // measured best: 7.33 vs 7.05 (G=2) M sys/s
     const char *rowsenv = getenv("BSOLVE_TMEM_LINE_ROWS");  // rows per thread: 8 or 4
     const int lr = rowsenv ? atoi(rowsenv) : 8;
-    const char *roundsenv = getenv("BSOLVE_ROUNDS");  // BiCGSTAB reduction rounds: 3 or 2
-    const int lrounds = roundsenv ? atoi(roundsenv) : 3;
-    // first pass: the requested geometry; second pass: any variant for the grid
+    // developer knobs: BSOLVE_LINE_CTAS = 2 selects the 2-CTA line kernel
+    // (line_kernel.cuh) instead of the 3-CTA one (line3_kernel.cuh);
+    // BSOLVE_ROUNDS = reduction rounds per BiCGSTAB iteration (3-CTA default
+    // 2 = DESIGN.md R29, 2-CTA default 3)
+    const char *ctasenv = getenv("BSOLVE_LINE_CTAS");
+    const int lctas = ctasenv ? atoi(ctasenv) : 3;
+    const char *roundsenv = getenv("BSOLVE_ROUNDS");
+    const int lrounds = roundsenv ? atoi(roundsenv) : (lctas == 3 ? 2 : 3);
+    // first pass: the requested geometry; second pass: any 2-CTA variant for the grid
     for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
       const LVariant &cand = lv[i % lcnt];
       if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
       if (!gm && cand.rounds != lrounds) continue;
-      if (i < lcnt && (cand.g != lg || cand.r != lr)) continue;
+      if (i < lcnt) {
+        if (cand.ctas != lctas) continue;
+        if (lctas == 2 && (cand.g != lg || cand.r != lr)) continue;
+      } else if (cand.ctas != 2) {
+        continue;
+      }
       const int NX = cand.nx;
       const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
       int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
@@ -620,6 +634,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       for (int c = 0; c < 8; ++c) h->c2s[c] = line_c2s[c];
       h->nt = 1024 / line_v->r;
       h->r = line_v->r;
+      h->line_ctas = line_v->ctas;
     } else {
       // developer knobs: rows per TMEM load group, threads per CTA
       const char *tenv = getenv("BSOLVE_TMEM_THREADS");
@@ -652,15 +667,32 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     // and leave the rest of the unified L1 to the 16-byte value loads
     int carve = (int)cudaSharedmemCarveoutMaxShared;
     if (h->line_nx) {
-      const long long need = 2LL * (h->smem_bytes + 1024);
+      const long long need = (long long)h->line_ctas * (h->smem_bytes + 1024);
       carve = (int)std::min<long long>(100, (need * 100 + prop.sharedMemPerMultiprocessor - 1) /
                                                  prop.sharedMemPerMultiprocessor + 5);
     }
     cudaFuncSetAttribute((const void *)h->var_tmem, cudaFuncAttributePreferredSharedMemoryCarveout,
                          carve);
-    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->ctas_per_sm, h->var_tmem, h->nt,
+    ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->occ_api, h->var_tmem, h->nt,
                                                        h->smem_bytes);
-    if (ce != cudaSuccess || h->ctas_per_sm < 1)
+    if (ce != cudaSuccess)
+      return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant occupancy query failed"));
+    // resident CTAs per SM from the kernel's own limits (registers in 256-
+    // register warp units, SMEM incl. the 1 KB per-CTA reservation, threads,
+    // TMEM columns: 512 per SM): what ncu reports as launch__occupancy_limit_*
+    {
+      cudaFuncAttributes fa;
+      CUDA_TRY(cudaFuncGetAttributes(&fa, (const void *)h->var_tmem));
+      h->regs = fa.numRegs;
+      const int warp_regs = (fa.numRegs * 32 + 255) / 256 * 256;
+      const int by_regs = prop.regsPerMultiprocessor / (warp_regs * (h->nt / 32));
+      const int by_smem = (int)(prop.sharedMemPerMultiprocessor / (h->smem_bytes + 1024));
+      const int by_threads = prop.maxThreadsPerMultiProcessor / h->nt;
+      const int tcols = h->line_nx ? (h->line_ctas == 3 ? 160 : 128) : 128 * (h->nt / 128);
+      const int by_tmem = 512 / tcols;
+      h->ctas_per_sm = std::min(std::min(by_regs, by_smem), std::min(by_threads, by_tmem));
+    }
+    if (h->ctas_per_sm < 1)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));
     // persistent variant with TMA prefetch of the next system (needs 16-byte
     // aligned system blocks; the launch also checks the buffer addresses)
@@ -881,6 +913,8 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->rows_per_thread = h->r;
   info->smem_bytes = h->smem_bytes;
   info->ctas_per_sm = h->ctas_per_sm;
+  info->regs_per_thread = h->regs;
+  info->occupancy_api = h->occ_api;
   info->num_sms = h->num_sms;
   info->grid = h->place == PLACE_REGS      ? (int)std::min<long long>(h->grid_persist, h->batch)
                : h->place == PLACE_CLUSTER ? h->batch * h->cluster

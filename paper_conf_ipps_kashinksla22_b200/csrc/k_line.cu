@@ -2,6 +2,7 @@
 // stencils (line_kernel.cuh): grid widths NX with 8 | rows per thread, G rows
 // per TMEM load group.  NX = 32 is the paper's 32 x 31 velocity grid
 // (PAPER.md:519-530); NX = 31 its transpose (tests).  Launched from bsolve.cu.
+#include "line3_kernel.cuh"
 #include "line_kernel.cuh"
 #include "variants.h"
 
@@ -9,18 +10,27 @@ using namespace bsolve;
 
 #define LSMEM_(NX, R) ((R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 + 16)
 #define LV_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 3, \
-                       (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB>}
+                       (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB>, 2}
+// 3 CTAs per SM (line3_kernel.cuh, the default plan): r^, a_ii in TMEM, x in
+// SMEM, <= 168 registers, 3 partial sums per SpMV row.  RD = 2: rho and ||r||
+// from the omega round (R29, default); RD = 3: the literal 3-round
+// schedule of bicgstab_core.  (Measured and removed: double-buffered TMEM rows,
+// one FMA chain per row, a shallower one-value reduction, gathers one row
+// ahead -- DESIGN.md perf log.)
+#define LV3_(NX, RD) {NX, 8, 3, SOLVER_BICGSTAB, Line3Geom<NX>::SMEM_BYTES, RD, \
+                      (solve_fn)bicgstab_line3_kernel<NX, RD>, 3}
 // two reduction rounds per iteration (deferred stop test 1, algebraic rho)
 #define LV2_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 2, \
-                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB, 2, 2>}
+                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB, 2, 2>, 2}
 // GMRES: + the Krylov basis and the triangular factor in SMEM
 #define LVG_(NX, R, G) {NX, R, G, SOLVER_GMRES,                                          \
                         LSMEM_(NX, R) + (kMaxRestart * 1024 + kMaxRestart * kMaxRestart) * 8, 0, \
-                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_GMRES>}
+                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_GMRES>, 2}
 static const LVariant kLVariants[] = {LV_(32, 8, 2),  LV_(32, 8, 4),  LV_(32, 4, 2),
                                       LV_(32, 4, 4),  LV_(31, 8, 4),  LV_(31, 4, 2),
                                       LVG_(32, 8, 2), LVG_(31, 8, 2), LV2_(32, 8, 4),
-                                      LV2_(31, 8, 4)};
+                                      LV2_(31, 8, 4), LV3_(32, 2),    LV3_(31, 2),
+                                      LV3_(32, 3),    LV3_(31, 3)};
 
 const LVariant *variants_line(int *count) {
   *count = (int)(sizeof(kLVariants) / sizeof(kLVariants[0]));

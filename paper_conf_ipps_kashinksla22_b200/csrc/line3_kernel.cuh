@@ -1,0 +1,470 @@
+// line3_kernel.cuh -- the line-tiled TMEM plan at THREE CTAs per SM
+// (DESIGN.md "Kernels" 12; round-2 redesign of bicgstab_tmem_line_kernel).
+//
+// What it computes: Algorithm 1 of the paper (Sec. IV-D),
+// BiCGSTAB right-preconditioned with scalar Jacobi, one CTA per system, each
+// system stopping on its own -- the same schedule, stop
+// tests, breakdown and true-residual guard as bicgstab_core (kernels.cuh,
+// readings R1-R10 of DESIGN.md); only WHERE the per-row state lives changes.
+//
+// Why: the 2-CTA line kernel (252 registers x 128 threads) is latency-bound
+// (round-1 ncu: 12.4% warps active, "wait" and "short scoreboard" stalls,
+// SMEM pipe 39% busy).  A third resident CTA needs <= 168 registers per
+// thread (65,536 / 384).  The register diet:
+//   * registers: only r (then s), p, v and d = 1/a_ii, 8 rows each;
+//   * tensor memory: besides the 8 off-diagonal values of each row (128
+//     columns, as before) a SECOND allocation of 32 columns per CTA holds the
+//     shadow residual r^ (columns 0-15) and the diagonal a_ii (16-31):
+//     3 x (128 + 32) = 480 <= 512 columns per SM;
+//   * shared memory: the iterate x, thread-private (double2 layout, every
+//     access conflict-free): read and written once per iteration;
+//   * the SpMV operand of the thread's own rows, d_j * p_j (or d_j * s_j), is
+//     recomputed where it is needed instead of being kept: the same product
+//     the publish stored, so the same bits;
+//   * one TMEM row (16 columns) in flight at a time, a sliding window of
+//     gathered operands.
+#pragma once
+#include "line_kernel.cuh"
+
+namespace bsolve {
+
+// SMEM layout of one CTA: [gather planes R*S][reduction scratch 16*NWARP]
+// [x: R*NT][2 TMEM base slots].
+template <int NX>
+struct Line3Geom {
+  static constexpr int R = 8, NT = 128, NWARP = 4;
+  using L = LineGeom<NX, NT, R>;
+  static constexpr int OFF_RED = R * L::S;
+  static constexpr int OFF_X = ((OFF_RED + 16 * NWARP) + 1) & ~1;  // 16-byte aligned
+  static constexpr int SMEM_BYTES = (OFF_X + R * NT) * 8 + 16;
+};
+
+__device__ __forceinline__ void tmem_ld2(uint32_t taddr, uint32_t (&r)[2]) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0,%1}, [%2];"
+               : "=r"(r[0]), "=r"(r[1])
+               : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_regs_ready2(uint32_t (&r)[2]) {
+  asm volatile("" : "+r"(r[0]), "+r"(r[1]));
+}
+
+// y = A (d .* g) for rows 8t .. 8t+7 with the operands of the thread's own
+// rows recomputed as d_j * g_j; values from TMEM, diagonal a_jj from the aux
+// TMEM columns; neighbours gathered from the published planes.  One row at a
+// time: its TMEM loads, the two plane operands it is the first to need
+// (a sliding window: registers), wait, then three independent partial sums
+// (line above | own line | line below) added at the end -- the 9-term FMA
+// chain of one row was the latency bound (ncu "wait" stalls; DESIGN.md perf
+// log).  The row sum is a fixed order, so results are deterministic.
+template <int NX>
+__device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const double *gq,
+                                           const double (&dd)[8], const double (&g)[8],
+                                           double (&y)[8]) {
+  constexpr int R = 8;
+  using L = LineGeom<NX, 128, R>;
+  uint32_t w[16], aw[2];
+  double gm[R + 2], gp[R + 2], gr = 0.0;
+#pragma unroll
+  for (int e = 0; e < 3; ++e) {
+    gm[e] = gq[L::idx(-NX + e - 1)];
+    gp[e] = gq[L::idx(NX + e - 1)];
+  }
+  const double gl = gq[L::idx(-1)];
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    tmem_ld16(tval + 16 * j, w);
+    tmem_ld2(ta0 + 2 * j, aw);
+    if (j > 0) {  // the two operands row j is the first to need
+      gm[j + 2] = gq[L::idx(-NX + j + 1)];
+      gp[j + 2] = gq[L::idx(NX + j + 1)];
+    }
+    if (j == R - 1) gr = gq[L::idx(R)];
+    tmem_wait_ld();
+    tmem_regs_ready(w);
+    tmem_regs_ready2(aw);
+    const double a0 = __hiloint2double(static_cast<int>(aw[1]), static_cast<int>(aw[0]));
+    const double own = dd[j] * g[j];
+    const double left = j == 0 ? gl : dd[j == 0 ? 0 : j - 1] * g[j == 0 ? 0 : j - 1];
+    const double right = j == R - 1 ? gr : dd[j == R - 1 ? j : j + 1] * g[j == R - 1 ? j : j + 1];
+    double c0 = tmem_f64(w, 0) * gm[j];
+    double c1 = a0 * own;
+    double c2 = tmem_f64(w, 5) * gp[j];
+    c0 = fma(tmem_f64(w, 1), gm[j + 1], c0);
+    c1 = fma(tmem_f64(w, 3), left, c1);
+    c2 = fma(tmem_f64(w, 6), gp[j + 1], c2);
+    c0 = fma(tmem_f64(w, 2), gm[j + 2], c0);
+    c1 = fma(tmem_f64(w, 4), right, c1);
+    c2 = fma(tmem_f64(w, 7), gp[j + 2], c2);
+    y[j] = (c0 + c1) + c2;  // rows >= n: zero values and diagonal -> 0
+  }
+}
+
+template <int NX, int ROUNDS = 2>
+__global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParams P) {
+  using G3 = Line3Geom<NX>;
+  constexpr int R = G3::R, NT = G3::NT;
+  using L = typename G3::L;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sg = reinterpret_cast<double *>(smem_raw);
+  double *sred = sg + G3::OFF_RED;
+  double2 *sx2 = reinterpret_cast<double2 *>(sg + G3::OFF_X) + threadIdx.x;  // x pair k at [k*NT]
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + G3::OFF_X + R * NT);
+
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long sys = blockIdx.x;
+  const int row0 = R * tid;
+  const double *gval = P.values + sys * P.sys_stride;
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(128));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s + 1)),
+                 "n"(32));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  for (int i = tid; i < R * (L::S - NT); i += NT) {  // zero guard columns
+    const int pl = i / (L::S - NT), q = i % (L::S - NT);
+    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
+  }
+  if (tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {  // L2 prefetch, as line kernel
+    const long long ns = sys + P.pf_ahead;
+    const void *va = P.values + ns * P.sys_stride;
+    const void *ba = P.b + ns * n;
+    if (((reinterpret_cast<uintptr_t>(va) | reinterpret_cast<uintptr_t>(ba)) & 15u) == 0) {
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(va),
+                   "r"(static_cast<uint32_t>(P.sys_stride * 8) & ~15u)
+                   : "memory");
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
+                   "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                   : "memory");
+      const void *xa = P.x0 ? P.x0 + ns * n : nullptr;
+      if (xa && (reinterpret_cast<uintptr_t>(xa) & 15u) == 0)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(xa),
+                     "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                     : "memory");
+    }
+  }
+  bool act[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t lane_hi = static_cast<uint32_t>(32 * warp) << 16;
+  const uint32_t tval = tbase_s[0] + lane_hi;  // 8 rows x 16 columns of values
+  const uint32_t trh = tbase_s[1] + lane_hi;   // r^ (8 doubles)
+  const uint32_t ta0 = trh + 16;               // a_jj (8 doubles)
+
+  // ---- this thread's rows: values -> TMEM, diagonal -> TMEM + d ------------
+  double d[R];
+  {
+    const bool vec = ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
+                     row0 + R <= n;
+    uint32_t aw[16];
+#pragma unroll
+    for (int j = 0; j < R; j += 2) {
+      double a0p[2], vv[2][8];
+      if (vec) {
+        const double2 dg = __ldg(reinterpret_cast<const double2 *>(gval + row0 + j));
+        a0p[0] = dg.x;
+        a0p[1] = dg.y;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const int k = P.c2s[c];
+          double2 v = make_double2(0.0, 0.0);
+          if (k >= 0) v = __ldg(reinterpret_cast<const double2 *>(gval + (long long)k * n + row0 + j));
+          vv[0][c] = v.x;
+          vv[1][c] = v.y;
+        }
+      } else {
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const bool a = act[j + h];
+          a0p[h] = a ? __ldg(gval + row0 + j + h) : 0.0;
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {
+            const int k = P.c2s[c];
+            vv[h][c] = (a && k >= 0) ? __ldg(gval + (long long)k * n + row0 + j + h) : 0.0;
+          }
+        }
+      }
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        uint32_t w[16];
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          w[2 * c] = static_cast<uint32_t>(__double2loint(vv[h][c]));
+          w[2 * c + 1] = static_cast<uint32_t>(__double2hiint(vv[h][c]));
+        }
+        tmem_st16(tval + 16 * (j + h), w);
+        d[j + h] = jacobi_inv(P.precond, a0p[h]);
+        aw[2 * (j + h)] = static_cast<uint32_t>(__double2loint(a0p[h]));
+        aw[2 * (j + h) + 1] = static_cast<uint32_t>(__double2hiint(a0p[h]));
+      }
+    }
+    tmem_st16(ta0, aw);
+  }
+  const double *bsys = P.b + sys * n;
+  double r[R], p[R], v[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) r[j] = act[j] ? __ldg(bsys + row0 + j) : 0.0;
+  tmem_wait_st();
+
+  LineComm<NX, NT, R> comm(sg, sred, act);
+  const double one[R] = {1, 1, 1, 1, 1, 1, 1, 1};
+  auto spmv = [&](const double(&dd)[R], const double(&g)[R], double(&y)[R]) {
+    line3_spmv<NX>(tval, ta0, comm.gq, dd, g, y);
+  };
+  auto x_load = [&](double(&xx)[R]) {
+#pragma unroll
+    for (int k = 0; k < R / 2; ++k) {
+      const double2 q = sx2[k * NT];
+      xx[2 * k] = q.x;
+      xx[2 * k + 1] = q.y;
+    }
+  };
+  auto x_store = [&](const double(&xx)[R]) {
+#pragma unroll
+    for (int k = 0; k < R / 2; ++k) sx2[k * NT] = make_double2(xx[2 * k], xx[2 * k + 1]);
+  };
+  auto rh_store = [&](const double(&q)[R]) {
+    uint32_t w[16];
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      w[2 * j] = static_cast<uint32_t>(__double2loint(q[j]));
+      w[2 * j + 1] = static_cast<uint32_t>(__double2hiint(q[j]));
+    }
+    tmem_st16(trh, w);
+    tmem_wait_st();
+  };
+  auto rh_load = [&](uint32_t(&w)[16]) {
+    tmem_ld16(trh, w);
+    tmem_wait_ld();
+    tmem_regs_ready(w);
+  };
+
+  // ---- a3: x = x0 (or 0), r = b - A x0, r^ = r, ||b|| ----------------------
+  double red3[2] = {0.0, 0.0};
+#pragma unroll
+  for (int j = 0; j < R; ++j) red3[0] += r[j] * r[j];  // b.b
+  {
+    double xx[R];
+#pragma unroll
+    for (int j = 0; j < R; ++j) xx[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + j) : 0.0;
+    x_store(xx);
+    if (P.x0) {
+#pragma unroll
+      for (int j = 0; j < R; ++j) comm.publish(j, xx[j]);
+      comm.sync();
+      spmv(one, xx, v);
+#pragma unroll
+      for (int j = 0; j < R; ++j) r[j] = r[j] - v[j];
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < R; ++j) {
+    p[j] = 0.0;
+    v[j] = 0.0;
+    red3[1] += r[j] * r[j];
+  }
+  rh_store(r);
+  comm.template sum<2>(red3);
+  const double bnorm = sqrt(red3[0]);
+  const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
+  const double tau2 = tau * tau;
+  const bool sq = tau2 > 1e-300 && tau2 < 1e300;  // R7: squared-norm stop tests
+  auto below = [&](double nrm2) { return sq ? nrm2 < tau2 : sqrt(nrm2) < tau; };
+  double rnorm2 = red3[1];
+  double rho = red3[1];  // r^.r with r^ = r
+
+  double *xout = P.x + sys * n;
+  if (P.stop == STOP_REL_B && bnorm == 0.0) {
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (act[j]) xout[row0 + j] = 0.0;
+    if (tid == 0) {
+      P.iters[sys] = 0;
+      P.resnorm[sys] = 0.0;
+      if (P.status) P.status[sys] = SYS_CONVERGED;
+    }
+  } else {
+    // true residual ||b - A x||^2 into q (publishes x; one more barrier)
+    auto true_residual = [&](double(&q)[R]) -> double {
+      double xx[R];
+      x_load(xx);
+#pragma unroll
+      for (int j = 0; j < R; ++j) comm.publish(j, xx[j]);
+      comm.sync();
+      spmv(one, xx, q);
+      double tr[1] = {0.0};
+#pragma unroll
+      for (int j = 0; j < R; ++j) {
+        const double bj = act[j] ? __ldg(bsys + row0 + j) : 0.0;
+        q[j] = act[j] ? bj - q[j] : 0.0;
+        tr[0] += q[j] * q[j];
+      }
+      comm.template sum<1>(tr);
+      return tr[0];
+    };
+
+    int it = 0, st = -1, exit_kind = 0;
+    double alpha = 1.0, omega = 1.0;
+    double beta_c = 1.0;  // alpha / (rho' omega): beta = rho * beta_c (R2)
+    double final_res = -1.0;
+    for (;;) {
+      exit_kind = 0;
+      while (true) {
+        if (below(rnorm2)) { exit_kind = 1; break; }        // stop test 1
+        if (it >= P.maxiter) break;
+        if (bad(rho)) { st = SYS_BREAKDOWN; break; }
+        // R2: beta = (rho / rho') (alpha / omega), the division done after the
+        // previous omega; ROUNDS == 2 keeps beta itself in beta_c (R29)
+        const double beta = ROUNDS == 2 ? beta_c : rho * beta_c;
+        // a5: p = r + beta (p - omega v); publish p^ = d p
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+          p[j] = r[j] + beta * (p[j] - omega * v[j]);
+          comm.publish(j, d[j] * p[j]);
+        }
+        comm.sync();
+        spmv(d, p, v);                                      // a6: v = A p^
+        ++it;
+        double rv[1];
+        {
+          uint32_t hw[16];
+          rh_load(hw);
+          rv[0] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * v[j]; });
+        }
+        comm.template sum<1>(rv);                           // a7: r^.v
+        if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
+        alpha = rho / rv[0];                                // R3
+        // s = r - alpha v (kept in r); publish s^ = d s
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+          r[j] = r[j] - alpha * v[j];
+          comm.publish(j, d[j] * r[j]);
+        }
+        comm.sync();
+        // ROUNDS == 3: t.s, t.t, s.s here and ||r||^2, r^.r in a third round.
+        // ROUNDS == 2 (R29): + r^.s, r^.t, so that rho_{i+1} =
+        // r^.s - omega r^.t and ||r_{i+1}||^2 = s.s - omega t.s come from this
+        // round (exact identities for r = s - omega t, omega = t.s / t.t); the
+        // third round runs only when an identity cancels more than 8 digits.
+        constexpr int KT = ROUNDS == 2 ? 5 : 3;
+        double ts[KT];
+        ts[2] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
+        if constexpr (ROUNDS == 2) {
+          uint32_t hw[16];
+          rh_load(hw);
+          ts[3] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * r[j]; });
+        }
+        double t[R];
+        spmv(d, r, t);                                      // a9: t = A s^ (speculative)
+        ts[0] = rows_sum<R>([&](int j) { return t[j] * r[j]; });
+        ts[1] = rows_sum<R>([&](int j) { return t[j] * t[j]; });
+        if constexpr (ROUNDS == 2) {
+          uint32_t hw[16];
+          rh_load(hw);
+          ts[4] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * t[j]; });
+        }
+        comm.template sum<KT>(ts);
+        if (below(ts[2])) {                                 // stop test 2
+          double xx[R];
+          x_load(xx);
+#pragma unroll
+          for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]);
+          x_store(xx);
+          exit_kind = 2;
+          break;
+        }
+        if (bad(ts[1])) { st = SYS_BREAKDOWN; break; }
+        omega = ts[0] / ts[1];
+        if (bad(omega)) { st = SYS_BREAKDOWN; break; }
+        if constexpr (ROUNDS == 3) beta_c = alpha / (rho * omega);  // rho becomes rho' below
+        {
+          double xx[R];
+          x_load(xx);
+#pragma unroll
+          for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]) + omega * (d[j] * r[j]);
+          x_store(xx);
+        }
+#pragma unroll
+        for (int j = 0; j < R; ++j) r[j] = r[j] - omega * t[j];   // r = s - omega t
+        bool explicit_round = ROUNDS == 3;
+        if constexpr (ROUNDS == 2) {
+          const double rho_n = ts[3] - omega * ts[4];
+          const double rr2 = ts[2] - omega * ts[0];
+          explicit_round = !(rr2 > 1e-8 * ts[2]) ||
+                           !(fabs(rho_n) > 1e-8 * (fabs(ts[3]) + fabs(omega * ts[4])));
+          if (!explicit_round) {
+            // beta_{i+1} = (rho_{i+1} / rho_i)(alpha / omega) with rho_{i+1} t.t =
+            // r^.s t.t - t.s r^.t: one division, independent of omega's
+            beta_c = alpha * (ts[3] * ts[1] - ts[0] * ts[4]) / (rho * ts[0]);
+            rnorm2 = rr2;
+            rho = rho_n;
+          }
+        }
+        if (explicit_round) {
+          double rr[2];
+          rr[0] = rows_sum<R>([&](int j) { return r[j] * r[j]; });
+          {
+            uint32_t hw[16];
+            rh_load(hw);
+            rr[1] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * r[j]; });
+          }
+          comm.template sum<2>(rr);                         // ||r||^2, r^.r
+          if constexpr (ROUNDS == 2) beta_c = rr[1] * alpha / (rho * omega);
+          rnorm2 = rr[0];
+          rho = rr[1];
+        }
+      }
+      if (st == SYS_BREAKDOWN || exit_kind == 0 || !P.trc) break;
+      // ---- a11: true-residual guard (R4) ------------------------
+      double q[R];
+      const double tr2 = true_residual(q);
+      final_res = sqrt(tr2);
+      if (final_res < tau || it >= P.maxiter) break;
+#pragma unroll
+      for (int j = 0; j < R; ++j) {  // restart from the true residual, keep counting
+        r[j] = q[j];
+        p[j] = 0.0;
+        v[j] = 0.0;
+      }
+      rh_store(q);
+      alpha = omega = beta_c = 1.0;
+      rnorm2 = tr2;
+      rho = tr2;
+      final_res = -1.0;
+    }
+    if (final_res < 0.0) {
+      comm.barrier();  // earlier gathers of this CTA done before x is published
+      double q[R];
+      final_res = sqrt(true_residual(q));
+    }
+    if (st != SYS_BREAKDOWN) {
+      if (P.trc) st = final_res < tau ? SYS_CONVERGED : SYS_MAXITER;
+      else st = exit_kind != 0 ? SYS_CONVERGED : SYS_MAXITER;
+    }
+    double xx[R];
+    x_load(xx);
+#pragma unroll
+    for (int j = 0; j < R; ++j)
+      if (act[j]) xout[row0 + j] = xx[j];
+    if (tid == 0) {
+      P.iters[sys] = it;
+      P.resnorm[sys] = final_res;
+      if (P.status) P.status[sys] = static_cast<int8_t>(st);
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[1]), "n"(32));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[0]), "n"(128));
+  }
+}
+
+}  // namespace bsolve

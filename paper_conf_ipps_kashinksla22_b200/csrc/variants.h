@@ -46,6 +46,7 @@ struct LVariant {
   int smem_bytes;  // dynamic SMEM of one CTA (gather planes + scratch + TMEM slot)
   int rounds;      // BiCGSTAB reduction rounds per iteration (3, or 2: algebraic rho)
   solve_fn fn;
+  int ctas;        // resident CTAs per SM the kernel is built for (launch bounds)
 };
 
 // batched banded LU (dgbsv analogue), k_banded.cu

@@ -563,6 +563,7 @@ def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
     """Line kernel with 8 rows x 128 threads or 4 rows x 256 threads per CTA
     (two warps per TMEM lane quarter) and other TMEM load groups: same parity
     bar, warm start included."""
+    monkeypatch.setenv("BSOLVE_LINE_CTAS", "2")  # geometries of the 2-CTA kernel
     monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
     monkeypatch.setenv("BSOLVE_TMEM_LINE_ROWS", str(rows))
     B = X.make_batch(0, 64, nx=nx, ny=ny)
