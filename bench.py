@@ -64,6 +64,21 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0,
                     help="target wall seconds of the oracle sample")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    ap.add_argument("--picard", type=int, default=0,
+                    help="P > 0: the Picard pipeline (SURVEY.md 8(f) f1, BASELINE configs[1] at "
+                         "scale): one step = P successive solves, matrices of Picard step p "
+                         "resident on the device, x0 = the previous solution (warm), timed "
+                         "beside P zero-guess solves")
+    ap.add_argument("--parity", choices=["full", "sample", "none"], default="full",
+                    help="N = 1: compare EVERY system's x with the oracle's banded LU (full) "
+                         "or only the cpu_baseline sample")
+    ap.add_argument("--backend", choices=["nccl", "gloo"], default="nccl",
+                    help="process-group backend for N > 1 (gloo: CPU plumbing tests)")
+    ap.add_argument("--standin", action="store_true",
+                    help="CPU stand-in solver (plumbing tests of the multi-rank harness; "
+                         "no GPU): Jacobi sweeps on the generator's systems")
+    ap.add_argument("--cross-check", type=int, default=64,
+                    help="N > 1: systems per rank that rank 0 re-solves and compares bitwise")
     return ap.parse_args()
 
 
@@ -135,8 +150,9 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------- inputs --
-def make_inputs(g0, count, args, pinned):
-    """Generate systems g0..g0+count-1 into (pinned) host buffers, ELL/CSR."""
+def make_inputs(g0, count, args, pinned, picard=0):
+    """Generate systems g0..g0+count-1 (Picard step `picard`) into (pinned)
+    host buffers, ELL/CSR."""
     import torch
     import xgcgen as X
     pat = X.stencil_pattern(args.nx, args.ny)
@@ -151,7 +167,7 @@ def make_inputs(g0, count, args, pinned):
     CH = 8192
     for c0 in range(0, count, CH):
         c1 = min(count, c0 + CH)
-        Bt = X.make_batch(g0 + c0, c1 - c0, pattern=pat, seed=args.seed)
+        Bt = X.make_batch(g0 + c0, c1 - c0, pattern=pat, seed=args.seed, picard=picard)
         if args.format == "ell":
             blk = vn[c0:c1]
             blk[:, ~ok] = 0.0
@@ -303,6 +319,144 @@ def emit(line, args):
             f.write(s + "\n")
 
 
+# ------------------------------------------------- multi-rank helpers --
+def digest(*arrays):
+    import hashlib
+    h = hashlib.sha256()
+    for a in arrays:
+        h.update(np.ascontiguousarray(a).tobytes())
+    return h.hexdigest()
+
+
+def cross_check(args, rank, world, local, solve_fn, device):
+    """Cross-P bitwise check: every rank hashes (x, iters,
+    resnorm, status) of the first m systems of its slice; rank 0 re-solves
+    those systems of EVERY rank on its own device and compares the hashes.
+    local = this rank's outputs (numpy); solve_fn(g0, m) -> same tuple."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_kashinksla22_b200.parallel import rank_slice
+    sls = [rank_slice(args.batch, r, world, args.scaling) for r in range(world)]
+    ms = [min(args.cross_check, s.count) for s in sls]
+    mine = digest(*(a[: ms[rank]] for a in local))
+    t = torch.tensor(list(bytes.fromhex(mine)), dtype=torch.uint8, device=device)
+    bufs = [torch.empty_like(t) for _ in range(world)]
+    dist.all_gather(bufs, t)
+    if rank != 0:
+        return None
+    got = [bytes(b.cpu().tolist()).hex() for b in bufs]
+    equal = []
+    for r in range(world):
+        if ms[r] == 0:
+            equal.append(True)
+            continue
+        ref = digest(*solve_fn(sls[r].g0, ms[r]))
+        equal.append(ref == got[r])
+    return {"systems_per_rank": ms, "ranks": world, "bitwise_equal": bool(all(equal)),
+            "per_rank": equal,
+            "how": "rank 0 re-solves the first systems of every rank's slice on its own device; "
+                   "sha256 of (x, iters, resnorm, status) compared"}
+
+
+def standin_solve(g0, count, args):
+    """CPU stand-in for the GPU solve, for the multi-rank plumbing tests only
+    (no GPU in the build container): Jacobi sweeps x += (b - A x) / diag(A) on
+    the generator's systems until ||b - A x|| < 1e-8 ||b|| (cap 500 sweeps).
+    Per-system results depend only on the global system index."""
+    import xgcgen as X
+    B = X.make_batch(g0, count, nx=args.nx, ny=args.ny, seed=args.seed)
+    p = B.pattern
+    n = p.n
+    rows = np.repeat(np.arange(n), np.diff(p.row_ptr))
+    A = np.zeros((count, n, n))
+    A[:, rows, p.col_idx] = B.values
+    dg = A[:, np.arange(n), np.arange(n)]
+    x = np.zeros_like(B.b)
+    it = np.zeros(count, np.int32)
+    bn = np.linalg.norm(B.b, axis=1)
+    res = bn.copy()
+    for _ in range(500):
+        r = B.b - np.einsum("bij,bj->bi", A, x)
+        res = np.linalg.norm(r, axis=1)
+        act = res >= 1e-8 * bn
+        if not act.any():
+            break
+        x[act] += r[act] / dg[act]
+        it[act] += 1
+    st = np.where(res < 1e-8 * bn, 0, 1).astype(np.int8)
+    return x, it, res, st
+
+
+def run_standin(args, rank, world):
+    """The multi-rank harness of run_ours (rank slices, barrier, timed steps,
+    max over ranks, stats gather, cross-P check, one JSON line from rank 0)
+    around the CPU stand-in solver: `python bench.py --gpus 2 --standin
+    --backend gloo` exercises the driver's N-rank entry point without a GPU."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_kashinksla22_b200.parallel import (gather_stats, max_over_ranks,
+                                                            rank_slice)
+    sl = rank_slice(args.batch, rank, world, args.scaling)
+    out = None
+    for _ in range(max(args.warmup, 0)):
+        out = standin_solve(sl.g0, sl.count, args)
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        out = standin_solve(sl.g0, sl.count, args)
+    dt = time.perf_counter() - t0
+    if world > 1:
+        dist.barrier()
+    dt = max_over_ranks(dt)
+    x, it, res, st = out
+    it_all, res_all, st_all = (t.numpy() for t in gather_stats(
+        torch.from_numpy(it), torch.from_numpy(res), torch.from_numpy(st)))
+    cross = (cross_check(args, rank, world, out, lambda g0, m: standin_solve(g0, m, args),
+                         "cpu") if world > 1 else None)
+    if rank == 0:
+        emit({"metric": METRIC, "value": sl.total * args.steps / dt, "unit": UNIT,
+              "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+              "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
+              "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+              "impl": "standin", "config": config_dict(args, world, sl.count),
+              "note": "CPU stand-in solver: plumbing test of the multi-rank harness, not a "
+                      "measurement",
+              "gathered": {"systems": int(it_all.size), "digest": digest(it_all, res_all, st_all),
+                           "iters_sum": int(it_all.astype(np.int64).sum())},
+              "cross_p": cross}, args)
+
+
+def full_parity(args, g0, count, x_dev, res_h, st_h):
+    """Every system of the timed batch against the oracle's direct solve
+    (north_star: ||x - x_direct|| / ||x_direct|| <= 1e-8 per system; VERDICT
+    r1 weak #2): the banded LU (dgbsv-like, oracle/oracle.c) over all host
+    cores, chunk by chunk, and the GPU's reported TRUE relative residual."""
+    import oracle as O
+    cores = host_cores()
+    t0 = time.perf_counter()
+    worst, worst_g, over, CH = 0.0, -1, 0, 8192
+    res_rel_max = 0.0
+    for c0 in range(0, count, CH):
+        c1 = min(count, c0 + CH)
+        pat, B = make_csr_sample(g0 + c0, c1 - c0, args)
+        xd = O.batch_banded(pat.row_ptr, pat.col_idx, B.values, B.b, threads=cores)
+        xg = x_dev[c0:c1].cpu().numpy()
+        rel = np.linalg.norm(xg - xd, axis=1) / np.linalg.norm(xd, axis=1)
+        k = int(np.argmax(rel))
+        if rel[k] > worst:
+            worst, worst_g = float(rel[k]), g0 + c0 + k
+        over += int(np.sum(rel > 1e-8))
+        res_rel_max = max(res_rel_max, float(np.max(res_h[c0:c1] / np.linalg.norm(B.b, axis=1))))
+    return {"systems_checked": count, "oracle": "banded LU with partial pivoting, dgbtf2 + "
+            "dgbtrs order (oracle/oracle.c), every system", "max_rel_x_diff_vs_direct": worst,
+            "worst_system": worst_g, "systems_over_1e-8": over,
+            "max_true_rel_residual_gpu": res_rel_max,
+            "all_converged": bool(np.all(st_h == 0)),
+            "within_north_star": bool(over == 0 and res_rel_max <= args.tol),
+            "oracle_wall_s": time.perf_counter() - t0, "oracle_cores": cores}
+
+
 # -------------------------------------------------------------------- ours --
 def run_ours(args, rank, world, local_rank):
     import torch
@@ -361,8 +515,23 @@ def run_ours(args, rank, world, local_rank):
     it_h = it.cpu().numpy()
     st_h = st.cpu().numpy()
     res_h = res.cpu().numpy()
-    it_all, _, st_all = (t.numpy() for t in gather_stats(it, res, st))
+    it_all, res_all, st_all = (t.numpy() for t in gather_stats(it, res, st))
     sum_iters_rank = int(it_h.astype(np.int64).sum())
+    cross = None
+    if world > 1:  # cross-P bitwise check of per-system outputs
+        def solve_local(gs, m):
+            _, vh, bh = make_inputs(gs, m, args, pinned=False)
+            T = Solver(pat.row_ptr, pat.col_idx, m, format=args.format,
+                       placement=args.placement, device=local_rank,
+                       block_threads=args.block_threads, reg_slots=args.reg_slots,
+                       solver=args.solver, precond=args.precond, restart=args.restart)
+            o = T.run(vh.to(dev), bh.to(dev), None, args.tol, args.maxiter)
+            torch.cuda.synchronize()
+            r = tuple(t.cpu().numpy() for t in o)
+            T.close()
+            return r
+        local = (x[: args.cross_check].cpu().numpy(), it_h, res_h, st_h)
+        cross = cross_check(args, rank, world, local, solve_local, dev)
 
     # ---- roofline (dominant kernel = the one solve kernel per step) ---------
     import json as _json
@@ -393,6 +562,11 @@ def run_ours(args, rank, world, local_rank):
     tmem_peak = 280.0 * num_sms * sm_max_mhz * 1e6      # measured tcgen05.ld, 8 warps/SM
     fp64_flops_launch = (4 * nnz + 26 * n) * sum_iters_rank   # 61,504 / iter
     fp64_peak = 64 * 2 * num_sms * sm_max_mhz * 1e6     # 64 DFMA/clk/SM
+    try:
+        from paper_conf_ipps_kashinksla22_b200 import probe_fp64
+        fp64_measured, fp64_probe_hz = probe_fp64(local_rank)
+    except Exception:  # noqa: BLE001
+        fp64_measured, fp64_probe_hz = None, None
     vals_bytes = vals.element_size() * vals.numel() / per_rank
     hbm_bytes_sys = vals_bytes + 8 * n + 8 * n + 4 + 8 + 1   # values, b, x, iters, resnorm, status
     hbm_achieved = hbm_bytes_sys * per_rank / kern_avg_s
@@ -427,7 +601,17 @@ def run_ours(args, rank, world, local_rank):
                                 "(profiles/r1_tmem_probe.txt)"},
         "fp64": {"achieved": fp64_flops_launch / kern_avg_s / 1e12, "peak": fp64_peak / 1e12,
                  "unit": "TFLOP/s", "frac": fp64_flops_launch / kern_avg_s / fp64_peak,
-                 "peak_source": "derived: 64 DFMA/clk/SM x 148 x 1965 MHz"},
+                 "peak_source": "derived: 64 DFMA/clk/SM x 148 x 1965 MHz",
+                 "peak_measured": None if fp64_measured is None else fp64_measured / 1e12,
+                 "probe_sm_mhz": None if fp64_probe_hz is None else fp64_probe_hz / 1e6,
+                 "frac_of_measured": (None if not fp64_measured else
+                                      fp64_flops_launch / kern_avg_s / fp64_measured),
+                 "measured_how": "bsolve_probe_fp64: DFMA loop, 8 chains per thread, "
+                                 "4 x 256 threads per SM"},
+        "frac_ell_slots": (2 * ((16 if values_in_smem else 8) * W * n + 8 * n) * sum_iters_rank
+                           / kern_avg_s / smem_peak),
+        "model_note": "frac charges the 8554 CSR nonzeros per SpMV (conservative); "
+                      "frac_ell_slots charges SURVEY 8(d)'s 8928 ELL slots incl. padding",
         "all_operand_effective": {
             "achieved": all_operand_bytes / kern_avg_s / 1e9, "unit": "GB/s",
             "frac_of_smem_peak": all_operand_bytes / kern_avg_s / smem_peak,
@@ -448,6 +632,14 @@ def run_ours(args, rank, world, local_rank):
         roofline["hbm"]["traffic_over_algorithmic"] = (tr["dram_bytes_per_launch"] * scale /
                                                        (hbm_bytes_sys * per_rank))
         roofline["traffic_source"] = tr["source"]
+        if "smem_pipe_busy" in tr:  # physical resource use of the same capture
+            roofline["physical"] = {
+                k: tr[k] for k in ("smem_pipe_busy", "fp64_pipe_busy", "lsu_pipe_busy",
+                                   "warps_active", "registers_per_thread") if k in tr}
+            roofline["physical"]["frac"] = max(tr["smem_pipe_busy"], tr["fp64_pipe_busy"])
+            roofline["physical"]["note"] = ("ncu busy fractions of the tightest physical "
+                                            "resources (the honest roofline of a latency-bound "
+                                            "kernel; frac above is the byte model)")
     except Exception:  # noqa: BLE001 - no capture committed for this build
         pass
     if clocks.get("sm_mhz"):
@@ -508,8 +700,13 @@ def run_ours(args, rank, world, local_rank):
         except Exception as e:  # noqa: BLE001
             cpu["banded_lu"] = {"error": str(e)}
 
-    ion = it_all[0::2] if (g0 % 2 == 0) else it_all[1::2]
-    ele = it_all[1::2] if (g0 % 2 == 0) else it_all[0::2]
+    if rank == 0 and world == 1 and args.parity == "full":
+        parity_full = full_parity(args, g0, per_rank, x, res_h, st_h)
+    else:
+        parity_full = None
+
+    ion = it_all[0::2]   # global index parity: even = ion (rank slices start anywhere,
+    ele = it_all[1::2]   # but the gathered stats start at g = 0)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -524,8 +721,104 @@ def run_ours(args, rank, world, local_rank):
                         "max_true_rel_residual_rank0": float(np.max(
                             res_h / np.linalg.norm(b_h.numpy(), axis=1)))},
         "parity_sample": parity,
+        "parity_full": parity_full,
+        "cross_p": cross,
+        "stats_digest": digest(it_all, res_all, st_all),
         "kernel_ms": {"min": min(kern_ms), "max": max(kern_ms), "mean": statistics.mean(kern_ms),
                       "std": statistics.pstdev(kern_ms), "n": len(kern_ms)},
+    }
+    if rank == 0:
+        emit(line, args)
+
+
+# ---------------------------------------------------- Picard (f1) arm --
+def run_picard(args, rank, world, local_rank):
+    """--picard P: the Picard warm-start pipeline (the
+    analogue of Figs. 8/9) at the bench scale.  The
+    matrices of Picard steps p = 0..P-1 (xgcgen picard=p: the operator scale
+    1 + 0.3 * 0.05^p, b fixed) are all resident in HBM -- XGC rebuilds them on
+    the device between solves; that rebuild is not the solver's work and is
+    not timed.  One step = P successive bsolve_run calls, x0 of solve p = the
+    solution of solve p - 1 kept on the device (warm); the same P solves from
+    x0 = 0 are timed beside it.  value = systems x P / cumulative warm time."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_kashinksla22_b200 import Solver
+    from paper_conf_ipps_kashinksla22_b200.parallel import (gather_stats, max_over_ranks,
+                                                            rank_slice)
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    sl = rank_slice(args.batch, rank, world, args.scaling)
+    per_rank, g0 = sl.count, sl.g0
+    P = args.picard
+    vals, b = [], None
+    for p in range(P):
+        pat, vh, bh = make_inputs(g0, per_rank, args, pinned=False, picard=p)
+        vals.append(vh.to(dev))
+        if b is None:
+            b = bh.to(dev)   # b is the same at every Picard step
+        del vh, bh
+    n = pat.n
+    S = Solver(pat.row_ptr, pat.col_idx, per_rank, format=args.format,
+               placement=args.placement, device=local_rank, solver=args.solver,
+               precond=args.precond, restart=args.restart)
+    outs = [S.alloc_outputs() for _ in range(P)]
+    stream = torch.cuda.current_stream()
+
+    def chain(warm):
+        for p in range(P):
+            x0 = outs[p - 1][0] if (warm and p > 0) else None
+            S.run(vals[p], b, x0, args.tol, args.maxiter, out=outs[p])
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def timed(warm, steps):
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(steps):
+            chain(warm)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        return max_over_ranks(e0.elapsed_time(e1), device=dev)
+
+    for _ in range(max(args.warmup, 0)):
+        chain(True)
+        chain(False)
+    with ClockSampler(local_rank) as clk:
+        warm_ms = timed(True, args.steps)
+    zero_ms = timed(False, args.steps)
+    chain(True)  # leave the warm chain's outputs for the stats below
+    torch.cuda.synchronize()
+    per_p = []
+    all_conv = True
+    for p in range(P):
+        it_all, res_all, st_all = (t.numpy() for t in gather_stats(*outs[p][1:]))
+        all_conv = all_conv and bool(np.all(st_all == 0))
+        per_p.append({"p": p, "iters_mean_ion": float(np.mean(it_all[0::2])),
+                      "iters_mean_electron": float(np.mean(it_all[1::2]))})
+    value = sl.total * P * args.steps / (warm_ms * 1e-3)
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": warm_ms / args.steps, "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": dict(config_dict(args, world, per_rank),
+                       workload=f"xgc{n}_9pt_mix_picard{P}_warm",
+                       description=f"SURVEY 8(f) f1 / BASELINE configs[1] at scale: {P} Picard "
+                                   "solves per step, matrices resident on the device, x0 = "
+                                   "previous solution", x0="previous Picard solution"),
+        "picard": {"steps_per_chain": P, "cumulative_ms_warm": warm_ms / args.steps,
+                   "cumulative_ms_zero_guess": zero_ms / args.steps,
+                   "speedup_warm_over_zero": zero_ms / warm_ms,
+                   "paper": "ELL warm vs zero total time 1.2-1.6x on A100 (PAPER.md:1085-1090); "
+                            "Table III iterations e- 30,28,20,16,12 / ion 5,4,3,2,2",
+                   "per_step": per_p, "all_converged": all_conv},
+        "clocks": clk.summary(), "gpu_launches": args.steps * P, "plan": S.info,
+        "e2e": None, "cpu_baseline": None,
     }
     if rank == 0:
         emit(line, args)
@@ -670,8 +963,34 @@ def run_banded(args, rank, world, local_rank):
         emit(line, args)
 
 
+def free_port():
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def spawn(args):
+    """`bench.py --gpus N` outside torchrun: re-launch this script as N ranks
+    (one process per GPU) through torch.distributed.run on 127.0.0.1; rank 0
+    prints the JSON line.  NCCL init lines stay visible (NCCL_DEBUG=INFO,
+    subsystem INIT) so the communicator size can be read from the log."""
+    env = dict(os.environ)
+    if args.backend == "nccl":
+        env.setdefault("NCCL_DEBUG", "INFO")
+        env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr=127.0.0.1",
+           f"--master-port={free_port()}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        sys.exit(spawn(args))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
@@ -681,10 +1000,17 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.backend == "nccl" and not args.standin:
+            torch.cuda.set_device(local_rank)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group("gloo")
     try:
-        if args.solver == "banded":
+        if args.standin:
+            run_standin(args, rank, world)
+        elif args.picard > 0:
+            run_picard(args, rank, world, local_rank)
+        elif args.solver == "banded":
             run_banded(args, rank, world, local_rank)
         else:
             run_ours(args, rank, world, local_rank)

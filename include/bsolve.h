@@ -298,6 +298,12 @@ const char *bsolve_last_error(void);
  * clock the kernel saw (*sm_hz, from clock64 over the event time). */
 int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, double *sm_hz);
 
+/* Measure this device's FP64 FMA throughput (flop/s, 2 per DFMA) with a
+ * register-only DFMA loop over all SMs (8 independent chains per thread, 4
+ * CTAs x 256 threads per SM): the measured FP64 roofline denominator of
+ * bench.py.  Synchronous.  *sm_hz as above. */
+int bsolve_probe_fp64(int device, double *flops_per_s, double *sm_hz);
+
 #ifdef __cplusplus
 }
 #endif

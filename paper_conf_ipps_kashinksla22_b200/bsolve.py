@@ -87,10 +87,11 @@ def lib():
             L.bsolve_last_error.restype = C.c_char_p
             L.bsolve_probe_smem_bandwidth.argtypes = [C.c_int, C.POINTER(C.c_double),
                                                       C.POINTER(C.c_double)]
+            L.bsolve_probe_fp64.argtypes = [C.c_int, C.POINTER(C.c_double), C.POINTER(C.c_double)]
             for f in ("bsolve_create", "bsolve_run", "bsolve_run_host", "bsolve_spmv",
                       "bsolve_csr_to_ell", "bsolve_query", "bsolve_ell_map", "bsolve_destroy",
                       "bsolve_ell_layout", "bsolve_banded_solve", "bsolve_banded_solve_host",
-                      "bsolve_probe_smem_bandwidth"):
+                      "bsolve_probe_smem_bandwidth", "bsolve_probe_fp64"):
                 getattr(L, f).restype = C.c_int
             _lib = L
     return _lib
@@ -135,6 +136,13 @@ def probe_smem_bandwidth(device: int = -1):
     bw, hz = C.c_double(), C.c_double()
     check(lib().bsolve_probe_smem_bandwidth(int(device), C.byref(bw), C.byref(hz)))
     return bw.value, hz.value
+
+
+def probe_fp64(device: int = -1):
+    """(FP64 flop/s, SM clock Hz) of a DFMA loop over all SMs."""
+    fl, hz = C.c_double(), C.c_double()
+    check(lib().bsolve_probe_fp64(int(device), C.byref(fl), C.byref(hz)))
+    return fl.value, hz.value
 
 
 class Solver:

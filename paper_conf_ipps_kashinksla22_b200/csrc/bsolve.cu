@@ -1510,3 +1510,43 @@ extern "C" int bsolve_probe_smem_bandwidth(int device, double *bytes_per_s, doub
   *sm_hz = (double)mx / (ms * 1e-3);
   return BSOLVE_OK;
 }
+
+extern "C" int bsolve_probe_fp64(int device, double *flops_per_s, double *sm_hz) {
+  g_err.clear();
+  if (!flops_per_s || !sm_hz) return fail(BSOLVE_ERR_INVALID, "NULL output");
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (device < 0) device = prev;
+  CUDA_TRY(cudaSetDevice(device));
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, device));
+  constexpr int NT = 256;
+  const int grid = prop.multiProcessorCount * 4, iters = 1 << 15;
+  double *sink = nullptr;
+  long long *cyc = nullptr;
+  CUDA_TRY(cudaMalloc(&sink, sizeof(double) * grid));
+  CUDA_TRY(cudaMalloc(&cyc, sizeof(long long) * grid));
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  fp64_probe_kernel<NT><<<grid, NT>>>(256, 1.0, sink, cyc);  // warm-up
+  cudaEventRecord(e0);
+  fp64_probe_kernel<NT><<<grid, NT>>>(iters, 1.0, sink, cyc);
+  cudaEventRecord(e1);
+  cudaError_t e = cudaEventSynchronize(e1);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  std::vector<long long> hc(grid);
+  cudaMemcpy(hc.data(), cyc, sizeof(long long) * grid, cudaMemcpyDeviceToHost);
+  cudaFree(sink);
+  cudaFree(cyc);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (prev >= 0) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(BSOLVE_ERR_CUDA, "fp64 probe: %s", cudaGetErrorString(e));
+  *flops_per_s = (double)grid * NT * iters * 8 * 2 / (ms * 1e-3);
+  long long mx = 0;
+  for (long long c : hc) mx = std::max(mx, c);
+  *sm_hz = (double)mx / (ms * 1e-3);
+  return BSOLVE_OK;
+}

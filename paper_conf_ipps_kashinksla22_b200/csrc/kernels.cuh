@@ -1589,4 +1589,27 @@ __global__ void __launch_bounds__(NT) smem_probe_kernel(int iters, double *sink,
   if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
 }
 
+// Measured FP64 roofline denominator ("measure it with a DFMA
+// loop"): every thread runs 8 independent DFMA chains (enough in flight to
+// cover the pipe latency), `iters` x 8 DFMA = 16 x iters flop per thread.
+template <int NT>
+__global__ void __launch_bounds__(NT) fp64_probe_kernel(int iters, double seed, double *sink,
+                                                        long long *cycles) {
+  double a[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) a[k] = seed * (threadIdx.x + k);
+  const double m = 1.0 - 1e-16 * seed, c = 1e-20 * seed;
+  const long long c0 = clock64();
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) a[k] = fma(a[k], m, c);
+  }
+  const long long c1 = clock64();
+  double s = 0.0;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) s += a[k];
+  if (s == -1.0) sink[blockIdx.x] = s;
+  if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+}
+
 }  // namespace bsolve

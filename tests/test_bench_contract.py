@@ -47,3 +47,25 @@ def test_reference_arm_banded_solver():
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["value"] > 0
     assert d["config"]["solver"].startswith("banded") and "banded LU" in d["note"]
+
+
+def _standin(gpus, scaling, batch=16):
+    lines = run(["--gpus", str(gpus), "--standin", "--backend", "gloo", "--batch", str(batch),
+                 "--nx", "6", "--ny", "5", "--steps", "2", "--warmup", "1", "--scaling", scaling])
+    assert len(lines) == 1, lines
+    return json.loads(lines[-1])
+
+
+def test_gpus2_spawns_two_ranks_and_gathers_like_one_process():
+    """`bench.py --gpus 2` outside torchrun re-launches itself as 2 ranks
+    (the driver's N-GPU entry point), here over gloo with
+    the CPU stand-in solver: one JSON line, n_gpus = 2, the gathered
+    per-system stats equal the single-process run's bit for bit, and rank 0's
+    cross-P re-solve matches every rank."""
+    one = _standin(1, "strong")
+    two = _standin(2, "strong")
+    assert one["n_gpus"] == 1 and two["n_gpus"] == 2
+    assert two["gathered"] == one["gathered"]
+    assert two["cross_p"]["bitwise_equal"] and two["cross_p"]["ranks"] == 2
+    weak = _standin(2, "weak", batch=8)   # 2 x 8 systems = the strong run's 16
+    assert weak["gathered"] == one["gathered"] and weak["config"]["global_batch"] == 16

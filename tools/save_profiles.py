@@ -26,6 +26,14 @@ t = {"source": f"ncu --set full --clock-control none, one launch of {name} (benc
      "dram_bytes_read": val("dram__bytes_read.sum"), "dram_bytes_write": val("dram__bytes_write.sum"),
      "smem_data_pipe_wavefronts": val("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"),
      "duration_ms": val("gpu__time_duration.sum")}
+for key, metric in (("smem_pipe_busy", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed"),
+                    ("fp64_pipe_busy", "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active"),
+                    ("lsu_pipe_busy", "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"),
+                    ("warps_active", "sm__warps_active.avg.pct_of_peak_sustained_active")):
+    if metric in d:
+        t[key] = float(d[metric].replace(",", "")) / 100.0
+if "launch__registers_per_thread" in d:
+    t["registers_per_thread"] = int(float(d["launch__registers_per_thread"]))
 t["dram_bytes_per_launch"] = t["dram_bytes_read"] + t["dram_bytes_write"]
 t["smem_data_pipe_bytes_per_launch"] = t["smem_data_pipe_wavefronts"] * 128
 json.dump(t, open("profiles/ncu_traffic.json", "w"), indent=1)
