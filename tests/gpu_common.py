@@ -4,6 +4,10 @@ north_star (DESIGN.md "Parity bar"):
   * true relative residual ||b - A x|| / ||b|| <= 1e-10 (REL_B, tol 1e-10)
   * ||x - x_direct|| / ||x_direct|| <= 1e-8 against the oracle's banded LU
   * |iters_gpu - iters_oracle| <= 2 against the oracle's Algorithm 1
+    (kappa >= 1e3: the count is chaotic in the rounding -- one ulp of input
+    perturbation moves the ORACLE's own count by up to 25-68 iterations -- so
+    it is compared as a distribution against that ulp spread, R28,
+    iter_spread_ok below)
   * identical status
 """
 import numpy as np
@@ -50,8 +54,9 @@ def compare(row_ptr, col_idx, csr_values, b, g, o=None, xd=None, res_tol=RES_TOL
     batch = csr_values.shape[0]
     bn = np.linalg.norm(b, axis=1)
     assert np.array_equal(g["status"], o["status"]), (g["status"], o["status"])
-    di = np.abs(g["iters"].astype(int) - o["iters"].astype(int))
-    assert di.max() <= iter_tol, f"iteration mismatch max {di.max()}"
+    if iter_tol is not None:  # None: kappa >= 1e3 sets, compared as a distribution (R28)
+        di = np.abs(g["iters"].astype(int) - o["iters"].astype(int))
+        assert di.max() <= iter_tol, f"iteration mismatch max {di.max()}"
     conv = g["status"] == 0
     ok_b = bn > 0
     rel = np.where(ok_b, g["resnorm"] / np.where(ok_b, bn, 1), g["resnorm"])
@@ -67,3 +72,24 @@ def compare(row_ptr, col_idx, csr_values, b, g, o=None, xd=None, res_tol=RES_TOL
             if nrm > 0:
                 assert np.linalg.norm(g["x"][i] - xd[i]) / nrm <= fwd_tol, i
     return o, xd
+
+
+def perturb_ulp(vals, seed=0):
+    """Every value times (1 +- 2^-52), random sign: one ulp of input noise."""
+    rng = np.random.default_rng(seed)
+    return vals * (1.0 + rng.choice([-1.0, 1.0], size=vals.shape) * 2.0 ** -52)
+
+
+def iter_spread_ok(gi, oi, ui, slack=0.1):
+    """DESIGN.md R28: the GPU-vs-oracle iteration differences must be no wider
+    than the oracle-vs-oracle(ulp-perturbed input) differences: the fraction
+    within +-2 at most `slack` lower, the median |difference| at most 1
+    higher, the 90% quantile at most 2 x higher (+2)."""
+    dg = np.abs(gi.astype(int) - oi.astype(int))
+    du = np.abs(ui.astype(int) - oi.astype(int))
+    fg, fu = np.mean(dg <= 2), np.mean(du <= 2)
+    ok = (fg >= fu - slack and np.median(dg) <= np.median(du) + 1 and
+          np.quantile(dg, 0.9) <= 2 * np.quantile(du, 0.9) + 2)
+    return ok, dict(frac_within2_gpu=float(fg), frac_within2_ulp=float(fu),
+                    median_gpu=float(np.median(dg)), median_ulp=float(np.median(du)),
+                    q90_gpu=float(np.quantile(dg, 0.9)), q90_ulp=float(np.quantile(du, 0.9)))

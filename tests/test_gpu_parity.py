@@ -182,18 +182,37 @@ def test_no_true_residual_check():
 
 @pytest.mark.parametrize("placement", ["smem", "regs"])
 def test_ill_conditioned_guard(placement):
-    """configs[4] flavour: kappa ~ 1e3..1e5 electrons (R18): the
-    iteration count is chaotic in the summation order at this conditioning,
-    so parity is x vs the direct solve (1e-8), the TRUE residual (<= tau) and
-    the status; iterations agree within 50% of the oracle's."""
+    """configs[4] flavour: kappa ~ 1e3..1e5 electrons (R18): x vs
+    the direct solve (1e-8), the TRUE residual (<= tau) and the status per
+    system; the iteration count is compared as a distribution (R28,
+    test_ill_conditioned_iteration_spread)."""
     for margin in (1e-1, 1e-2, 1e-3):
         ill = X.Species(X.ELECTRON_K, cross=0.0, margin=margin)
         B = X.make_batch(1, 8, electron=ill)
         p = B.pattern
         g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000, placement=placement)
         o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=2000)
-        compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o,
-                iter_tol=max(10, int(0.5 * o["iters"].max())))
+        compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, iter_tol=None)
+
+
+@pytest.mark.parametrize("margin", [1e-1, 1e-2, 1e-3])
+def test_ill_conditioned_iteration_spread(margin):
+    """DESIGN.md R28: on 300 ill-conditioned electrons (cross = 0, kappa ~
+    1.2e3 / 1.4e4 / 1.4e5) every system passes the per-system bar (status,
+    TRUE residual <= 1e-10, ||x - x_direct|| <= 1e-8) and the GPU-vs-oracle
+    iteration differences are no wider than what ONE ulp of input noise does
+    to the oracle itself (gpu_common.iter_spread_ok)."""
+    from gpu_common import iter_spread_ok, perturb_ulp
+    ill = X.Species(X.ELECTRON_K, cross=0.0, margin=margin)
+    B = X.make_batch(1, 600, electron=ill)
+    p = B.pattern
+    vals, b = B.values[0::2].copy(), B.b[0::2].copy()   # the electrons (odd g)
+    g = gpu_solve(p.row_ptr, p.col_idx, vals, b, maxiter=3000)
+    o = O.batch_bicgstab(p.row_ptr, p.col_idx, vals, b, maxiter=3000)
+    u = O.batch_bicgstab(p.row_ptr, p.col_idx, perturb_ulp(vals), b, maxiter=3000)
+    compare(p.row_ptr, p.col_idx, vals, b, g, o=o, iter_tol=None)
+    ok, info = iter_spread_ok(g["iters"], o["iters"], u["iters"])
+    assert ok, info
 
 
 # ------------------------------------------------- invariants on the GPU --
@@ -393,15 +412,13 @@ def test_cluster_warm_start_ill_conditioned_and_deterministic():
     p = pat
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3000)
     o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, maxiter=3000)
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o,
-            iter_tol=max(10, int(0.5 * o["iters"].max())))
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, iter_tol=None)  # R28
     # warm start from a perturbed direct solution
     xd = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b)
     x0 = xd * (1 + 1e-5)
     g2 = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3000)
     o2 = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3000)
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g2, o=o2, xd=xd,
-            iter_tol=max(10, int(0.5 * o2["iters"].max())))
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g2, o=o2, xd=xd, iter_tol=None)  # R28
     # bitwise identical across runs and batch slicing
     g3 = gpu_solve(p.row_ptr, p.col_idx, B.values[3:], B.b[3:], maxiter=3000)
     for k in ("x", "iters", "resnorm", "status"):

@@ -1,13 +1,29 @@
-import re, sys
-lines = open(sys.argv[1]).read().split('\n')
-cur=None
-for l in lines:
-    m = re.search(r"Compiling entry function '(\S+)'", l)
-    if m: cur = m.group(1); spill=''; continue
-    m = re.search(r"(\d+) bytes spill stores, (\d+) bytes spill loads", l)
-    if m and cur: spill = f"spill {m.group(1)}/{m.group(2)}"
-    m = re.search(r"Used (\d+) registers", l)
+"""ptxas register / spill table of every kernel in a verbose build log:
+  python -c "from paper_conf_ipps_kashinksla22_b200 import _build; _build.build(force=True, verbose=True)" > build.log
+  python tools/ptxas_table.py build.log"""
+import re
+import subprocess
+import sys
+
+rows, cur, spill = [], None, ""
+for line in open(sys.argv[1]).read().split("\n"):
+    m = re.search(r"Compiling entry function '(\S+)'", line)
+    if m:
+        cur, spill, stack = m.group(1), "", ""
+        continue
+    m = re.search(r"(\d+) bytes stack frame, (\d+) bytes spill stores, (\d+) bytes spill loads", line)
     if m and cur:
-        k = re.search(r"bicgstab_kernelILi(\d)ELi(\d)ELi(\d+)ELb[01]ELi(\d)ELi(\d+)", cur)
-        if k: print(f"fmt={k.group(1)} place={k.group(2)} WB={k.group(3)} R={k.group(4)} NT={k.group(5)}: regs {m.group(1)} {spill}")
-        cur=None
+        stack, spill = m.group(1), f"{m.group(2)}/{m.group(3)}"
+    m = re.search(r"Used (\d+) registers", line)
+    if m and cur:
+        rows.append((cur, int(m.group(1)), spill, stack))
+        cur = None
+names = subprocess.run(["c++filt"], input="\n".join(r[0] for r in rows), capture_output=True,
+                       text=True).stdout.split("\n")
+seen = set()
+print(f"{'regs':>4s} {'spill st/ld B':>13s} {'stack B':>7s}  kernel")
+for (mangled, regs, spill, stack), name in sorted(zip(rows, names), key=lambda t: t[1]):
+    if name in seen:
+        continue
+    seen.add(name)
+    print(f"{regs:4d} {spill:>13s} {stack:>7s}  {name[:150]}")
