@@ -27,6 +27,12 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 STOP_REL_B = 0
 STOP_ABS = 1
 PREC_JACOBI, PREC_NONE = 0, 1
+PREC_BLOCK_JACOBI = 2  # blocks of 8 consecutive rows; block_jacobi(bs) for other sizes
+
+
+def block_jacobi(bs: int = 8) -> int:
+    """precond code of block-Jacobi with blocks of bs consecutive rows (R30)."""
+    return PREC_BLOCK_JACOBI | (int(bs) << 8)
 SOLVER_BICGSTAB, SOLVER_GMRES = 0, 2
 CONVERGED, MAXITER, BREAKDOWN = 0, 1, 2
 
@@ -89,6 +95,8 @@ def lib():
             L.oracle_batch_banded.argtypes = [C.c_int, C.c_int, C.c_int, _P, _P, _P, _P, _P,
                                               _P, C.c_int]
             L.oracle_batch_banded.restype = C.c_int
+            L.oracle_precond_apply.argtypes = [C.c_int, _P, _P, _P, C.c_int, _P, _P]
+            L.oracle_precond_apply.restype = C.c_int
             _lib = L
     return _lib
 
@@ -172,6 +180,16 @@ def bicgstab(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, stop=ST
     return x, R
 
 
+def precond_apply(row_ptr, col_idx, val, y, precond=PREC_JACOBI):
+    """M^-1 y for one system (the preconditioner alone, oracle.c precond_apply)."""
+    rp, ci, v, yy = _i32(row_ptr), _i32(col_idx), _f64(val), _f64(y)
+    out = np.empty(rp.size - 1)
+    if lib().oracle_precond_apply(rp.size - 1, _ptr(rp), _ptr(ci), _ptr(v), int(precond),
+                                  _ptr(yy), _ptr(out)):
+        raise MemoryError("oracle_precond_apply")
+    return out
+
+
 def batch_bicgstab(row_ptr, col_idx, values, b, x0=None, tol=1e-10, maxiter=1000,
                    stop=STOP_REL_B, true_res_check=True, threads=0):
     """Alg. 1 on every system (values [batch, nnz] CSR order).
@@ -229,8 +247,8 @@ def gmres(row_ptr, col_idx, val, b, x0=None, tol=1e-10, maxiter=1000, restart=8,
 def batch_krylov(row_ptr, col_idx, values, b, solver=SOLVER_BICGSTAB, precond=PREC_JACOBI,
                  restart=8, x0=None, tol=1e-10, maxiter=1000, stop=STOP_REL_B,
                  true_res_check=True, threads=0):
-    """BiCGSTAB or GMRES(restart) with Jacobi or no preconditioner on every
-    system.  Returns dict(x, iters, resnorm, status, restarts)."""
+    """BiCGSTAB or GMRES(restart) with Jacobi, block-Jacobi (R30) or no
+    preconditioner on every system.  Returns dict(x, iters, resnorm, status, restarts)."""
     rp, ci, v, bb = _i32(row_ptr), _i32(col_idx), _f64(values), _f64(b)
     batch, nnz = v.shape
     n = rp.size - 1
