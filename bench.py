@@ -54,7 +54,8 @@ def parse():
     ap.add_argument("--solver", choices=["bicgstab", "gmres", "banded"], default="bicgstab",
                     help="BiCGSTAB = the paper's Algorithm 1; gmres = f3; banded = the "
                          "dgbsv-analogue direct solver (SURVEY.md 8(f) f4)")
-    ap.add_argument("--precond", choices=["jacobi", "none"], default="jacobi")
+    ap.add_argument("--precond", choices=["jacobi", "none", "block_jacobi"], default="jacobi",
+                    help="block_jacobi: 8-row blocks (SURVEY.md 8(f) f3, DESIGN.md R30)")
     ap.add_argument("--restart", type=int, default=7, help="GMRES restart length m")
     ap.add_argument("--tol", type=float, default=1e-10)
     ap.add_argument("--maxiter", type=int, default=1000)
@@ -206,14 +207,17 @@ def oracle_krylov(O, pat, B, args, cores):
     """The oracle's solver for this run's --solver / --precond / --restart."""
     return O.batch_krylov(pat.row_ptr, pat.col_idx, B.values, B.b,
                           solver=O.SOLVER_GMRES if args.solver == "gmres" else O.SOLVER_BICGSTAB,
-                          precond=O.PREC_NONE if args.precond == "none" else O.PREC_JACOBI,
+                          precond={"none": O.PREC_NONE, "jacobi": O.PREC_JACOBI,
+                                   "block_jacobi": O.block_jacobi(8)}[args.precond],
                           restart=args.restart, tol=args.tol, maxiter=args.maxiter, threads=cores)
 
 
 def oracle_algorithm(args):
     name = ("GMRES(%d)" % args.restart if args.solver == "gmres"
             else "Alg. 1 BiCGSTAB")
-    return f"{name} + {'Jacobi' if args.precond == 'jacobi' else 'no preconditioner'} (oracle/oracle.c)"
+    pre = {"jacobi": "Jacobi", "none": "no preconditioner",
+           "block_jacobi": "block-Jacobi(8)"}[args.precond]
+    return f"{name} + {pre} (oracle/oracle.c)"
 
 
 def oracle_sample_rate(g0, max_count, args, target_s, kind="bicgstab"):

@@ -107,10 +107,16 @@ enum {
 };
 #define BSOLVE_MAX_RESTART 7
 
-/* Preconditioner M^-1 = diag(d) applied on the right. */
+/* Preconditioner M^-1 applied on the right. */
 enum {
   BSOLVE_PREC_JACOBI = 0, /* d_i = 1 / a_ii (a zero diagonal gives 1)          */
-  BSOLVE_PREC_NONE = 1    /* d_i = 1                                           */
+  BSOLVE_PREC_NONE = 1,   /* d_i = 1                                           */
+  BSOLVE_PREC_BLOCK_JACOBI = 2 /* M = block diagonal of A with
+                              blocks of 8 consecutive rows, each solved exactly
+                              (R30).  BiCGSTAB on the line-tiled TMEM
+                              plan only (2D 9-point stencils, grid width 31 or
+                              32, n <= 1024, where every block is tridiagonal);
+                              UNSUPPORTED elsewhere                           */
 };
 
 /* Per-system outcome written to status[] (R10). */

@@ -21,7 +21,7 @@ FMT_AUTO, FMT_CSR, FMT_ELL = 0, 1, 2
 PLACE_AUTO, PLACE_SMEM, PLACE_STREAM, PLACE_REGS, PLACE_CLUSTER, PLACE_TMEM = 0, 1, 2, 3, 4, 5
 STOP_REL_B, STOP_ABS = 0, 1
 SOLVER_BICGSTAB, SOLVER_GMRES = 0, 1
-PREC_JACOBI, PREC_NONE = 0, 1
+PREC_JACOBI, PREC_NONE, PREC_BLOCK_JACOBI = 0, 1, 2
 MAX_RESTART = 7
 SYS_CONVERGED, SYS_MAXITER, SYS_BREAKDOWN, SYS_DIRECT = 0, 1, 2, 3
 
@@ -30,7 +30,7 @@ _PLACE = {"auto": PLACE_AUTO, "smem": PLACE_SMEM, "stream": PLACE_STREAM, "regs"
           "cluster": PLACE_CLUSTER, "tmem": PLACE_TMEM}
 _STOP = {"rel_b": STOP_REL_B, "rel": STOP_REL_B, "abs": STOP_ABS}
 _SOLVER = {"bicgstab": SOLVER_BICGSTAB, "gmres": SOLVER_GMRES}
-_PREC = {"jacobi": PREC_JACOBI, "none": PREC_NONE}
+_PREC = {"jacobi": PREC_JACOBI, "none": PREC_NONE, "block_jacobi": PREC_BLOCK_JACOBI}
 
 
 class BsolveError(RuntimeError):
@@ -150,7 +150,8 @@ class Solver:
 
     Solver(row_ptr, col_idx, batch, format="ell", placement="auto",
            stop="rel_b", true_residual_check=True, device=None,
-           solver="bicgstab" | "gmres", precond="jacobi" | "none", restart=7,
+           solver="bicgstab" | "gmres",
+           precond="jacobi" | "none" | "block_jacobi" (8-row blocks, R30), restart=7,
            direct_fallback=False)
     .run(values, b, x0=None, tol=1e-10, maxiter=1000) -> (x, iters, resnorm, status)
     """

@@ -343,8 +343,11 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     return fail(BSOLVE_ERR_INVALID, "reg_slots must be 0, 2, 4, 6 or 8 (got %d)", opt.reg_slots);
   if (opt.solver != BSOLVE_SOLVER_BICGSTAB && opt.solver != BSOLVE_SOLVER_GMRES)
     return fail(BSOLVE_ERR_INVALID, "bad solver %d", opt.solver);
-  if (opt.precond != BSOLVE_PREC_JACOBI && opt.precond != BSOLVE_PREC_NONE)
+  if (opt.precond != BSOLVE_PREC_JACOBI && opt.precond != BSOLVE_PREC_NONE &&
+      opt.precond != BSOLVE_PREC_BLOCK_JACOBI)
     return fail(BSOLVE_ERR_INVALID, "bad preconditioner %d", opt.precond);
+  if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && opt.solver != BSOLVE_SOLVER_BICGSTAB)
+    return fail(BSOLVE_ERR_UNSUPPORTED, "block-Jacobi is implemented for BiCGSTAB only");
   if (opt.solver == BSOLVE_SOLVER_GMRES && (opt.restart < 1 || opt.restart > BSOLVE_MAX_RESTART))
     return fail(BSOLVE_ERR_INVALID, "GMRES restart must be 1..%d (got %d)", BSOLVE_MAX_RESTART,
                 opt.restart);
@@ -565,6 +568,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   {
     const char *lenv = getenv("BSOLVE_TMEM_LINE");
     const bool gm = opt.solver == BSOLVE_SOLVER_GMRES;
+    const bool bj = opt.precond == BSOLVE_PREC_BLOCK_JACOBI;
     const bool line_on = (gm || !(lenv && atoi(lenv) == 0)) && opt.block_threads == 0 &&
                          opt.reg_slots == 0 && h->kfmt == FMT_DIA && W <= 9 && n <= 1024 &&
                          h->place != PLACE_CLUSTER &&
@@ -587,9 +591,11 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
       const LVariant &cand = lv[i % lcnt];
       if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
-      if (!gm && cand.rounds != lrounds) continue;
+      if (!gm && !bj && cand.rounds != lrounds) continue;
+      if (cand.pre != (bj ? 1 : 0)) continue;
+      if (bj && i >= lcnt) continue;  // block-Jacobi: the 3-CTA kernel only
       if (i < lcnt) {
-        if (cand.ctas != lctas) continue;
+        if (!bj && cand.ctas != lctas) continue;
         if (lctas == 2 && (cand.g != lg || cand.r != lr)) continue;
       } else if (cand.ctas != 2) {
         continue;
@@ -613,6 +619,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
     }
   }
+  if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && !line_v)
+    return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                          "block-Jacobi needs the line-tiled plan: a 2D 9-point stencil on a grid "
+                          "of width 31 or 32, n <= 1024, placement AUTO or TMEM"));
   if (opt.solver == BSOLVE_SOLVER_GMRES && !line_v)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "GMRES needs a 2D stencil pattern (9- or 5-point, grid width 31 or "

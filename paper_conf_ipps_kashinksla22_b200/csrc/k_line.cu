@@ -18,7 +18,10 @@ using namespace bsolve;
 // one FMA chain per row, a shallower one-value reduction, gathers one row
 // ahead -- DESIGN.md perf log.)
 #define LV3_(NX, RD) {NX, 8, 3, SOLVER_BICGSTAB, Line3Geom<NX>::SMEM_BYTES, RD, \
-                      (solve_fn)bicgstab_line3_kernel<NX, RD>, 3}
+                      (solve_fn)bicgstab_line3_kernel<NX, RD>, 3, 0}
+// block-Jacobi preconditioner, one 8-row tridiagonal block per thread (f3, R30)
+#define LV3B_(NX) {NX, 8, 3, SOLVER_BICGSTAB, Line3Geom<NX, 1>::SMEM_BYTES, 2, \
+                   (solve_fn)bicgstab_line3_kernel<NX, 2, 1>, 3, 1}
 // two reduction rounds per iteration (deferred stop test 1, algebraic rho)
 #define LV2_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 2, \
                         (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB, 2, 2>, 2}
@@ -30,7 +33,8 @@ static const LVariant kLVariants[] = {LV_(32, 8, 2),  LV_(32, 8, 4),  LV_(32, 4,
                                       LV_(32, 4, 4),  LV_(31, 8, 4),  LV_(31, 4, 2),
                                       LVG_(32, 8, 2), LVG_(31, 8, 2), LV2_(32, 8, 4),
                                       LV2_(31, 8, 4), LV3_(32, 2),    LV3_(31, 2),
-                                      LV3_(32, 3),    LV3_(31, 3)};
+                                      LV3_(32, 3),    LV3_(31, 3),    LV3B_(32),
+                                      LV3B_(31)};
 
 const LVariant *variants_line(int *count) {
   *count = (int)(sizeof(kLVariants) / sizeof(kLVariants[0]));

@@ -34,7 +34,8 @@ enum { FMT_CSR = 1, FMT_ELL = 2, FMT_DIA = 3 };
 enum { PLACE_SMEM = 1, PLACE_STREAM = 2, PLACE_REGS = 3, PLACE_CLUSTER = 4, PLACE_TMEM = 5 };
 enum { STOP_REL_B = 0, STOP_ABS = 1 };
 enum { SYS_CONVERGED = 0, SYS_MAXITER = 1, SYS_BREAKDOWN = 2 };
-enum { PREC_JACOBI = 0, PREC_NONE = 1 };     // PRECOND(y) = d .* y
+enum { PREC_JACOBI = 0, PREC_NONE = 1,       // PRECOND(y) = d .* y
+       PREC_BLOCK_JACOBI = 2 };               // 8-row blocks, line3 kernel only (R30)
 enum { SOLVER_BICGSTAB = 0, SOLVER_GMRES = 1 };
 constexpr int kMaxW = 16;
 constexpr int kMaxRestart = 7;  // GMRES: CGS2 pass 2 reduces kMaxRestart + 1 <= 8 values at once

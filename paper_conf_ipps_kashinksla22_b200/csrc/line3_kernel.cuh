@@ -29,14 +29,16 @@
 namespace bsolve {
 
 // SMEM layout of one CTA: [gather planes R*S][reduction scratch 16*NWARP]
-// [x: R*NT][2 TMEM base slots].
-template <int NX>
+// [x: R*NT][PRE = 1: block-Jacobi factors 22*NT][2 TMEM base slots].
+template <int NX, int PRE = 0>
 struct Line3Geom {
   static constexpr int R = 8, NT = 128, NWARP = 4;
   using L = LineGeom<NX, NT, R>;
   static constexpr int OFF_RED = R * L::S;
   static constexpr int OFF_X = ((OFF_RED + 16 * NWARP) + 1) & ~1;  // 16-byte aligned
-  static constexpr int SMEM_BYTES = (OFF_X + R * NT) * 8 + 16;
+  static constexpr int OFF_F = OFF_X + R * NT;
+  static constexpr int NF = PRE ? 22 : 0;  // l_1..7, 1/u_0..7, a_(j,j+1) j = 0..6
+  static constexpr int SMEM_BYTES = (OFF_F + NF * NT) * 8 + 16;
 };
 
 __device__ __forceinline__ void tmem_ld2(uint32_t taddr, uint32_t (&r)[2]) {
@@ -99,16 +101,25 @@ __device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const do
   }
 }
 
-template <int NX, int ROUNDS = 2>
+// PRE = 0: PRECOND(y) = d .* y (scalar Jacobi, or none).
+// PRE = 1: block-Jacobi with one block per thread = its 8 consecutive rows
+// (R30).  On an NX >= 9 wide 9-point grid the
+// block A[8t..8t+7, 8t..8t+7] is tridiagonal (only the +-1 couplings fall
+// inside it); it is factored once per system without pivoting (Thomas,
+// l_j = a_(j,j-1) / u_(j-1), u_j = a_jj - l_j a_(j-1,j); a zero or non-finite
+// pivot makes the block the identity) into thread-private SMEM, and every
+// application is a forward and a back substitution in registers.
+template <int NX, int ROUNDS = 2, int PRE = 0>
 __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParams P) {
-  using G3 = Line3Geom<NX>;
+  using G3 = Line3Geom<NX, PRE>;
   constexpr int R = G3::R, NT = G3::NT;
   using L = typename G3::L;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double *sg = reinterpret_cast<double *>(smem_raw);
   double *sred = sg + G3::OFF_RED;
   double2 *sx2 = reinterpret_cast<double2 *>(sg + G3::OFF_X) + threadIdx.x;  // x pair k at [k*NT]
-  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + G3::OFF_X + R * NT);
+  double *sf = sg + G3::OFF_F + threadIdx.x;  // block-Jacobi factor k at sf[k * NT]
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + G3::OFF_F + G3::NF * NT);
 
   const int tid = threadIdx.x, warp = tid >> 5;
   const int n = P.n;
@@ -160,6 +171,7 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
 
   // ---- this thread's rows: values -> TMEM, diagonal -> TMEM + d ------------
   double d[R];
+  double bdiag[PRE ? R : 1], blo[PRE ? R : 1], bup[PRE ? R : 1];  // block-Jacobi block
   {
     const bool vec = ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
                      row0 + R <= n;
@@ -201,11 +213,35 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
         }
         tmem_st16(tval + 16 * (j + h), w);
         d[j + h] = jacobi_inv(P.precond, a0p[h]);
+        if constexpr (PRE == 1) {  // canonical offsets 3 = -1, 4 = +1 (line_kernel.cuh)
+          bdiag[j + h] = a0p[h];
+          blo[j + h] = vv[h][3];
+          bup[j + h] = vv[h][4];
+        }
         aw[2 * (j + h)] = static_cast<uint32_t>(__double2loint(a0p[h]));
         aw[2 * (j + h) + 1] = static_cast<uint32_t>(__double2hiint(a0p[h]));
       }
     }
     tmem_st16(ta0, aw);
+  }
+  if constexpr (PRE == 1) {
+    // Thomas factorisation of the thread's tridiagonal block (rows >= n: the
+    // identity, so their entries stay 0)
+    double l[R], u[R];
+    bool ok = true;
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const bool a = act[j];
+      l[j] = (j > 0 && a) ? blo[j] / u[j - 1] : 0.0;
+      u[j] = a ? bdiag[j] - l[j] * (j > 0 ? bup[j - 1] : 0.0) : 1.0;
+      ok = ok && u[j] != 0.0 && isfinite(u[j]) && isfinite(l[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      if (j > 0) sf[(j - 1) * NT] = ok ? l[j] : 0.0;
+      sf[(7 + j) * NT] = ok ? 1.0 / u[j] : 1.0;
+      if (j < R - 1) sf[(15 + j) * NT] = (ok && act[j + 1]) ? bup[j] : 0.0;
+    }
   }
   const double *bsys = P.b + sys * n;
   double r[R], p[R], v[R];
@@ -244,6 +280,15 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
     tmem_ld16(trh, w);
     tmem_wait_ld();
     tmem_regs_ready(w);
+  };
+  // z = M^-1 y for the thread's block (PRE = 1): forward then back substitution
+  auto bj_apply = [&](const double(&y)[R], double(&z)[R]) {
+    z[0] = y[0];
+#pragma unroll
+    for (int j = 1; j < R; ++j) z[j] = fma(-sf[(j - 1) * NT], z[j - 1], y[j]);
+    z[R - 1] = z[R - 1] * sf[(7 + R - 1) * NT];
+#pragma unroll
+    for (int j = R - 2; j >= 0; --j) z[j] = fma(-sf[(15 + j) * NT], z[j + 1], z[j]) * sf[(7 + j) * NT];
   };
 
   // ---- a3: x = x0 (or 0), r = b - A x0, r^ = r, ||b|| ----------------------
@@ -323,14 +368,24 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
         // R2: beta = (rho / rho') (alpha / omega), the division done after the
         // previous omega; ROUNDS == 2 keeps beta itself in beta_c (R29)
         const double beta = ROUNDS == 2 ? beta_c : rho * beta_c;
-        // a5: p = r + beta (p - omega v); publish p^ = d p
+        // a5: p = r + beta (p - omega v); publish p^ = PRECOND(p)
+        double ph[PRE ? R : 1];  // block-Jacobi: p^ (scalar Jacobi recomputes d p)
+        if constexpr (PRE == 1) {
 #pragma unroll
-        for (int j = 0; j < R; ++j) {
-          p[j] = r[j] + beta * (p[j] - omega * v[j]);
-          comm.publish(j, d[j] * p[j]);
+          for (int j = 0; j < R; ++j) p[j] = r[j] + beta * (p[j] - omega * v[j]);
+          bj_apply(p, ph);
+#pragma unroll
+          for (int j = 0; j < R; ++j) comm.publish(j, ph[j]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < R; ++j) {
+            p[j] = r[j] + beta * (p[j] - omega * v[j]);
+            comm.publish(j, d[j] * p[j]);
+          }
         }
         comm.sync();
-        spmv(d, p, v);                                      // a6: v = A p^
+        if constexpr (PRE == 1) spmv(one, ph, v);           // a6: v = A p^
+        else spmv(d, p, v);
         ++it;
         double rv[1];
         {
@@ -341,11 +396,27 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
         comm.template sum<1>(rv);                           // a7: r^.v
         if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
         alpha = rho / rv[0];                                // R3
-        // s = r - alpha v (kept in r); publish s^ = d s
+        // s = r - alpha v (kept in r); publish s^ = PRECOND(s)
+        double sh[PRE ? R : 1];
+        if constexpr (PRE == 1) {
+          // x + alpha p^ now (p^ dies here): the first half of x's update, in
+          // the oracle's order (x + alpha p^) + omega s^, and stop test 2's x
+          double xx[R];
+          x_load(xx);
 #pragma unroll
-        for (int j = 0; j < R; ++j) {
-          r[j] = r[j] - alpha * v[j];
-          comm.publish(j, d[j] * r[j]);
+          for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * ph[j];
+          x_store(xx);
+#pragma unroll
+          for (int j = 0; j < R; ++j) r[j] = r[j] - alpha * v[j];
+          bj_apply(r, sh);
+#pragma unroll
+          for (int j = 0; j < R; ++j) comm.publish(j, sh[j]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < R; ++j) {
+            r[j] = r[j] - alpha * v[j];
+            comm.publish(j, d[j] * r[j]);
+          }
         }
         comm.sync();
         // ROUNDS == 3: t.s, t.t, s.s here and ||r||^2, r^.r in a third round.
@@ -362,7 +433,8 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
           ts[3] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * r[j]; });
         }
         double t[R];
-        spmv(d, r, t);                                      // a9: t = A s^ (speculative)
+        if constexpr (PRE == 1) spmv(one, sh, t);           // a9: t = A s^ (speculative)
+        else spmv(d, r, t);
         ts[0] = rows_sum<R>([&](int j) { return t[j] * r[j]; });
         ts[1] = rows_sum<R>([&](int j) { return t[j] * t[j]; });
         if constexpr (ROUNDS == 2) {
@@ -372,11 +444,13 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
         }
         comm.template sum<KT>(ts);
         if (below(ts[2])) {                                 // stop test 2
-          double xx[R];
-          x_load(xx);
+          if constexpr (PRE == 0) {  // (block-Jacobi: x + alpha p^ is stored already)
+            double xx[R];
+            x_load(xx);
 #pragma unroll
-          for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]);
-          x_store(xx);
+            for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]);
+            x_store(xx);
+          }
           exit_kind = 2;
           break;
         }
@@ -387,8 +461,13 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
         {
           double xx[R];
           x_load(xx);
+          if constexpr (PRE == 1) {
 #pragma unroll
-          for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]) + omega * (d[j] * r[j]);
+            for (int j = 0; j < R; ++j) xx[j] = xx[j] + omega * sh[j];
+          } else {
+#pragma unroll
+            for (int j = 0; j < R; ++j) xx[j] = xx[j] + alpha * (d[j] * p[j]) + omega * (d[j] * r[j]);
+          }
           x_store(xx);
         }
 #pragma unroll

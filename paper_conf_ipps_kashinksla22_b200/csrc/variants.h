@@ -47,6 +47,7 @@ struct LVariant {
   int rounds;      // BiCGSTAB reduction rounds per iteration (3, or 2: algebraic rho)
   solve_fn fn;
   int ctas;        // resident CTAs per SM the kernel is built for (launch bounds)
+  int pre;         // 0: scalar preconditioner (Jacobi / none), 1: block-Jacobi (8 rows)
 };
 
 // batched banded LU (dgbsv analogue), k_banded.cu
