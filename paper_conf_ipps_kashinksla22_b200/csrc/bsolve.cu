@@ -99,6 +99,10 @@ struct bsolve_plan {
   solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
   int line_nx = 0;                   // > 0: line-tiled TMEM kernel for an NX-wide 9-point grid
   int line_ctas = 0;                 // its resident CTAs per SM (launch bounds)
+  int st_ok = 0;                     // pattern is a uniform-offset stencil (st_doff valid)
+  int st_doff[kMaxW] = {};           // byte offset d_k * 8 of ELL slot k (stencils)
+  int32_t *d_vidx = nullptr;         // CSR values on the line plan: [9][n] value index of
+                                     // canonical slot c (8 = diagonal) of row r, -1 none
   int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};  // its canonical offset -> ELL slot map
   persist_fn var_tmem_p = nullptr;   // persistent TMEM kernel (aligned buffers)
   int smem_bytes_tmem_p = 0, grid_tmem_p = 0;
@@ -171,6 +175,7 @@ static void free_plan(bsolve_plan *h) {
   cudaFree(h->d_ctr);
   cudaFree(h->d_bnd);
   cudaFree(h->d_bcol);
+  cudaFree(h->d_vidx);
   cudaFree(h->d_bws);
   cudaFree(h->d_fbws);
   cudaFree(h->d_fbl);
@@ -403,9 +408,12 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   build_ell_map(n, row_ptr, col_idx, W, h->h_ell_col, h->h_csr2ell, ell_diag);
   if (h->fmt == FMT_ELL) diag = ell_diag;  // kernel needs the diagonal's slot in its format
   h->kfmt = h->fmt;
-  if (h->fmt == FMT_ELL) {
+  {
     // DIA (uniform-offset) addressing if every real entry of slot k sits at
-    // column row + d_k for one d_k per slot: true for stencil patterns
+    // column row + d_k for one d_k per slot: true for stencil patterns.  A
+    // property of the pattern (st_ok, st_doff: the line-tiled plans take it
+    // for both value layouts); ELL values also switch the generic kernels to
+    // DIA addressing.
     std::vector<long long> dk(W, LLONG_MIN);
     bool uniform = true;
     for (int k = 0; k < W && uniform; ++k)
@@ -422,8 +430,14 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         g = std::max<long long>(g, dk[k] < 0 ? -dk[k] : dk[k]);
         h->doff[k] = (int)(dk[k] * 8);
       }
-      h->guard = (int)((g + 1) & ~1LL);
-      h->kfmt = FMT_DIA;
+      h->st_ok = 1;
+      for (int k = 0; k < W; ++k) h->st_doff[k] = h->doff[k];
+      if (h->fmt == FMT_ELL) {
+        h->guard = (int)((g + 1) & ~1LL);
+        h->kfmt = FMT_DIA;
+      } else {
+        for (int k = 0; k < W; ++k) h->doff[k] = 0;  // CSR kernels: column tables
+      }
     }
   }
 
@@ -570,7 +584,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const bool gm = opt.solver == BSOLVE_SOLVER_GMRES;
     const bool bj = opt.precond == BSOLVE_PREC_BLOCK_JACOBI;
     const bool line_on = (gm || !(lenv && atoi(lenv) == 0)) && opt.block_threads == 0 &&
-                         opt.reg_slots == 0 && h->kfmt == FMT_DIA && W <= 9 && n <= 1024 &&
+                         opt.reg_slots == 0 && h->st_ok && W <= 9 && n <= 1024 &&
                          h->place != PLACE_CLUSTER &&
                          (opt.placement == BSOLVE_PLACE_AUTO ||
                           opt.placement == BSOLVE_PLACE_TMEM);
@@ -608,7 +622,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         bool real = false;  // slot k holds at least one entry of the pattern
         for (int r = 0; r < n && !real; ++r) real = h->h_csr2ell[(size_t)k * n + r] >= 0;
         if (!real) continue;
-        const int o = h->doff[k] / 8;
+        const int o = h->st_doff[k] / 8;
         int c = 0;
         while (c < 8 && canon[c] != o) ++c;
         if (c == 8 || c2s[c] >= 0) ok = false;
@@ -713,6 +727,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     // (BSOLVE_LINE_PERSIST=1; 16-byte aligned system blocks, 8 rows/thread)
     const char *lpenv = getenv("BSOLVE_LINE_PERSIST");
     if (h->line_nx && lpenv && atoi(lpenv) == 1 && h->r == 8 && n % 2 == 0 &&
+        h->fmt == FMT_ELL && h->line_ctas == 2 &&
         (h->sys_stride * 8) % 16 == 0) {
       int sb = 0;
       persist_fn f = variant_line_persist(h->line_nx, &sb, h->smem_vals, h->n_pad);
@@ -879,6 +894,19 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
           cudaSuccess ||
       cudaMemcpy(h->d_diag, diag.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail_free(fail(BSOLVE_ERR_CUDA, "copy of the pattern to the device failed"));
+  if (h->line_nx && h->fmt == FMT_CSR && h->place == PLACE_TMEM) {
+    // CSR values on the line-tiled plan: where each (row, canonical slot)
+    // value sits inside a system's CSR block (the ELL slot map's source index)
+    std::vector<int32_t> vidx((size_t)9 * n, -1);
+    for (int c = 0; c < 8; ++c)
+      if (h->c2s[c] >= 0)
+        for (int r = 0; r < n; ++r) vidx[(size_t)c * n + r] = h->h_csr2ell[(size_t)h->c2s[c] * n + r];
+    for (int r = 0; r < n; ++r) vidx[(size_t)8 * n + r] = h->h_csr2ell[r];  // slot 0: diagonal
+    if (cudaMalloc(&h->d_vidx, sizeof(int32_t) * vidx.size()) != cudaSuccess ||
+        cudaMemcpy(h->d_vidx, vidx.data(), sizeof(int32_t) * vidx.size(), cudaMemcpyHostToDevice) !=
+            cudaSuccess)
+      return fail_free(fail(BSOLVE_ERR_CUDA, "copy of the CSR value index table failed"));
+  }
   if (h->direct_fallback) {
     // banded tables + fallback buffers now, so bsolve_run never allocates:
     // the fused banded kernel on at most one wave of resident CTAs, its
@@ -996,6 +1024,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   P.guard = h->guard;
   for (int k = 0; k < kMaxW; ++k) P.doff[k] = h->doff[k];
   for (int c = 0; c < 8; ++c) P.c2s[c] = h->c2s[c];
+  P.vidx = h->d_vidx;
   P.precond = h->precond;
   P.restart = h->restart;
   // line plan: each CTA asks L2 for the system that will start about one

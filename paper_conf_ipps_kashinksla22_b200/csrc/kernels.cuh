@@ -59,6 +59,9 @@ struct SolveParams {
   int guard;                // zero doubles before and after the gather body (DIA)
   int doff[kMaxW];          // DIA: byte offset d_k * 8 of slot k
   int c2s[8];               // line-tiled stencil plan: ELL slot of canonical offset c, -1 none
+  const int32_t *vidx;      // line plan with CSR values: [9][n] index of canonical slot c
+                            // (8 = diagonal) of row r in a system's CSR block, -1 none;
+                            // nullptr: ELL values (slot c2s[c] of the ELL block)
   int precond;              // PREC_JACOBI (d = 1 / a_ii) or PREC_NONE (d = 1)
   int restart;              // GMRES: Krylov steps per restart cycle (1 .. kMaxRestart)
   int pf_ahead;             // line plan: prefetch system sys + pf_ahead into L2 (0: off)

@@ -173,7 +173,7 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
   double d[R];
   double bdiag[PRE ? R : 1], blo[PRE ? R : 1], bup[PRE ? R : 1];  // block-Jacobi block
   {
-    const bool vec = ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
+    const bool vec = !P.vidx && ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
                      row0 + R <= n;
     uint32_t aw[16];
 #pragma unroll
@@ -195,11 +195,22 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const bool a = act[j + h];
-          a0p[h] = a ? __ldg(gval + row0 + j + h) : 0.0;
+          const int row = row0 + j + h;
+          if (P.vidx) {  // CSR values: the handle's (row, canonical slot) -> CSR index table
+            const int e0 = a ? __ldg(P.vidx + 8 * n + row) : -1;
+            a0p[h] = e0 >= 0 ? __ldg(gval + e0) : 0.0;
 #pragma unroll
-          for (int c = 0; c < 8; ++c) {
-            const int k = P.c2s[c];
-            vv[h][c] = (a && k >= 0) ? __ldg(gval + (long long)k * n + row0 + j + h) : 0.0;
+            for (int c = 0; c < 8; ++c) {
+              const int e = a ? __ldg(P.vidx + c * n + row) : -1;
+              vv[h][c] = e >= 0 ? __ldg(gval + e) : 0.0;
+            }
+          } else {
+            a0p[h] = a ? __ldg(gval + row) : 0.0;
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+              const int k = P.c2s[c];
+              vv[h][c] = (a && k >= 0) ? __ldg(gval + (long long)k * n + row) : 0.0;
+            }
           }
         }
       }

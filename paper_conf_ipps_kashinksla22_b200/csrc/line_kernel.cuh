@@ -209,7 +209,7 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
   bool act[R];
   double x[R], r[R], d[R], a0[R];
   double val[R][8];
-  const bool vec = ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
+  const bool vec = !P.vidx && ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
                    row0 + R <= n;
 #pragma unroll
   for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
@@ -226,6 +226,17 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
         if (k >= 0) v = __ldg(reinterpret_cast<const double2 *>(gval + (long long)k * n + row0 + j));
         val[j][c] = v.x;
         val[j + 1][c] = v.y;
+      }
+    }
+  } else if (P.vidx) {  // CSR values: the handle's (row, canonical slot) -> CSR index table
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const int e0 = act[j] ? __ldg(P.vidx + 8 * n + row0 + j) : -1;
+      a0[j] = e0 >= 0 ? __ldg(gval + e0) : 0.0;
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const int e = act[j] ? __ldg(P.vidx + c * n + row0 + j) : -1;
+        val[j][c] = e >= 0 ? __ldg(gval + e) : 0.0;
       }
     }
   } else {
@@ -575,7 +586,7 @@ __global__ void __launch_bounds__(128, 2) bicgstab_tmem_line_cluster_kernel(cons
   double val[R][8];
 #pragma unroll
   for (int j = 0; j < R; ++j) act[j] = lrow0 + j < nloc;
-  const bool vec = ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
+  const bool vec = !P.vidx && ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
                    lrow0 + R <= nloc;
   if (vec) {
 #pragma unroll

@@ -30,8 +30,9 @@ def test_config0_ion_electron_pair(fmt):
     B = X.make_batch(0, 2)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt=fmt)
-    # AUTO: 9-point stencil ELL -> TMEM-resident values; CSR -> SMEM staged
-    assert g["info"]["placement"] == (5 if fmt == "ell" else 1)
+    # AUTO: 9-point stencil -> TMEM-resident values on the line-tiled plan, for
+    # ELL and (round 2, through the CSR value index table) CSR values alike
+    assert g["info"]["placement"] == 5 and g["info"]["kernel_mode"] == 4
     compare(p.row_ptr, p.col_idx, B.values, B.b, g)
 
 
@@ -624,3 +625,25 @@ def test_cluster_maxiter_exhausted(line, monkeypatch):
     assert g["info"]["cluster"] == 4
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
     assert np.any(g["status"] == 1)
+
+
+@pytest.mark.parametrize("nx,ny,solver,precond", [(32, 31, "bicgstab", "jacobi"),
+                                                  (31, 32, "bicgstab", "jacobi"),
+                                                  (32, 31, "gmres", "jacobi"),
+                                                  (32, 31, "bicgstab", "block_jacobi")])
+def test_csr_values_on_the_line_plan(nx, ny, solver, precond):
+    """CSR-ordered values take the same line-tiled TMEM kernels as ELL ones
+    (the kernel reads each (row, canonical slot) value through the handle's
+    CSR index table at CTA start): same plan, bitwise the same results as the
+    ELL layout of the same values, and oracle parity."""
+    B = X.make_batch(0, 96, nx=nx, ny=ny)
+    p = B.pattern
+    gc = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt="csr", solver=solver, precond=precond)
+    ge = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, fmt="ell", solver=solver, precond=precond)
+    assert gc["info"]["kernel_mode"] == 4 and gc["info"]["placement"] == 5
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(gc[k], ge[k]), k
+    if solver == "bicgstab":
+        o = O.batch_krylov(p.row_ptr, p.col_idx, B.values, B.b,
+                           precond=O.block_jacobi(8) if precond == "block_jacobi" else O.PREC_JACOBI)
+        compare(p.row_ptr, p.col_idx, B.values, B.b, gc, o=o)
