@@ -496,29 +496,38 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       // strided-row kernel at n = 4032 (its halo rows are sent by 9 threads
       // with 8 st.async each; 255 registers with spills)
       const char *clenv = getenv("BSOLVE_CLUSTER_LINE");
+      const int cl_line = clenv ? atoi(clenv) : 3;  // 3: 3-CTA line kernel, 1: 2-CTA, 0: strided
       int line_smem = 0;
-      if (ctmem && clenv && atoi(clenv) == 1) {
+      // canonical stencil slot -> ELL slot for an NX-wide grid (false: not that grid)
+      auto map_c2s = [&](int NX, int (&c2s)[8]) {
+        const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
+        for (int cc = 0; cc < 8; ++cc) c2s[cc] = -1;
+        for (int k = 1; k < W; ++k) {
+          bool real = false;
+          for (int rr = 0; rr < n && !real; ++rr) real = h->h_csr2ell[(size_t)k * n + rr] >= 0;
+          if (!real) continue;
+          const int o = h->doff[k] / 8;
+          int cc = 0;
+          while (cc < 8 && canon[cc] != o) ++cc;
+          if (cc == 8 || c2s[cc] >= 0) return false;
+          c2s[cc] = k;
+        }
+        return true;
+      };
+      if (ctmem && (cl_line == 1 || cl_line == 3)) {
         int cnt = 0;
-        const CVariant *t = variants_cluster_line(&cnt, &line_smem);
+        const CVariant *t = cl_line == 3 ? variants_cluster_line3(&cnt, &line_smem)
+                                         : variants_cluster_line(&cnt, &line_smem);
+        const char *csenv = getenv("BSOLVE_CLUSTER_SYNC");  // "barrier": the reference exchange
+        const int mb = (csenv && std::strcmp(csenv, "barrier") == 0) ? 0 : 1;
         for (int i = 0; i < cnt && !h->cvar; ++i) {
           if (t[i].c != c) continue;
-          const int NX = t[i].kreg;
-          const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
-          int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
-          bool ok = true;
-          for (int k = 1; k < W && ok; ++k) {
-            bool real = false;
-            for (int rr = 0; rr < n && !real; ++rr) real = h->h_csr2ell[(size_t)k * n + rr] >= 0;
-            if (!real) continue;
-            const int o = h->doff[k] / 8;
-            int cc = 0;
-            while (cc < 8 && canon[cc] != o) ++cc;
-            if (cc == 8 || c2s[cc] >= 0) ok = false;
-            else c2s[cc] = k;
-          }
-          if (!ok) continue;
+          if (cl_line == 3 && t[i].rounds != mb) continue;
+          int c2s[8];
+          if (!map_c2s(t[i].kreg, c2s)) continue;
           h->cvar = &t[i];
-          h->line_nx = NX;
+          h->line_nx = t[i].kreg;
+          h->line_ctas = cl_line == 3 ? 3 : 2;
           for (int cc = 0; cc < 8; ++cc) h->c2s[cc] = c2s[cc];
         }
       }
@@ -549,6 +558,8 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, h->smem_bytes);
       if (ce != cudaSuccess)
         return fail_free(fail(BSOLVE_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(ce)));
+      cudaFuncSetAttribute((const void *)h->cvar->fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                           cudaSharedmemCarveoutMaxShared);
       cudaLaunchConfig_t cfg = {};
       cfg.gridDim = dim3(c * 64);
       cfg.blockDim = dim3(128);

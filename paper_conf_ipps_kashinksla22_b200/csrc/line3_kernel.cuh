@@ -101,74 +101,20 @@ __device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const do
   }
 }
 
-// PRE = 0: PRECOND(y) = d .* y (scalar Jacobi, P:236-237, or none).
-// PRE = 1: block-Jacobi with one block per thread = its 8 consecutive rows
-// (SURVEY.md 8(f) f3; DESIGN.md R30).  On an NX >= 9 wide 9-point grid the
-// block A[8t..8t+7, 8t..8t+7] is tridiagonal (only the +-1 couplings fall
-// inside it); it is factored once per system without pivoting (Thomas,
-// l_j = a_(j,j-1) / u_(j-1), u_j = a_jj - l_j a_(j-1,j); a zero or non-finite
-// pivot makes the block the identity) into thread-private SMEM, and every
-// application is a forward and a back substitution in registers.
-template <int NX, int ROUNDS = 2, int PRE = 0>
-__global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParams P) {
-  using G3 = Line3Geom<NX, PRE>;
-  constexpr int R = G3::R, NT = G3::NT;
-  using L = typename G3::L;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double *sg = reinterpret_cast<double *>(smem_raw);
-  double *sred = sg + G3::OFF_RED;
-  double2 *sx2 = reinterpret_cast<double2 *>(sg + G3::OFF_X) + threadIdx.x;  // x pair k at [k*NT]
-  double *sf = sg + G3::OFF_F + threadIdx.x;  // block-Jacobi factor k at sf[k * NT]
-  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + G3::OFF_F + G3::NF * NT);
-
-  const int tid = threadIdx.x, warp = tid >> 5;
+// Algorithm 1 for one system on this CTA's rows (the whole system for the
+// single-CTA kernel, rows grow0 .. grow0 + 1023 of it on a cluster): every
+// global row index is grow0 + 8 t + j; the communication policy Comm
+// (LineComm: CTA-local; Line3ClusterComm: halo rows and reduction partials
+// through distributed shared memory) publishes, synchronises and reduces.
+template <int NX, int ROUNDS, int PRE, class Comm>
+__device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys, int grow0,
+                                            bool leader, const bool (&act)[8], Comm &comm,
+                                            double *sf, double2 *sx2, uint32_t tval,
+                                            uint32_t trh, uint32_t ta0) {
+  constexpr int R = 8, NT = 128;
   const int n = P.n;
-  const long long sys = blockIdx.x;
-  const int row0 = R * tid;
+  const int row0 = grow0 + R * threadIdx.x;  // global index of this thread's first row
   const double *gval = P.values + sys * P.sys_stride;
-
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_addr(tbase_s)),
-                 "n"(128));
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_addr(tbase_s + 1)),
-                 "n"(32));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  for (int i = tid; i < R * (L::S - NT); i += NT) {  // zero guard columns
-    const int pl = i / (L::S - NT), q = i % (L::S - NT);
-    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
-  }
-  if (tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {  // L2 prefetch, as line kernel
-    const long long ns = sys + P.pf_ahead;
-    const void *va = P.values + ns * P.sys_stride;
-    const void *ba = P.b + ns * n;
-    if (((reinterpret_cast<uintptr_t>(va) | reinterpret_cast<uintptr_t>(ba)) & 15u) == 0) {
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(va),
-                   "r"(static_cast<uint32_t>(P.sys_stride * 8) & ~15u)
-                   : "memory");
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
-                   "r"(static_cast<uint32_t>(n * 8) & ~15u)
-                   : "memory");
-      const void *xa = P.x0 ? P.x0 + ns * n : nullptr;
-      if (xa && (reinterpret_cast<uintptr_t>(xa) & 15u) == 0)
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(xa),
-                     "r"(static_cast<uint32_t>(n * 8) & ~15u)
-                     : "memory");
-    }
-  }
-  bool act[R];
-#pragma unroll
-  for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;");
-  const uint32_t lane_hi = static_cast<uint32_t>(32 * warp) << 16;
-  const uint32_t tval = tbase_s[0] + lane_hi;  // 8 rows x 16 columns of values
-  const uint32_t trh = tbase_s[1] + lane_hi;   // r^ (8 doubles)
-  const uint32_t ta0 = trh + 16;               // a_jj (8 doubles)
-
   // ---- this thread's rows: values -> TMEM, diagonal -> TMEM + d ------------
   double d[R];
   double bdiag[PRE ? R : 1], blo[PRE ? R : 1], bup[PRE ? R : 1];  // block-Jacobi block
@@ -260,7 +206,6 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
   for (int j = 0; j < R; ++j) r[j] = act[j] ? __ldg(bsys + row0 + j) : 0.0;
   tmem_wait_st();
 
-  LineComm<NX, NT, R> comm(sg, sred, act);
   const double one[R] = {1, 1, 1, 1, 1, 1, 1, 1};
   auto spmv = [&](const double(&dd)[R], const double(&g)[R], double(&y)[R]) {
     line3_spmv<NX>(tval, ta0, comm.gq, dd, g, y);
@@ -341,7 +286,7 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
 #pragma unroll
     for (int j = 0; j < R; ++j)
       if (act[j]) xout[row0 + j] = 0.0;
-    if (tid == 0) {
+    if (leader) {
       P.iters[sys] = 0;
       P.resnorm[sys] = 0.0;
       if (P.status) P.status[sys] = SYS_CONVERGED;
@@ -543,14 +488,363 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
 #pragma unroll
     for (int j = 0; j < R; ++j)
       if (act[j]) xout[row0 + j] = xx[j];
-    if (tid == 0) {
+    if (leader) {
       P.iters[sys] = it;
       P.resnorm[sys] = final_res;
       if (P.status) P.status[sys] = static_cast<int8_t>(st);
     }
   }
+}
+
+// PRE = 0: PRECOND(y) = d .* y (scalar Jacobi, P:236-237, or none).
+// PRE = 1: block-Jacobi with one block per thread = its 8 consecutive rows
+// (SURVEY.md 8(f) f3; DESIGN.md R30).  On an NX >= 9 wide 9-point grid the
+// block A[8t..8t+7, 8t..8t+7] is tridiagonal (only the +-1 couplings fall
+// inside it); it is factored once per system without pivoting (Thomas,
+// l_j = a_(j,j-1) / u_(j-1), u_j = a_jj - l_j a_(j-1,j); a zero or non-finite
+// pivot makes the block the identity) into thread-private SMEM, and every
+// application is a forward and a back substitution in registers.
+template <int NX, int ROUNDS = 2, int PRE = 0>
+__global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParams P) {
+  using G3 = Line3Geom<NX, PRE>;
+  constexpr int R = G3::R, NT = G3::NT;
+  using L = typename G3::L;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sg = reinterpret_cast<double *>(smem_raw);
+  double *sred = sg + G3::OFF_RED;
+  double2 *sx2 = reinterpret_cast<double2 *>(sg + G3::OFF_X) + threadIdx.x;  // x pair k at [k*NT]
+  double *sf = sg + G3::OFF_F + threadIdx.x;  // block-Jacobi factor k at sf[k * NT]
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + G3::OFF_F + G3::NF * NT);
+
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long sys = blockIdx.x;
+  const int row0 = R * tid;
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(128));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s + 1)),
+                 "n"(32));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  for (int i = tid; i < R * (L::S - NT); i += NT) {  // zero guard columns
+    const int pl = i / (L::S - NT), q = i % (L::S - NT);
+    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
+  }
+  if (tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {  // L2 prefetch, as line kernel
+    const long long ns = sys + P.pf_ahead;
+    const void *va = P.values + ns * P.sys_stride;
+    const void *ba = P.b + ns * n;
+    if (((reinterpret_cast<uintptr_t>(va) | reinterpret_cast<uintptr_t>(ba)) & 15u) == 0) {
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(va),
+                   "r"(static_cast<uint32_t>(P.sys_stride * 8) & ~15u)
+                   : "memory");
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
+                   "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                   : "memory");
+      const void *xa = P.x0 ? P.x0 + ns * n : nullptr;
+      if (xa && (reinterpret_cast<uintptr_t>(xa) & 15u) == 0)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(xa),
+                     "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                     : "memory");
+    }
+  }
+  bool act[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t lane_hi = static_cast<uint32_t>(32 * warp) << 16;
+  const uint32_t tval = tbase_s[0] + lane_hi;  // 8 rows x 16 columns of values
+  const uint32_t trh = tbase_s[1] + lane_hi;   // r^ (8 doubles)
+  const uint32_t ta0 = trh + 16;               // a_jj (8 doubles)
+
+  LineComm<NX, NT, R> comm(sg, sred, act);
+  line3_solve<NX, ROUNDS, PRE>(P, sys, 0, tid == 0, act, comm, sf, sx2, tval, trh, ta0);
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[1]), "n"(32));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[0]), "n"(128));
+  }
+}
+
+// ------------------------------------------------ the 3-CTA plan on a cluster --
+// Systems larger than one CTA (n > 1024, e.g. the 63 x 64 grid, n = 4032:
+// SURVEY.md 8(f) f2, BASELINE configs[4]) on a cluster of C CTAs of 1024
+// consecutive rows each, every CTA running line3_solve on its rows.  The
+// exchange is BARRIER-based: publishing row li also stores it (st.shared::
+// cluster) into the left neighbour's right guard (li < NX + 1) or the right
+// neighbour's left guard (li >= nloc - NX - 1); sync() is a cluster barrier
+// (arrive.release / wait.acquire), after which every CTA's SpMV reads only
+// its own planes.  Reductions push each warp's partial into every CTA's
+// scratch and pass one cluster barrier.  WAR safety: a CTA rewrites its
+// planes (and its neighbours' guards) only after a reduction barrier that
+// every CTA reaches after its previous SpMV; reduction scratch alternates
+// between two halves.  No mbarrier, no transaction counting: racecheck
+// models these barriers.
+__device__ __forceinline__ void st_cluster_f64(uint32_t addr, double v) {
+  asm volatile("st.shared::cluster.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
+}
+// Bulk copy of `bytes` (multiple of 16, 16-byte aligned) from this CTA's
+// shared memory to a peer's (shared::cluster address), completing the bytes on
+// the peer's mbarrier.
+__device__ __forceinline__ void bulk_s2c(uint32_t dst, uint32_t src, uint32_t bytes, uint32_t rbar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(dst), "r"(src), "r"(bytes), "r"(rbar)
+      : "memory");
+}
+__device__ __forceinline__ void cluster_barrier() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+
+// MB = 1 (default): point-to-point transaction barriers instead of cluster
+// barriers -- halo rows and reduction partials travel by st.async, each
+// completing 8 bytes on the RECEIVER's mbarrier; the receiver's thread 0 arms
+// the expected byte count, everyone waits with acquire.cluster semantics.  No
+// cluster-wide barrier (and no membar) per exchange.  Ordering (the same
+// transitive argument as DESIGN.md Kernels 8): a neighbour pushes the next
+// halo into my guards only after a reduction that needs my partial, which I
+// push after my SpMV read those guards; racecheck does not model that chain,
+// so MB = 0 (BSOLVE_CLUSTER_SYNC=barrier) is kept as the checkable reference.
+template <int NX, int C, int MB>
+struct Line3ClusterComm {
+  static constexpr int R = 8, NT = 128, NWARP = 4, RPC = R * NT, G = NX + 1;
+  static constexpr int NP = C * NWARP;  // partials per reduced value
+  using L = LineGeom<NX, NT, R>;
+  double *gq;    // sg + GQ + threadIdx.x
+  double *sred;  // scratch [2][8][NP]
+  // this thread's rows j < nleft go to the left neighbour's right guard, rows
+  // j >= rfirst to the right neighbour's left guard: row j of thread t sits
+  // in plane j, column GQ + t + 128 (left) or GQ + t - 128 (right) there
+  uint32_t lbase = 0, rbase = 0, sred_s;
+  int nleft = 0, rfirst = R, buf = 0, rank;
+  // MB = 1: [0] halo, [1], [2] reduction halves; the neighbours' halo barriers
+  uint64_t *bars;
+  uint32_t lhbar = 0, rhbar = 0, phases = 0;  // phases: bit 0/1 reduction halves, bit 2 halo
+  uint32_t lseg = 0, rseg = 0;  // MB = 1: bulk-copy destinations (plane 0) in the neighbours
+  int n;
+  __device__ __forceinline__ Line3ClusterComm(double *sg, double *sred_, uint64_t *bars_, int rank_,
+                                              int n_)
+      : gq(sg + L::GQ + threadIdx.x), sred(sred_), rank(rank_), bars(bars_), n(n_) {
+    const uint32_t sg_s = smem_addr(sg);
+    const int t = threadIdx.x;
+    const uint32_t bars_s = smem_addr(bars);
+    if (MB) {  // halo by bulk copies, issued by threads 0..7 (left) and 32..39 (right)
+      if (rank > 0 && t < 8) {
+        lseg = mapa_u32(sg_s, rank - 1) + 8u * static_cast<uint32_t>(L::GQ + NT);
+        lhbar = mapa_u32(bars_s, rank - 1);
+      }
+      static_assert(L::GQ >= 10 && NX + 1 <= 80, "halo segments: 10 columns cover the reach");
+      if (rank < C - 1 && t >= 32 && t < 40) {
+        rseg = mapa_u32(sg_s, rank + 1) + 8u * static_cast<uint32_t>(L::GQ - 10);
+        rhbar = mapa_u32(bars_s, rank + 1);
+      }
+    } else {
+      if (rank > 0 && R * t < G) {
+        lbase = mapa_u32(sg_s, rank - 1) + 8u * static_cast<uint32_t>(L::GQ + t + NT);
+        nleft = min(R, G - R * t);
+      }
+      if (rank < C - 1 && R * t + R > RPC - G) {  // (only the last CTA has nloc < RPC)
+        rbase = mapa_u32(sg_s, rank + 1) + 8u * static_cast<uint32_t>(L::GQ + t - NT);
+        rfirst = max(0, RPC - G - R * t);
+      }
+    }
+    sred_s = smem_addr(sred);
+  }
+  // halo bytes this CTA receives: G rows from each neighbour (the right
+  // neighbour's first G rows; the left neighbour's last G rows)
+  __device__ __forceinline__ uint32_t halo_bytes() const {  // 8 segments per neighbour
+    return 8u * SEG * static_cast<uint32_t>((rank > 0 ? 1 : 0) + (rank < C - 1 ? 1 : 0));
+  }
+  __device__ __forceinline__ void push(uint32_t addr, double v, uint32_t rbar) {
+    st_async_f64(addr, v, rbar);
+  }
+  // MB = 0 stores through generic pointers to the peer's shared memory
+  // (cooperative_groups map_shared_rank), the form compute-sanitizer tracks
+  __device__ __forceinline__ static double *peer(double *local, int r) {
+    return cooperative_groups::this_cluster().map_shared_rank(local, r);
+  }
+  __device__ __forceinline__ void publish(int j, double v) {
+    gq[j * L::S] = v;
+    if (MB) {
+      // (the halo leaves in sync(), by bulk copies)
+    } else {
+      if (j < nleft) peer(gq, rank - 1)[NT + j * L::S] = v;
+      if (j >= rfirst) peer(gq, rank + 1)[j * L::S - NT] = v;
+    }
+  }
+  // MB = 1: one 80-byte bulk copy per plane and side moves the halo: my rows
+  // 0..64 (plane j, columns GQ..GQ+9) into the left neighbour's right guard
+  // (columns GQ+128..), my rows 959..1023 (columns GQ+118..GQ+127) into the
+  // right neighbour's left guard (columns 0..9); the extra rows copied are
+  // never read (the stencil reaches 65 rows).  S and GQ are even, so every
+  // segment is 16-byte aligned.
+  static constexpr uint32_t SEG = 80;
+  __device__ __forceinline__ void sync() {
+    if (MB) {
+      fence_proxy_async_smem();  // my plane stores before the async-proxy copies read them
+      if (threadIdx.x == 0) mbar_arrive_expect_tx(bars, halo_bytes());
+      __syncthreads();
+      const int t = threadIdx.x;
+      if (t < 8 && rank > 0) {  // thread t copies plane t to the left
+        const uint32_t src = smem_addr(gq - t) + 8u * static_cast<uint32_t>(t * L::S);
+        bulk_s2c(lseg + 8u * static_cast<uint32_t>(t * L::S), src, SEG, lhbar);
+      } else if (t >= 32 && t < 40 && rank < C - 1) {  // thread 32 + j: plane j to the right
+        const int j = t - 32;
+        const uint32_t src = smem_addr(gq - t) + 8u * static_cast<uint32_t>(j * L::S + NT - 10);
+        bulk_s2c(rseg + 8u * static_cast<uint32_t>(j * L::S), src, SEG, rhbar);
+      }
+      mbar_wait_parity_cluster(bars, (phases >> 2) & 1u);
+      phases ^= 4u;
+    } else {
+      cooperative_groups::this_cluster().sync();
+    }
+  }
+  // before a publish that follows no exchange: the CTA's own readers only
+  // (every peer's earlier SpMV is ordered by the last reduction)
+  __device__ __forceinline__ void barrier() {
+    if (MB) __syncthreads();
+    else cooperative_groups::this_cluster().sync();
+  }
+  template <int K>
+  __device__ __forceinline__ void sum(double (&v)[K]) {
+    static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    constexpr int KP = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
+    constexpr int SPAN = 32 / KP;
+    double a[KP];
+#pragma unroll
+    for (int i = 0; i < KP; ++i) a[i] = i < K ? v[i] : 0.0;
+#pragma unroll
+    for (int cnt = KP, o = 16; cnt > 1; cnt >>= 1, o >>= 1) {  // recursive halving
+      const bool hi = lane & o;
+#pragma unroll
+      for (int i = 0; i < cnt / 2; ++i) {
+        const double send = hi ? a[i] : a[i + cnt / 2];
+        const double keep = hi ? a[i + cnt / 2] : a[i];
+        a[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+      }
+    }
+#pragma unroll
+    for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
+    const int q = lane / SPAN;
+    if (MB && threadIdx.x == 0) mbar_arrive_expect_tx(bars + 1 + buf, static_cast<uint32_t>(K * NP * 8));
+    if ((lane % SPAN) == 0 && q < K) {
+      const uint32_t off = static_cast<uint32_t>((buf * 8 * NP + q * NP + rank * NWARP + warp) * 8);
+#pragma unroll
+      for (int r = 0; r < C; ++r) {
+        if (MB) push(mapa_u32(sred_s + off, r), a[0], mapa_u32(smem_addr(bars + 1 + buf), r));
+        else peer(sred, r)[off / 8] = a[0];
+      }
+    }
+    if (MB) {
+      const uint32_t bit = 1u << buf;
+      mbar_wait_parity_cluster(bars + 1 + buf, (phases & bit) ? 1u : 0u);
+      phases ^= bit;
+    } else {
+      cooperative_groups::this_cluster().sync();
+    }
+    const double *Sx = sred + buf * (8 * NP);
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      double part[NP];
+      const double2 *S2 = reinterpret_cast<const double2 *>(Sx + k * NP);
+#pragma unroll
+      for (int w = 0; w < NP / 2; ++w) {
+        const double2 qq = S2[w];
+        part[2 * w] = qq.x;
+        part[2 * w + 1] = qq.y;
+      }
+      v[k] = tree_sum<NP>(part);
+    }
+    buf ^= 1;
+  }
+};
+
+template <int NX, int C>
+struct Line3ClusterGeom {
+  using G3 = Line3Geom<NX, 0>;
+  static constexpr int R = 8, NT = 128;
+  static constexpr int OFF_RED = G3::OFF_RED;                         // [2][8][C*4]
+  static constexpr int OFF_X = (OFF_RED + 2 * 8 * C * 4 + 1) & ~1;
+  static constexpr int OFF_BAR = OFF_X + R * NT;  // 3 mbarriers (MB = 1)
+  static constexpr int SMEM_BYTES = (OFF_BAR + 3) * 8 + 16;
+};
+
+// One system per cluster of C CTAs x 1024 rows (blockIdx.x / C = system).
+template <int NX, int C, int MB = 1, int ROUNDS = 2>
+__global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const SolveParams P) {
+  using CG = Line3ClusterGeom<NX, C>;
+  constexpr int R = 8, NT = 128;
+  using L = LineGeom<NX, NT, R>;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double *sg = reinterpret_cast<double *>(smem_raw);
+  double *sred = sg + CG::OFF_RED;
+  double2 *sx2 = reinterpret_cast<double2 *>(sg + CG::OFF_X) + threadIdx.x;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(sg + CG::OFF_BAR);
+  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + CG::OFF_BAR + 3);
+  uint32_t crank;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+  const int rank = static_cast<int>(crank);
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int n = P.n;
+  const long long sys = blockIdx.x / C;
+  const int grow0 = rank * 1024;
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s)),
+                 "n"(128));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_addr(tbase_s + 1)),
+                 "n"(32));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  for (int i = tid; i < R * (L::S - NT); i += NT) {  // guards: global edges stay 0
+    const int pl = i / (L::S - NT), q = i % (L::S - NT);
+    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
+  }
+  if (rank == 0 && tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {
+    const long long ns = sys + P.pf_ahead;
+    const void *va = P.values + ns * P.sys_stride;
+    const void *ba = P.b + ns * n;
+    if (((reinterpret_cast<uintptr_t>(va) | reinterpret_cast<uintptr_t>(ba)) & 15u) == 0) {
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(va),
+                   "r"(static_cast<uint32_t>(P.sys_stride * 8) & ~15u)
+                   : "memory");
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ba),
+                   "r"(static_cast<uint32_t>(n * 8) & ~15u)
+                   : "memory");
+    }
+  }
+  if (MB && tid == 32) {
+    for (int i = 0; i < 3; ++i) mbar_init(bars + i, 1);
+    fence_mbar_init();
+  }
+  bool act[R];
+#pragma unroll
+  for (int j = 0; j < R; ++j) act[j] = grow0 + R * tid + j < n;
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  // TMEM addresses published; every CTA's guards zeroed and mbarriers
+  // initialised before any peer pushes into them
+  cluster_barrier();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t lane_hi = static_cast<uint32_t>(32 * warp) << 16;
+  const uint32_t tval = tbase_s[0] + lane_hi;
+  const uint32_t trh = tbase_s[1] + lane_hi;
+  const uint32_t ta0 = trh + 16;
+  Line3ClusterComm<NX, C, MB> comm(sg, sred, bars, rank, n);
+  line3_solve<NX, ROUNDS, 0>(P, sys, grow0, rank == 0 && tid == 0, act, comm, nullptr, sx2, tval,
+                             trh, ta0);
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  cluster_barrier();  // no CTA leaves while a peer may still store into its SMEM
   if (warp == 0) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[1]), "n"(32));
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[0]), "n"(128));

@@ -49,7 +49,9 @@ struct LineGeom {
     return o >= 0 ? o / R : -((-o + R - 1) / R);
   }
   static constexpr int GQ = (NX + 1 + R - 1) / R + 1;  // zero columns before the body
-  static constexpr int S = NT + 2 * GQ + 1;            // doubles per plane
+  // doubles per plane, even: every plane (and the GQ-column halo segment of
+  // the cluster kernels' bulk copies) starts 16-byte aligned
+  static constexpr int S = (NT + 2 * GQ + 1 + 1) & ~1;
   // element offset of row R t + o relative to sg + GQ + t
   __host__ __device__ static constexpr int idx(int o) {
     return (o - R * floordivR(o)) * S + floordivR(o);

@@ -595,12 +595,15 @@ def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
 
 
-@pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4)])
-def test_cluster_line_kernel(nx, ny, C, monkeypatch):
-    """Opt-in line-tiled TMEM cluster kernel (BSOLVE_CLUSTER_LINE=1): the
-    plane guards carry the neighbours' halo rows (st.async + mbarrier); same
-    parity bar, warm start included."""
-    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", "1")
+@pytest.mark.parametrize("line", ["3", "1"])
+@pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4), (64, 120, 8)])
+def test_cluster_line_kernel(nx, ny, C, line, monkeypatch):
+    """Line-tiled TMEM cluster kernels: BSOLVE_CLUSTER_LINE=3 (default, the
+    3-CTA line3 kernel per cluster CTA, halo rows and reduction partials by
+    st.shared::cluster + cluster barriers) and =1 (the 2-CTA line kernel,
+    st.async + mbarrier): the plane guards carry the neighbours' halo rows;
+    same parity bar, warm start included."""
+    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", line)
     B = X.make_batch(0, 12, nx=nx, ny=ny)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
@@ -612,7 +615,7 @@ def test_cluster_line_kernel(nx, ny, C, monkeypatch):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
 
 
-@pytest.mark.parametrize("line", ["0", "1"])
+@pytest.mark.parametrize("line", ["0", "1", "3"])
 def test_cluster_maxiter_exhausted(line, monkeypatch):
     """Cluster plans (strided and line-tiled) when maxiter runs out: the final
     true-residual check must not wait for a halo nobody sent (regression: the
