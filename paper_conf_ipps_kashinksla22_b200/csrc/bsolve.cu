@@ -519,7 +519,13 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         const CVariant *t = cl_line == 3 ? variants_cluster_line3(&cnt, &line_smem)
                                          : variants_cluster_line(&cnt, &line_smem);
         const char *csenv = getenv("BSOLVE_CLUSTER_SYNC");  // "barrier": the reference exchange
-        const int mb = (csenv && std::strcmp(csenv, "barrier") == 0) ? 0 : 1;
+        // BSOLVE_CLUSTER_SYNC: default / "halo": bulk halo copies + two-stage
+        // reductions on mbarriers (measured fastest); "state": halo state kept
+        // per CTA, 2 exchanges per iteration (slower: element-wise pushes);
+        // "barrier": cluster barriers (the reference)
+        const int mb = !csenv ? 1 : std::strcmp(csenv, "barrier") == 0 ? 0
+                                  : std::strcmp(csenv, "state") == 0  ? 2
+                                                                       : 1;
         for (int i = 0; i < cnt && !h->cvar; ++i) {
           if (t[i].c != c) continue;
           if (cl_line == 3 && t[i].rounds != mb) continue;

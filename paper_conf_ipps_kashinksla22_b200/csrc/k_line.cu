@@ -65,13 +65,15 @@ const CVariant *variants_cluster_line(int *count, int *smem_bytes) {
 }
 
 // 3-CTA line-tiled plan on a cluster of C CTAs (line3_kernel.cuh), NX = 64
-// (rounds field: 1 = st.async + mbarrier exchange (default), 0 = cluster
-// barriers, the racecheck-verifiable reference, BSOLVE_CLUSTER_SYNC=barrier)
-#define L3CV_(NX, C, MB) {C, NX, MB, (solve_fn)bicgstab_line3_cluster_kernel<NX, C, MB>}
+// rounds field: 2 = halo state kept per CTA, 2 exchanges per iteration (default);
+// 1 = halo by bulk copies, 4 exchanges; 0 = cluster barriers (reference)
+#define L3CV_(NX, C, M) {C, NX, M, (solve_fn)bicgstab_line3_cluster_kernel<NX, C, M >= 1, M == 2>}
 static const CVariant kL3CVariants[] = {
-    L3CV_(64, 2, 1), L3CV_(64, 3, 1), L3CV_(64, 4, 1), L3CV_(64, 5, 1), L3CV_(64, 6, 1),
-    L3CV_(64, 7, 1), L3CV_(64, 8, 1), L3CV_(64, 2, 0), L3CV_(64, 3, 0), L3CV_(64, 4, 0),
-    L3CV_(64, 5, 0), L3CV_(64, 6, 0), L3CV_(64, 7, 0), L3CV_(64, 8, 0)};
+    L3CV_(64, 2, 2), L3CV_(64, 3, 2), L3CV_(64, 4, 2), L3CV_(64, 5, 2), L3CV_(64, 6, 2),
+    L3CV_(64, 7, 2), L3CV_(64, 8, 2), L3CV_(64, 2, 1), L3CV_(64, 3, 1), L3CV_(64, 4, 1),
+    L3CV_(64, 5, 1), L3CV_(64, 6, 1), L3CV_(64, 7, 1), L3CV_(64, 8, 1), L3CV_(64, 2, 0),
+    L3CV_(64, 3, 0), L3CV_(64, 4, 0), L3CV_(64, 5, 0), L3CV_(64, 6, 0), L3CV_(64, 7, 0),
+    L3CV_(64, 8, 0)};
 const CVariant *variants_cluster_line3(int *count, int *smem_bytes) {
   *count = (int)(sizeof(kL3CVariants) / sizeof(kL3CVariants[0]));
   *smem_bytes = Line3ClusterGeom<64, 8>::SMEM_BYTES;

@@ -272,7 +272,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
     red3[1] += r[j] * r[j];
   }
   rh_store(r);
-  comm.template sum<2>(red3);
+  comm.template sum_x<2>(red3, r, 2, d);  // (+ boundary r and d: the halo state)
   const double bnorm = sqrt(red3[0]);
   const double tau = (P.stop == STOP_ABS) ? P.tol : P.tol * bnorm;
   const double tau2 = tau * tau;
@@ -307,7 +307,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
         q[j] = act[j] ? bj - q[j] : 0.0;
         tr[0] += q[j] * q[j];
       }
-      comm.template sum<1>(tr);
+      comm.template sum_x<1>(tr, q, 3, q);  // (+ boundary q: the restart's halo r)
       return tr[0];
     };
 
@@ -339,7 +339,12 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
             comm.publish(j, d[j] * p[j]);
           }
         }
-        comm.sync();
+        if constexpr (Comm::kHalo2) {
+          comm.halo_p(beta, omega);  // the neighbours' boundary rows, recomputed here
+          comm.sync_local();
+        } else {
+          comm.sync();
+        }
         if constexpr (PRE == 1) spmv(one, ph, v);           // a6: v = A p^
         else spmv(d, p, v);
         ++it;
@@ -349,7 +354,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
           rh_load(hw);
           rv[0] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * v[j]; });
         }
-        comm.template sum<1>(rv);                           // a7: r^.v
+        comm.template sum_x<1>(rv, v, 1, v);                // a7: r^.v (+ boundary v)
         if (bad(rv[0])) { st = SYS_BREAKDOWN; break; }
         alpha = rho / rv[0];                                // R3
         // s = r - alpha v (kept in r); publish s^ = PRECOND(s)
@@ -374,7 +379,12 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
             comm.publish(j, d[j] * r[j]);
           }
         }
-        comm.sync();
+        if constexpr (Comm::kHalo2) {
+          comm.halo_s(alpha);
+          comm.sync_local();
+        } else {
+          comm.sync();
+        }
         // ROUNDS == 3: t.s, t.t, s.s here and ||r||^2, r^.r in a third round.
         // ROUNDS == 2 (R29): + r^.s, r^.t, so that rho_{i+1} =
         // r^.s - omega r^.t and ||r_{i+1}||^2 = s.s - omega t.s come from this
@@ -398,7 +408,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
           rh_load(hw);
           ts[4] = rows_sum<R>([&](int j) { return tmem_f64(hw, j) * t[j]; });
         }
-        comm.template sum<KT>(ts);
+        comm.template sum_x<KT>(ts, t, 4, t);               // (+ boundary t)
         if (below(ts[2])) {                                 // stop test 2
           if constexpr (PRE == 0) {  // (block-Jacobi: x + alpha p^ is stored already)
             double xx[R];
@@ -428,6 +438,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
         }
 #pragma unroll
         for (int j = 0; j < R; ++j) r[j] = r[j] - omega * t[j];   // r = s - omega t
+        if constexpr (Comm::kHalo2) comm.halo_r(omega);
         bool explicit_round = ROUNDS == 3;
         if constexpr (ROUNDS == 2) {
           const double rho_n = ts[3] - omega * ts[4];
@@ -468,6 +479,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
         p[j] = 0.0;
         v[j] = 0.0;
       }
+      if constexpr (Comm::kHalo2) comm.halo_restart();
       rh_store(q);
       alpha = omega = beta_c = 1.0;
       rnorm2 = tr2;
@@ -613,13 +625,24 @@ __device__ __forceinline__ void cluster_barrier() {
 // halo into my guards only after a reduction that needs my partial, which I
 // push after my SpMV read those guards; racecheck does not model that chain,
 // so MB = 0 (BSOLVE_CLUSTER_SYNC=barrier) is kept as the checkable reference.
-template <int NX, int C, int MB>
+template <int NX, int C, int MB, int H2 = 0>
 struct Line3ClusterComm {
   static constexpr int R = 8, NT = 128, NWARP = 4, RPC = R * NT, G = NX + 1;
+  // H2 = 1 (MB = 1 only; DESIGN.md Kernels 14): two exchanges per iteration
+  // instead of four.  The p^ and s^ halos are not sent: every CTA keeps the
+  // state (d, p, r|s, v, t) of its neighbours' G boundary rows next to its
+  // guards and updates it with the owner's expressions (the same source
+  // expressions, so the same contraction into the same fma sequence: the
+  // guard values are the owner's bits -- checked bitwise against the
+  // exchanging variants by the tests); the owner's new v and t for those rows
+  // ride along with the two reductions that follow the SpMVs.
+  static constexpr bool kHalo2 = H2 != 0;
+  static constexpr int HS = 66;  // halo state: [side][field][HS], sides L = 0, R = 1
+  enum { F_D = 0, F_P = 1, F_R = 2, F_V0 = 3, F_V1 = 4, F_T = 5, NF = 6 };
   static constexpr int NP = C * NWARP;  // partials per reduced value
   using L = LineGeom<NX, NT, R>;
   double *gq;    // sg + GQ + threadIdx.x
-  double *sred;  // scratch [2][8][NP]
+  double *sred;  // scratch [2][8][NWARP + C]: warp partials, CTA partials
   // this thread's rows j < nleft go to the left neighbour's right guard, rows
   // j >= rfirst to the right neighbour's left guard: row j of thread t sits
   // in plane j, column GQ + t + 128 (left) or GQ + t - 128 (right) there
@@ -630,9 +653,11 @@ struct Line3ClusterComm {
   uint32_t lhbar = 0, rhbar = 0, phases = 0;  // phases: bit 0/1 reduction halves, bit 2 halo
   uint32_t lseg = 0, rseg = 0;  // MB = 1: bulk-copy destinations (plane 0) in the neighbours
   int n;
+  double *hst = nullptr;        // H2: halo state (this CTA's copy of the neighbours' rows)
+  int vk = 0;                   // H2: v exchanges so far (v is double-buffered by parity)
   __device__ __forceinline__ Line3ClusterComm(double *sg, double *sred_, uint64_t *bars_, int rank_,
-                                              int n_)
-      : gq(sg + L::GQ + threadIdx.x), sred(sred_), rank(rank_), bars(bars_), n(n_) {
+                                              int n_, double *hst_ = nullptr)
+      : gq(sg + L::GQ + threadIdx.x), sred(sred_), rank(rank_), bars(bars_), n(n_), hst(hst_) {
     const uint32_t sg_s = smem_addr(sg);
     const int t = threadIdx.x;
     const uint32_t bars_s = smem_addr(bars);
@@ -657,6 +682,7 @@ struct Line3ClusterComm {
       }
     }
     sred_s = smem_addr(sred);
+    if (H2) init_push();
   }
   // halo bytes this CTA receives: G rows from each neighbour (the right
   // neighbour's first G rows; the left neighbour's last G rows)
@@ -701,7 +727,11 @@ struct Line3ClusterComm {
         const uint32_t src = smem_addr(gq - t) + 8u * static_cast<uint32_t>(j * L::S + NT - 10);
         bulk_s2c(rseg + 8u * static_cast<uint32_t>(j * L::S), src, SEG, rhbar);
       }
-      mbar_wait_parity_cluster(bars, (phases >> 2) & 1u);
+      // only the warps whose gathers reach a guard wait for the halo (threads
+      // t <= 8 and t >= 119 with the stencil reach G = NX + 1 <= 72); the
+      // middle warps start their SpMV while the copies are in flight
+      const int w = threadIdx.x >> 5;
+      if (w == 0 || w == NWARP - 1) mbar_wait_parity_cluster(bars, (phases >> 2) & 1u);
       phases ^= 4u;
     } else {
       cooperative_groups::this_cluster().sync();
@@ -715,7 +745,57 @@ struct Line3ClusterComm {
   }
   template <int K>
   __device__ __forceinline__ void sum(double (&v)[K]) {
+    const double none[R] = {0, 0, 0, 0, 0, 0, 0, 0};
+    sum_x<K>(v, none, 0, none);
+  }
+  __device__ __forceinline__ int nloc() const { return min(RPC, n - rank * RPC); }
+  // H2: the rows this thread owns that a neighbour keeps as halo state go to
+  // that neighbour's state field f (the left neighbour's right side, the
+  // right neighbour's left side), completing on its reduction barrier.  Only
+  // the threads of the first G and the last G rows (nleft / rfirst, set by
+  // init_push) send.
+  uint32_t hl = 0, hr = 0, hlb = 0, hrb = 0;  // remote state rows / barriers of this thread
+  __device__ __forceinline__ void init_push() {
+    const int t = threadIdx.x, nl = nloc();
+    if (rank > 0 && R * t < G) {
+      nleft = min(R, G - R * t);
+      hl = mapa_u32(smem_addr(hst + HS * NF + R * t), rank - 1);
+      hlb = mapa_u32(smem_addr(bars + 1), rank - 1);
+    }
+    if (rank < C - 1 && R * t + R > nl - G && R * t < nl) {
+      rfirst = max(0, nl - G - R * t);
+      hr = mapa_u32(smem_addr(hst + (R * t - (nl - G))), rank + 1);
+      hrb = mapa_u32(smem_addr(bars + 1), rank + 1);
+    }
+  }
+  __device__ __forceinline__ void push_rows(const double (&a)[R], int f, int half) {
+    if (nleft == 0 && rfirst == R) return;
+    const uint32_t fo = 8u * static_cast<uint32_t>(f * HS), bo = 8u * static_cast<uint32_t>(half);
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      if (j < nleft) st_async_f64(hl + fo + 8u * j, a[j], hlb + bo);
+      if (j >= rfirst) st_async_f64(hr + fo + 8u * j, a[j], hrb + bo);
+    }
+  }
+  // Cluster-wide sum of K values in two stages (every exchange variant uses
+  // the same order, so all give the same bits): warp butterflies, the 4 warp
+  // partials of the CTA added by lane q of warp 0 (value q), that CTA partial
+  // pushed to every CTA, then the C CTA partials added in rank order.
+  // what: 0 nothing, 1 v, 4 t, 2 r and d (xb), 3 r (restart): the boundary
+  // rows pushed with the reduction (H2)
+  template <int K>
+  __device__ __forceinline__ void sum_x(double (&v)[K], const double (&xa)[R], int what,
+                                        const double (&xb)[R]) {
     static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
+    uint32_t hbytes = 0;
+    if (H2 && what) {
+      const int nb = (rank > 0 ? 1 : 0) + (rank < C - 1 ? 1 : 0);
+      hbytes = static_cast<uint32_t>(8 * G * nb * (what == 2 ? 2 : 1));
+      const int f = what == 1 ? ((vk & 1) ? F_V1 : F_V0) : what == 4 ? F_T : F_R;
+      push_rows(xa, f, buf);
+      if (what == 2) push_rows(xb, F_D, buf);
+      if (what == 1) ++vk;
+    }
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     constexpr int KP = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
     constexpr int SPAN = 32 / KP;
@@ -734,14 +814,22 @@ struct Line3ClusterComm {
     }
 #pragma unroll
     for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
+    double *Wb = sred + buf * (8 * (NWARP + C));  // [8][NWARP] warp partials
+    double *Sb = Wb + 8 * NWARP;                  // [8][C] CTA partials (pushed by peers)
     const int q = lane / SPAN;
-    if (MB && threadIdx.x == 0) mbar_arrive_expect_tx(bars + 1 + buf, static_cast<uint32_t>(K * NP * 8));
-    if ((lane % SPAN) == 0 && q < K) {
-      const uint32_t off = static_cast<uint32_t>((buf * 8 * NP + q * NP + rank * NWARP + warp) * 8);
+    if ((lane % SPAN) == 0 && q < K) Wb[q * NWARP + warp] = a[0];
+    if (MB && threadIdx.x == 0)
+      mbar_arrive_expect_tx(bars + 1 + buf, static_cast<uint32_t>(K * C * 8) + hbytes);
+    __syncthreads();
+    if (threadIdx.x < K) {  // lane k of warp 0: the CTA partial of value k, to every CTA
+      const double2 w01 = reinterpret_cast<const double2 *>(Wb + threadIdx.x * NWARP)[0];
+      const double2 w23 = reinterpret_cast<const double2 *>(Wb + threadIdx.x * NWARP)[1];
+      const double cp = (w01.x + w01.y) + (w23.x + w23.y);
+      const uint32_t off = static_cast<uint32_t>((Sb - sred + threadIdx.x * C + rank) * 8);
 #pragma unroll
       for (int r = 0; r < C; ++r) {
-        if (MB) push(mapa_u32(sred_s + off, r), a[0], mapa_u32(smem_addr(bars + 1 + buf), r));
-        else peer(sred, r)[off / 8] = a[0];
+        if (MB) push(mapa_u32(sred_s + off, r), cp, mapa_u32(smem_addr(bars + 1 + buf), r));
+        else peer(sred, r)[off / 8] = cp;
       }
     }
     if (MB) {
@@ -751,21 +839,70 @@ struct Line3ClusterComm {
     } else {
       cooperative_groups::this_cluster().sync();
     }
-    const double *Sx = sred + buf * (8 * NP);
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      double part[NP];
-      const double2 *S2 = reinterpret_cast<const double2 *>(Sx + k * NP);
+      double part[C];
 #pragma unroll
-      for (int w = 0; w < NP / 2; ++w) {
-        const double2 qq = S2[w];
-        part[2 * w] = qq.x;
-        part[2 * w + 1] = qq.y;
-      }
-      v[k] = tree_sum<NP>(part);
+      for (int r = 0; r < C; ++r) part[r] = Sb[k * C + r];
+      v[k] = tree_sum<C>(part);
     }
     buf ^= 1;
   }
+  // ---- H2 halo state updates (threads t < G, one row per side each) --------
+  // guard slot of halo row i of side s in this CTA's planes
+  __device__ __forceinline__ double *guard(int side, int i) const {
+    const int x = side == 0 ? i - G : nloc() + i;  // local row index (< 0 or >= nloc)
+    const int q = x >= 0 ? x / R : -((-x + R - 1) / R);
+    return gq - threadIdx.x + (x - R * q) * L::S + q;
+  }
+  __device__ __forceinline__ bool side_ok(int side) const {
+    return side == 0 ? rank > 0 : rank < C - 1;
+  }
+  __device__ __forceinline__ double &hv(int side, int f, int i) const {
+    return hst[side * (HS * NF) + f * HS + i];
+  }
+  __device__ __forceinline__ void halo_p(double beta, double omega) {  // p = r + beta (p - omega v)
+    const int i = threadIdx.x;
+    if (!H2 || i >= G) return;
+    const int fv = ((vk - 1) & 1) ? F_V1 : F_V0;
+#pragma unroll
+    for (int sd = 0; sd < 2; ++sd)
+      if (side_ok(sd)) {
+        const double pn = hv(sd, F_R, i) + beta * (hv(sd, F_P, i) - omega * hv(sd, fv, i));
+        hv(sd, F_P, i) = pn;
+        *guard(sd, i) = hv(sd, F_D, i) * pn;
+      }
+  }
+  __device__ __forceinline__ void halo_s(double alpha) {  // s = r - alpha v
+    const int i = threadIdx.x;
+    if (!H2 || i >= G) return;
+    const int fv = ((vk - 1) & 1) ? F_V1 : F_V0;
+#pragma unroll
+    for (int sd = 0; sd < 2; ++sd)
+      if (side_ok(sd)) {
+        const double sn = hv(sd, F_R, i) - alpha * hv(sd, fv, i);
+        hv(sd, F_R, i) = sn;
+        *guard(sd, i) = hv(sd, F_D, i) * sn;
+      }
+  }
+  __device__ __forceinline__ void halo_r(double omega) {  // r = s - omega t
+    const int i = threadIdx.x;
+    if (!H2 || i >= G) return;
+#pragma unroll
+    for (int sd = 0; sd < 2; ++sd)
+      if (side_ok(sd)) hv(sd, F_R, i) = hv(sd, F_R, i) - omega * hv(sd, F_T, i);
+  }
+  __device__ __forceinline__ void halo_restart() {  // p = v = 0 (r came with the residual)
+    const int i = threadIdx.x;
+    if (!H2 || i >= G) return;
+#pragma unroll
+    for (int sd = 0; sd < 2; ++sd) {
+      hv(sd, F_P, i) = 0.0;
+      hv(sd, F_V0, i) = 0.0;
+      hv(sd, F_V1, i) = 0.0;
+    }
+  }
+  __device__ __forceinline__ void sync_local() { __syncthreads(); }
 };
 
 template <int NX, int C>
@@ -773,13 +910,14 @@ struct Line3ClusterGeom {
   using G3 = Line3Geom<NX, 0>;
   static constexpr int R = 8, NT = 128;
   static constexpr int OFF_RED = G3::OFF_RED;                         // [2][8][C*4]
-  static constexpr int OFF_X = (OFF_RED + 2 * 8 * C * 4 + 1) & ~1;
-  static constexpr int OFF_BAR = OFF_X + R * NT;  // 3 mbarriers (MB = 1)
+  static constexpr int OFF_X = (OFF_RED + 2 * 8 * (4 + C) + 1) & ~1;  // scratch [2][8][4 + C]
+  static constexpr int OFF_HS = OFF_X + R * NT;       // halo state [2][6][66] (H2)
+  static constexpr int OFF_BAR = OFF_HS + 2 * 6 * 66;  // 3 mbarriers (MB = 1)
   static constexpr int SMEM_BYTES = (OFF_BAR + 3) * 8 + 16;
 };
 
 // One system per cluster of C CTAs x 1024 rows (blockIdx.x / C = system).
-template <int NX, int C, int MB = 1, int ROUNDS = 2>
+template <int NX, int C, int MB = 1, int H2 = 1, int ROUNDS = 2>
 __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const SolveParams P) {
   using CG = Line3ClusterGeom<NX, C>;
   constexpr int R = 8, NT = 128;
@@ -789,6 +927,7 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const So
   double *sred = sg + CG::OFF_RED;
   double2 *sx2 = reinterpret_cast<double2 *>(sg + CG::OFF_X) + threadIdx.x;
   uint64_t *bars = reinterpret_cast<uint64_t *>(sg + CG::OFF_BAR);
+  double *hst = sg + CG::OFF_HS;
   uint32_t *tbase_s = reinterpret_cast<uint32_t *>(sg + CG::OFF_BAR + 3);
   uint32_t crank;
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
@@ -811,6 +950,8 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const So
     const int pl = i / (L::S - NT), q = i % (L::S - NT);
     sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
   }
+  if (H2)
+    for (int i = tid; i < 2 * 6 * 66; i += NT) hst[i] = 0.0;
   if (rank == 0 && tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {
     const long long ns = sys + P.pf_ahead;
     const void *va = P.values + ns * P.sys_stride;
@@ -840,11 +981,15 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const So
   const uint32_t tval = tbase_s[0] + lane_hi;
   const uint32_t trh = tbase_s[1] + lane_hi;
   const uint32_t ta0 = trh + 16;
-  Line3ClusterComm<NX, C, MB> comm(sg, sred, bars, rank, n);
+  Line3ClusterComm<NX, C, MB, H2> comm(sg, sred, bars, rank, n, hst);
   line3_solve<NX, ROUNDS, 0>(P, sys, grow0, rank == 0 && tid == 0, act, comm, nullptr, sx2, tval,
                              trh, ta0);
   asm volatile("tcgen05.fence::before_thread_sync;");
-  cluster_barrier();  // no CTA leaves while a peer may still store into its SMEM
+  // no CTA leaves while a peer may still store into its SMEM.  MB = 1: the
+  // last exchange is a reduction whose pushes into this CTA all completed on
+  // its barrier before the wait above returned -- a CTA barrier suffices
+  if (MB) __syncthreads();
+  else cluster_barrier();
   if (warp == 0) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[1]), "n"(32));
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase_s[0]), "n"(128));

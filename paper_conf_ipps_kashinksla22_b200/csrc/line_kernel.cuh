@@ -83,6 +83,18 @@ struct LineComm {
   __device__ __forceinline__ void sum(double (&v)[K]) {
     block_sum<K, NT / 32>(v, sred, buf, threadIdx.x & 31, threadIdx.x >> 5);
   }
+  // (cluster halo-state interface of line3_solve; nothing to exchange here)
+  static constexpr bool kHalo2 = false;
+  template <int K>
+  __device__ __forceinline__ void sum_x(double (&v)[K], const double (&)[R], int,
+                                        const double (&)[R]) {
+    sum<K>(v);
+  }
+  __device__ __forceinline__ void halo_p(double, double) {}
+  __device__ __forceinline__ void halo_s(double) {}
+  __device__ __forceinline__ void halo_r(double) {}
+  __device__ __forceinline__ void halo_restart() {}
+  __device__ __forceinline__ void sync_local() { __syncthreads(); }
 };
 
 __device__ __forceinline__ double tmem_f64(const uint32_t (&w)[16], int c) {

@@ -650,3 +650,29 @@ def test_csr_values_on_the_line_plan(nx, ny, solver, precond):
         o = O.batch_krylov(p.row_ptr, p.col_idx, B.values, B.b,
                            precond=O.block_jacobi(8) if precond == "block_jacobi" else O.PREC_JACOBI)
         compare(p.row_ptr, p.col_idx, B.values, B.b, gc, o=o)
+
+
+@pytest.mark.parametrize("nx,ny", [(64, 63), (64, 33), (64, 120)])
+def test_cluster_exchange_variants_bitwise(nx, ny, monkeypatch):
+    """The three exchanges of the 3-CTA cluster kernel compute the same
+    arithmetic: halo state recomputed per CTA (default, 2 exchanges per
+    iteration), bulk halo copies (4 exchanges) and the cluster-barrier
+    reference give bitwise identical x, iters, resnorm and status -- the
+    recomputed guard values are the owners' bits (warm start and maxiter
+    exhaustion included)."""
+    B = X.make_batch(0, 10, nx=nx, ny=ny)
+    p = B.pattern
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-4)
+    outs = []
+    for sync in ("state", "halo", "barrier"):
+        monkeypatch.setenv("BSOLVE_CLUSTER_SYNC", sync)
+        g = [gpu_solve(p.row_ptr, p.col_idx, B.values, B.b),
+             gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0),
+             gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=7)]
+        assert g[0]["info"]["placement"] == 4
+        outs.append(g)
+    for g in outs[1:]:
+        for a, b in zip(outs[0], g):
+            for k in ("x", "iters", "resnorm", "status"):
+                assert np.array_equal(a[k], b[k]), k
+    compare(p.row_ptr, p.col_idx, B.values, B.b, outs[0][0])
