@@ -104,8 +104,6 @@ struct bsolve_plan {
   int32_t *d_vidx = nullptr;         // CSR values on the line plan: [9][n] value index of
                                      // canonical slot c (8 = diagonal) of row r, -1 none
   int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};  // its canonical offset -> ELL slot map
-  persist_fn var_tmem_p = nullptr;   // persistent TMEM kernel (aligned buffers)
-  int smem_bytes_tmem_p = 0, grid_tmem_p = 0;
   int cluster = 0;                   // CTAs per system (cluster plan)
   int smem_bytes_fallback = 0, grid_persist = 0;
   unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
@@ -496,7 +494,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       // strided-row kernel at n = 4032 (its halo rows are sent by 9 threads
       // with 8 st.async each; 255 registers with spills)
       const char *clenv = getenv("BSOLVE_CLUSTER_LINE");
-      const int cl_line = clenv ? atoi(clenv) : 3;  // 3: 3-CTA line kernel, 1: 2-CTA, 0: strided
+      const int cl_line = clenv ? atoi(clenv) : 3;  // 3: 3-CTA line kernel, 0: strided rows
       int line_smem = 0;
       // canonical stencil slot -> ELL slot for an NX-wide grid (false: not that grid)
       auto map_c2s = [&](int NX, int (&c2s)[8]) {
@@ -514,10 +512,9 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         }
         return true;
       };
-      if (ctmem && (cl_line == 1 || cl_line == 3)) {
+      if (ctmem && cl_line == 3) {
         int cnt = 0;
-        const CVariant *t = cl_line == 3 ? variants_cluster_line3(&cnt, &line_smem)
-                                         : variants_cluster_line(&cnt, &line_smem);
+        const CVariant *t = variants_cluster_line3(&cnt, &line_smem);
         const char *csenv = getenv("BSOLVE_CLUSTER_SYNC");  // "barrier": the reference exchange
         // BSOLVE_CLUSTER_SYNC: default / "halo": bulk halo copies + two-stage
         // reductions on mbarriers (measured fastest); "state": halo state kept
@@ -528,12 +525,12 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                                                                        : 1;
         for (int i = 0; i < cnt && !h->cvar; ++i) {
           if (t[i].c != c) continue;
-          if (cl_line == 3 && t[i].rounds != mb) continue;
+          if (t[i].rounds != mb) continue;
           int c2s[8];
           if (!map_c2s(t[i].kreg, c2s)) continue;
           h->cvar = &t[i];
           h->line_nx = t[i].kreg;
-          h->line_ctas = cl_line == 3 ? 3 : 2;
+          h->line_ctas = 3;
           for (int cc = 0; cc < 8; ++cc) h->c2s[cc] = c2s[cc];
         }
       }
@@ -591,9 +588,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   // Line-tiled variant (DESIGN.md "Kernels" 10): the pattern is a 2D 9-point
   // (or 5-point, ...) stencil on an NX-wide grid for a compiled NX, i.e. every
   // slot offset is one of {+-1, +-NX, +-NX+-1}; it is preferred whenever it
-  // applies.  Developer knobs: BSOLVE_TMEM_LINE=0 keeps the strided kernel,
-  // BSOLVE_TMEM_GROUP = rows per TMEM load group.
-  const char *genv = getenv("BSOLVE_TMEM_GROUP");
+  // applies.  Developer knob: BSOLVE_TMEM_LINE=0 keeps the strided kernel.
   const LVariant *line_v = nullptr;
   int line_c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
   {
@@ -607,9 +602,6 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
                           opt.placement == BSOLVE_PLACE_TMEM);
     int lcnt = 0;
     const LVariant *lv = line_on ? variants_line(&lcnt) : nullptr;
-    const int lg = genv ? atoi(genv) : 4;  // measured best: 7.33 vs 7.05 (G=2) M sys/s
-    const char *rowsenv = getenv("BSOLVE_TMEM_LINE_ROWS");  // rows per thread: 8 or 4
-    const int lr = rowsenv ? atoi(rowsenv) : 8;
     // developer knobs: BSOLVE_LINE_CTAS = 2 selects the 2-CTA line kernel
     // (line_kernel.cuh) instead of the 3-CTA one (line3_kernel.cuh);
     // BSOLVE_ROUNDS = reduction rounds per BiCGSTAB iteration (3-CTA default
@@ -627,7 +619,6 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       if (bj && i >= lcnt) continue;  // block-Jacobi: the 3-CTA kernel only
       if (i < lcnt) {
         if (!bj && cand.ctas != lctas) continue;
-        if (lctas == 2 && (cand.g != lg || cand.r != lr)) continue;
       } else if (cand.ctas != 2) {
         continue;
       }
@@ -677,23 +668,15 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       h->r = line_v->r;
       h->line_ctas = line_v->ctas;
     } else {
-      // developer knobs: rows per TMEM load group, threads per CTA
-      const char *tenv = getenv("BSOLVE_TMEM_THREADS");
-      const int ntsel = opt.block_threads ? opt.block_threads : (tenv ? atoi(tenv) : 128);
-      const int gsel = genv ? atoi(genv) : (ntsel == 128 ? 4 : 2);
-      const char *renv = getenv("BSOLVE_TMEM_ROUNDS");  // developer knob: reduction rounds
-      const int rsel = renv ? atoi(renv) : 3;
+      // strided TMEM kernel (patterns the line plan does not cover): 128
+      // threads x 8 rows, 4 rows per tcgen05.ld wait
+      if (opt.block_threads != 0 && opt.block_threads != 128)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "the TMEM plan runs 128 threads per CTA"));
       int tcnt = 0;
       const TVariant *tv = variants_tmem(&tcnt);
-      for (int i = 0; i < tcnt; ++i)
-        if (tv[i].g == gsel && tv[i].nt == ntsel && tv[i].rounds == rsel) {
-          h->var_tmem = tv[i].fn;
-          h->nt = tv[i].nt;
-          h->r = tv[i].r;
-        }
-      if (!h->var_tmem)
-        return fail_free(fail(BSOLVE_ERR_INVALID, "no TMEM variant for %d threads, group %d",
-                              ntsel, gsel));
+      h->var_tmem = tv[0].fn;
+      h->nt = tv[0].nt;
+      h->r = tv[0].r;
       h->smem_bytes =
           h->smem_vals * 8 + (h->n_pad + 2 * h->guard) * 8 + 16 * (h->nt / 32) * 8 + 16;
     }
@@ -735,57 +718,6 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     }
     if (h->ctas_per_sm < 1)
       return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "TMEM variant cannot be resident"));
-    // persistent variant with TMA prefetch of the next system (needs 16-byte
-    // aligned system blocks; the launch also checks the buffer addresses)
-    // (opt-in via BSOLVE_TMEM_PERSIST=1: measured no faster than the per-system
-    // launch, 6.89 vs 6.91 M sys/s -- the co-resident CTA already hides a
-    // CTA's start-up)
-    // line-tiled plan, persistent with TMA prefetch of the next system
-    // (BSOLVE_LINE_PERSIST=1; 16-byte aligned system blocks, 8 rows/thread)
-    const char *lpenv = getenv("BSOLVE_LINE_PERSIST");
-    if (h->line_nx && lpenv && atoi(lpenv) == 1 && h->r == 8 && n % 2 == 0 &&
-        h->fmt == FMT_ELL && h->line_ctas == 2 &&
-        (h->sys_stride * 8) % 16 == 0) {
-      int sb = 0;
-      persist_fn f = variant_line_persist(h->line_nx, &sb, h->smem_vals, h->n_pad);
-      if (f && sb <= smem_optin &&
-          cudaFuncSetAttribute((const void *)f, cudaFuncAttributeMaxDynamicSharedMemorySize, sb) ==
-              cudaSuccess) {
-        cudaFuncSetAttribute((const void *)f, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             cudaSharedmemCarveoutMaxShared);
-        h->var_tmem_p = f;
-        h->smem_bytes_tmem_p = sb;
-        h->grid_tmem_p = 2 * h->num_sms;
-        if (cudaMalloc(&h->d_ctr, 2 * sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMemset(h->d_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
-          return fail_free(fail(BSOLVE_ERR_NOMEM, "work counter allocation failed"));
-      } else {
-        cudaGetLastError();
-      }
-    }
-    const char *penv = getenv("BSOLVE_TMEM_PERSIST");
-    const bool persist = (penv && atoi(penv) == 1) && !h->line_nx && h->nt == 128 && h->r == 8 &&
-                         n % 2 == 0 && (h->sys_stride * 8) % 16 == 0;
-    if (persist) {
-      h->var_tmem_p = variant_tmem_persist();
-      h->smem_bytes_tmem_p = h->smem_vals * 8 + 2 * h->n_pad * 8 +
-                             (h->n_pad + 2 * h->guard) * 8 + 16 * 4 * 8 + 32;
-      if (h->smem_bytes_tmem_p > smem_optin ||
-          cudaFuncSetAttribute((const void *)h->var_tmem_p,
-                               cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               h->smem_bytes_tmem_p) != cudaSuccess) {
-        cudaGetLastError();
-        h->var_tmem_p = nullptr;
-      } else {
-        cudaFuncSetAttribute((const void *)h->var_tmem_p,
-                             cudaFuncAttributePreferredSharedMemoryCarveout,
-                             cudaSharedmemCarveoutMaxShared);
-        h->grid_tmem_p = 2 * h->num_sms;  // 2 CTAs per SM (255 regs x 128 threads, ~96 KB)
-        if (cudaMalloc(&h->d_ctr, 2 * sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMemset(h->d_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
-          return fail_free(fail(BSOLVE_ERR_NOMEM, "work counter allocation failed"));
-      }
-    }
   }
   // rows per thread / CTA size.  Auto: 9-point stencils (DIA) up to 1024 rows
   // take the hybrid 128 threads x 8 rows with 4 off-diagonal slots in
@@ -1055,12 +987,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;
   if (h->place == PLACE_TMEM) {  // (unaligned values: the kernel copies without TMA)
-    if (h->var_tmem_p && aligned) {  // persistent (strided or line-tiled plan)
-      const int grid = (int)std::min<long long>(h->grid_tmem_p, count);
-      h->var_tmem_p<<<grid, h->nt, h->smem_bytes_tmem_p, stream>>>(P, h->d_ctr);
-    } else {
-      h->var_tmem<<<count, h->nt, h->smem_bytes, stream>>>(P);
-    }
+    h->var_tmem<<<count, h->nt, h->smem_bytes, stream>>>(P);
   } else if (h->place == PLACE_CLUSTER) {
     if ((reinterpret_cast<uintptr_t>(values) & 15u) != 0)
       return fail(BSOLVE_ERR_INVALID, "the cluster plan needs 16-byte aligned values (TMA)");

@@ -24,13 +24,8 @@ static const CVariant kCTVariants[] = {CVT_(2), CVT_(3), CVT_(4), CVT_(5),
                                        CVT_(6), CVT_(7), CVT_(8)};
 
 // TMEM-resident values: 128 threads x 8 rows (or 256 x 4), G rows per load group
-static const TVariant kTVariants[] = {
-    {128, 8, 1, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 1>},
-    {128, 8, 2, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 2>},
-    {128, 8, 4, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>},
-    // (2-round schedule variants measured 6.1-6.4 vs 6.9 M sys/s: removed)
-    {256, 4, 1, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 1>},
-    {256, 4, 2, 3, (solve_fn)bicgstab_tmem_kernel<4, 256, 2>}};
+// (row groups 1, 2 and 256 x 4 geometries measured slower: removed in round 2)
+static const TVariant kTVariants[] = {{128, 8, 4, 3, (solve_fn)bicgstab_tmem_kernel<8, 128, 4>}};
 
 #define COUNT_(T) (int)(sizeof(T) / sizeof(T[0]))
 const PVariant *variants_persist(int *count) {
@@ -49,4 +44,3 @@ const TVariant *variants_tmem(int *count) {
   *count = COUNT_(kTVariants);
   return kTVariants;
 }
-persist_fn variant_tmem_persist() { return (persist_fn)bicgstab_tmem_persist_kernel<8, 128, 4>; }

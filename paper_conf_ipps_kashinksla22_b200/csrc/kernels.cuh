@@ -1112,124 +1112,6 @@ __global__ void __launch_bounds__(NT, 2) bicgstab_tmem_kernel(const SolveParams 
                  "n"(TCOLS < 32 ? 32 : TCOLS));
 }
 
-// Persistent TMEM plan (PLACE_TMEM default): 2 CTAs per SM loop over systems
-// claimed from a self-resetting device counter.  Once a system's values sit
-// in TMEM (and b, x0 in registers) the SMEM staging buffers are free, so
-// thread 0 immediately claims the next system and TMA-prefetches its values,
-// b and x0 while the CTA iterates on the current one: the HBM load and the
-// CTA start-up leave the critical path.
-//   SMEM: [values staging: smem_vals] [b: n_pad] [x0: n_pad]
-//         [gather: guard | n_pad | guard] [scratch: 16*NWARP]
-//         [mbarrier] [next-system slot] [TMEM base]
-template <int R, int NT, int G>
-__global__ void __launch_bounds__(NT, 2) bicgstab_tmem_persist_kernel(const SolveParams P,
-                                                                      unsigned long long *ctr) {
-  constexpr int NWARP = NT / 32;
-  constexpr int WB = 9;
-  constexpr int TCOLS = 16 * R;
-  static_assert(NT == 128 && TCOLS <= 256, "one warp per TMEM lane quarter");
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double *sval = reinterpret_cast<double *>(smem_raw);
-  double *sb = sval + P.smem_vals;
-  double *sx0 = sb + P.n_pad;
-  double *sgf = sx0 + P.n_pad;
-  double *sg = sgf + P.guard;
-  double *sred = sgf + P.n_pad + 2 * P.guard;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
-  volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
-  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 2);
-  const unsigned char *gb = reinterpret_cast<const unsigned char *>(sg);
-
-  const int tid = threadIdx.x, warp = tid >> 5;
-  const int n = P.n;
-  const long long batch = P.batch;
-  const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
-  const uint32_t nbytes = static_cast<uint32_t>(n * 8);
-  auto issue = [&](long long s) {  // thread 0: TMA of system s into the staging buffers
-    mbar_arrive_expect_tx(mbar, vbytes + nbytes + (P.x0 ? nbytes : 0u));
-    const unsigned char *src = reinterpret_cast<const unsigned char *>(P.values + s * P.sys_stride);
-    constexpr uint32_t CH = 32768;
-    for (uint32_t off = 0; off < vbytes; off += CH)
-      tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off, src + off,
-                   vbytes - off < CH ? vbytes - off : CH, mbar);
-    tma_bulk_g2s(sb, P.b + s * n, nbytes, mbar);
-    if (P.x0) tma_bulk_g2s(sx0, P.x0 + s * n, nbytes, mbar);
-  };
-
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_addr(tbase_s)),
-                 "n"(TCOLS));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  for (int i = tid; i < P.guard; i += NT) {
-    sgf[i] = 0.0;
-    sg[P.n_pad + i] = 0.0;
-  }
-  bool act[R];
-  int vrow[R];
-#pragma unroll
-  for (int j = 0; j < R; ++j) {
-    const int row = tid + j * NT;
-    act[j] = row < n;
-    vrow[j] = row < n ? row : n - 1;
-  }
-  if (tid == 32) {
-    mbar_init(mbar, 1);
-    fence_mbar_init();
-    const long long first = static_cast<long long>(atomicAdd(ctr, 1ull));
-    *s_next = first;
-    if (first < batch) issue(first);
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;");
-  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
-  long long cur = *s_next;
-  uint32_t phase = 0;
-  CtaComm<R, NT> comm(sg, sred, act);
-  while (cur < batch) {
-    mbar_wait_parity(mbar, phase);
-    phase ^= 1u;
-    double x[R], r[R], d[R], a0[R], bv[R];
-    tmem_fill<R, WB>(tlane, sval, n, vrow, act, a0, d, P.precond);
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      bv[j] = act[j] ? sb[vrow[j]] : 0.0;
-      r[j] = bv[j];
-      x[j] = (P.x0 && act[j]) ? sx0[vrow[j]] : 0.0;
-    }
-    __syncthreads();  // every thread is done with the staging buffers
-    if (tid == 32) {
-      const long long nxt = static_cast<long long>(atomicAdd(ctr, 1ull));
-      *s_next = nxt;
-      if (nxt < batch) {
-        fence_proxy_async_smem();  // generic reads above before the async-proxy writes
-        issue(nxt);
-      }
-    }
-    bicgstab_core<R, NT, true, 3>(
-        P, cur, x, r, d, act, bv, comm, [&](const double(&own)[R], double(&y)[R]) {
-          tmem_spmv<R, G, WB>(tlane, gb, vrow, a0, act, P.doff, own, y);
-        });
-    cur = *s_next;  // written before the core's first barrier
-  }
-  // ---- release TMEM, reset the work counter ---------------------------------
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  if (warp == 0)
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s),
-                 "n"(TCOLS));
-  if (tid == 0) {
-    __threadfence();
-    const unsigned long long done = atomicAdd(ctr + 1, 1ull);
-    if (done == gridDim.x - 1) {
-      atomicExch(ctr, 0ull);
-      atomicExch(ctr + 1, 0ull);
-    }
-  }
-}
-
 // ------------------------------------------ thread-block cluster per system --
 // Systems too large for one CTA (n > 1024 rows, e.g. the 63x64 velocity
 // grid, n = 4032) are split over a cluster of C CTAs

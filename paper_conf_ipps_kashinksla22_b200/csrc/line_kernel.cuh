@@ -305,362 +305,4 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s), "n"(128));
 }
 
-// Persistent variant of the line-tiled TMEM kernel: 2 CTAs per SM loop over
-// systems claimed from a self-resetting work counter (dynamic, so ion and
-// electron systems balance).  While a CTA iterates on system i, a TMA bulk
-// copy stages system i+1's values, b and x0 into SMEM; at the switch the
-// threads move them SMEM -> registers / TMEM (tens of cycles instead of an
-// HBM round trip on the critical path).
-//   SMEM: [values staging: smem_vals] [b: n_pad] [x0: n_pad] [gather planes]
-//         [reduction scratch: 16 * NWARP] [mbarrier] [next system] [TMEM base]
-template <int NX, int R, int G>
-__host__ __device__ constexpr int line_persist_smem(int smem_vals, int n_pad) {
-  return (smem_vals + 2 * n_pad + R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 +
-         32;
-}
-
-template <int NX, int R, int G>
-__global__ void __launch_bounds__(1024 / R, 2)
-    bicgstab_tmem_line_persist_kernel(const SolveParams P, unsigned long long *ctr) {
-  constexpr int NT = 1024 / R, NWARP = NT / 32;
-  static_assert(R == 8, "8 rows per thread (one warp per TMEM lane quarter)");
-  using L = LineGeom<NX, NT, R>;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double *sval = reinterpret_cast<double *>(smem_raw);
-  double *sb = sval + P.smem_vals;
-  double *sx0 = sb + P.n_pad;
-  double *sg = sx0 + P.n_pad;
-  double *sred = sg + R * L::S;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * NWARP);
-  volatile long long *s_next = reinterpret_cast<volatile long long *>(mbar + 1);
-  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 2);
-
-  const int tid = threadIdx.x, warp = tid >> 5;
-  const int n = P.n;
-  const long long batch = P.batch;
-  const int row0 = R * tid;
-  const uint32_t vbytes = static_cast<uint32_t>(P.sys_stride * 8);
-  const uint32_t nbytes = static_cast<uint32_t>(n * 8);
-  auto issue = [&](long long s) {  // one thread: TMA of system s into the staging buffers
-    mbar_arrive_expect_tx(mbar, vbytes + nbytes + (P.x0 ? nbytes : 0u));
-    const unsigned char *src = reinterpret_cast<const unsigned char *>(P.values + s * P.sys_stride);
-    constexpr uint32_t CH = 32768;
-    for (uint32_t off = 0; off < vbytes; off += CH)
-      tma_bulk_g2s(reinterpret_cast<unsigned char *>(sval) + off, src + off,
-                   vbytes - off < CH ? vbytes - off : CH, mbar);
-    tma_bulk_g2s(sb, P.b + s * n, nbytes, mbar);
-    if (P.x0) tma_bulk_g2s(sx0, P.x0 + s * n, nbytes, mbar);
-  };
-
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_addr(tbase_s)),
-                 "n"(128));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  for (int i = tid; i < R * (L::S - NT); i += NT) {  // zero guard columns once
-    const int pl = i / (L::S - NT), q = i % (L::S - NT);
-    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
-  }
-  bool act[R];
-#pragma unroll
-  for (int j = 0; j < R; ++j) act[j] = row0 + j < n;
-  if (tid == 32) {
-    mbar_init(mbar, 1);
-    fence_mbar_init();
-    const long long first = static_cast<long long>(atomicAdd(ctr, 1ull));
-    *s_next = first;
-    if (first < batch) issue(first);
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;");
-  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
-  long long cur = *s_next;
-  uint32_t phase = 0;
-  LineComm<NX, NT, R> comm(sg, sred, act);
-  while (cur < batch) {
-    mbar_wait_parity(mbar, phase);
-    phase ^= 1u;
-    double x[R], r[R], d[R], a0[R], bv[R];
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      a0[j] = act[j] ? sval[row0 + j] : 0.0;
-      d[j] = jacobi_inv(P.precond, a0[j]);
-      bv[j] = act[j] ? sb[row0 + j] : 0.0;
-      r[j] = bv[j];
-      x[j] = (act[j] && P.x0) ? sx0[row0 + j] : 0.0;
-    }
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      uint32_t w[16];
-#pragma unroll
-      for (int c = 0; c < 8; ++c) {
-        const int k = P.c2s[c];
-        const double v = (act[j] && k >= 0) ? sval[(long long)k * n + row0 + j] : 0.0;
-        w[2 * c] = static_cast<uint32_t>(__double2loint(v));
-        w[2 * c + 1] = static_cast<uint32_t>(__double2hiint(v));
-      }
-      tmem_st16(tlane + 16 * j, w);
-    }
-    tmem_wait_st();
-    __syncthreads();  // every thread is done with the staging buffers
-    if (tid == 32) {
-      const long long nxt = static_cast<long long>(atomicAdd(ctr, 1ull));
-      *s_next = nxt;
-      if (nxt < batch) {
-        fence_proxy_async_smem();  // generic reads above before the async-proxy writes
-        issue(nxt);
-      }
-    }
-    auto spmv = [&](const double(&own)[R], double(&y)[R]) {
-      line_spmv<NX, NT, R, G>(tlane, comm.gq, a0, own, y);
-    };
-    bicgstab_core<R, NT, true, 3>(P, cur, x, r, d, act, bv, comm, spmv);
-    cur = *s_next;  // written before the core's first barrier
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  if (warp == 0)
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s), "n"(128));
-  if (tid == 0) {
-    __threadfence();
-    const unsigned long long done = atomicAdd(ctr + 1, 1ull);
-    if (done == gridDim.x - 1) {
-      atomicExch(ctr, 0ull);
-      atomicExch(ctr + 1, 0ull);
-    }
-  }
-}
-
-
-// ---------------------------------- line-tiled TMEM plan on a CTA cluster --
-// Systems larger than one CTA (n > 1024, e.g. the 63 x 64 grid, n = 4032;
-// SURVEY.md 8(f) f2, BASELINE configs[4]) on C CTAs of 1024 consecutive rows
-// each, every CTA running the line-tiled TMEM SpMV of bicgstab_tmem_line_kernel
-// on its rows.  The plane guards, which hold zeros in the single-CTA kernel,
-// hold the neighbours' halo rows here: publishing row li also st.async's it
-// into the left neighbour's right guard (li < G) or the right neighbour's
-// left guard (li >= nloc - G), G = NX + 1 (the stencil reach), completing the
-// neighbour's halo mbarrier; reductions exchange warp partials through DSMEM
-// (same protocol as ClusterComm, kernels.cuh).
-template <int NX, int C>
-struct ClusterLineComm {
-  static constexpr int R = 8, NT = 128, NWARP = NT / 32, RPC = R * NT;
-  static constexpr int G = NX + 1;
-  using L = LineGeom<NX, NT, R>;
-  double *gq;    // sg + GQ + threadIdx.x
-  double *sg;
-  double *sred;  // scratch [2][8][C * NWARP]
-  uint64_t *hbar, *rbar;
-  uint32_t left_sg = 0, right_sg = 0, left_hbar = 0, right_hbar = 0, sred_s, rbar_s;
-  uint32_t hphase = 0, rphase = 0;
-  int buf = 0, rank, nloc, halo_bytes;
-  const bool (&act)[R];
-  __device__ __forceinline__ ClusterLineComm(double *sg_, double *sred_, uint64_t *bars, int rank_,
-                                             int n, const bool (&act_)[R])
-      : gq(sg_ + L::GQ + threadIdx.x), sg(sg_), sred(sred_), hbar(bars), rbar(bars + 1),
-        rank(rank_), nloc(min(RPC, n - rank_ * RPC)), act(act_) {
-    const uint32_t sg_s = smem_addr(sg), hb_s = smem_addr(hbar);
-    if (rank > 0) {
-      left_sg = mapa_u32(sg_s, rank - 1);
-      left_hbar = mapa_u32(hb_s, rank - 1);
-    }
-    if (rank < C - 1) {
-      right_sg = mapa_u32(sg_s, rank + 1);
-      right_hbar = mapa_u32(hb_s, rank + 1);
-    }
-    sred_s = smem_addr(sred);
-    rbar_s = smem_addr(rbar);
-    const int nright = rank < C - 1 ? min(RPC, n - (rank + 1) * RPC) : 0;
-    halo_bytes = 8 * ((rank > 0 ? G : 0) + min(G, nright));
-  }
-  // element offset of local row li (may be < 0 or >= RPC: a guard) in the planes
-  __device__ __forceinline__ static uint32_t plane_off(int li) {
-    const int q = li >= 0 ? li / R : -((-li + R - 1) / R);
-    return static_cast<uint32_t>((li - R * q) * L::S + L::GQ + q);
-  }
-  __device__ __forceinline__ int grow(int j) const { return rank * RPC + R * threadIdx.x + j; }
-  __device__ __forceinline__ bool leader() const { return rank == 0 && threadIdx.x == 0; }
-  __device__ __forceinline__ void publish(int j, double v) {
-    gq[j * L::S] = v;
-    const int li = R * threadIdx.x + j;
-    if (act[j]) {
-      if (li < G && rank > 0)  // my first rows -> left neighbour's right guard
-        st_async_f64(left_sg + 8u * plane_off(RPC + li), v, left_hbar);
-      if (li >= nloc - G && rank < C - 1)  // my last rows -> right neighbour's left guard
-        st_async_f64(right_sg + 8u * plane_off(li - nloc), v, right_hbar);
-    }
-  }
-  // CTA barrier without a halo exchange (no publish preceded it)
-  __device__ __forceinline__ void barrier() { __syncthreads(); }
-  __device__ __forceinline__ void sync() {
-    if (threadIdx.x == 0) mbar_arrive_expect_tx(hbar, static_cast<uint32_t>(halo_bytes));
-    __syncthreads();
-    mbar_wait_parity_cluster(hbar, hphase);
-    hphase ^= 1u;
-  }
-  template <int K>
-  __device__ __forceinline__ void sum(double (&v)[K]) {
-    static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    constexpr int KP = K <= 1 ? 1 : K <= 2 ? 2 : K <= 4 ? 4 : 8;
-    constexpr int SPAN = 32 / KP;
-    double a[KP];
-#pragma unroll
-    for (int i = 0; i < KP; ++i) a[i] = i < K ? v[i] : 0.0;
-#pragma unroll
-    for (int cnt = KP, o = 16; cnt > 1; cnt >>= 1, o >>= 1) {
-      const bool hi = lane & o;
-#pragma unroll
-      for (int i = 0; i < cnt / 2; ++i) {
-        const double send = hi ? a[i] : a[i + cnt / 2];
-        const double keep = hi ? a[i + cnt / 2] : a[i];
-        a[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
-      }
-    }
-#pragma unroll
-    for (int o = SPAN / 2; o > 0; o >>= 1) a[0] += __shfl_xor_sync(0xffffffffu, a[0], o);
-    constexpr int P_ = C * NWARP;
-    const uint32_t bit = 1u << buf;
-    if (threadIdx.x == 0) mbar_arrive_expect_tx(rbar + buf, K * P_ * 8);
-    const int q = lane / SPAN;
-    if ((lane % SPAN) == 0 && q < K) {
-      const uint32_t off = static_cast<uint32_t>((buf * 8 * P_ + q * P_ + rank * NWARP + warp) * 8);
-#pragma unroll
-      for (int r = 0; r < C; ++r)
-        st_async_f64(mapa_u32(sred_s + off, r), a[0], mapa_u32(rbar_s + 8u * buf, r));
-    }
-    mbar_wait_parity_cluster(rbar + buf, (rphase & bit) ? 1u : 0u);
-    rphase ^= bit;
-    const double *Sx = sred + buf * (8 * P_);
-    double part[K][P_];
-#pragma unroll
-    for (int k = 0; k < K; ++k) {
-      const double2 *S2 = reinterpret_cast<const double2 *>(Sx + k * P_);
-#pragma unroll
-      for (int w = 0; w < P_ / 2; ++w) {
-        const double2 qq = S2[w];
-        part[k][2 * w] = qq.x;
-        part[k][2 * w + 1] = qq.y;
-      }
-    }
-#pragma unroll
-    for (int k = 0; k < K; ++k) v[k] = tree_sum<P_>(part[k]);
-    buf ^= 1;
-  }
-};
-
-template <int NX, int C>
-__host__ __device__ constexpr int line_cluster_smem() {
-  return (8 * LineGeom<NX, 128, 8>::S + 16 * C * 4) * 8 + 4 * 8 + 16;
-}
-
-// One system per cluster of C CTAs x 1024 rows, line-tiled TMEM SpMV per CTA.
-//   SMEM per CTA: [gather planes: 8 x S] [scratch: 2 x 8 x C x 4] [3 mbarriers] [TMEM base]
-template <int NX, int C>
-__global__ void __launch_bounds__(128, 2) bicgstab_tmem_line_cluster_kernel(const SolveParams P) {
-  constexpr int R = 8, NT = 128, RPC = R * NT;
-  using L = LineGeom<NX, NT, R>;
-  namespace cg = cooperative_groups;
-  cg::cluster_group cl = cg::this_cluster();
-  const int rank = static_cast<int>(cl.block_rank());
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double *sg = reinterpret_cast<double *>(smem_raw);
-  double *sred = sg + R * L::S;
-  uint64_t *mbar = reinterpret_cast<uint64_t *>(sred + 16 * C * 4);  // halo, red 0, red 1
-  uint32_t *tbase_s = reinterpret_cast<uint32_t *>(mbar + 3);
-
-  const int tid = threadIdx.x, warp = tid >> 5;
-  const int n = P.n;
-  const long long sys = blockIdx.x / C;
-  const int row0 = rank * RPC;
-  const int nloc = min(RPC, n - row0);
-  const int lrow0 = R * tid;  // this thread's first local row
-  const double *gval = P.values + sys * P.sys_stride;
-
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_addr(tbase_s)),
-                 "n"(128));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  if (tid == 32) {
-    for (int i = 0; i < 3; ++i) mbar_init(mbar + i, 1);
-    fence_mbar_init();
-  }
-  // guards: zero everywhere first (global edges stay 0; halo columns are
-  // overwritten by the neighbours' st.async before every gather)
-  for (int i = tid; i < R * (L::S - NT); i += NT) {
-    const int pl = i / (L::S - NT), q = i % (L::S - NT);
-    sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
-  }
-  bool act[R];
-  double x[R], r[R], d[R], a0[R];
-  double val[R][8];
-#pragma unroll
-  for (int j = 0; j < R; ++j) act[j] = lrow0 + j < nloc;
-  const bool vec = !P.vidx && ((n & 1) == 0) && ((reinterpret_cast<uintptr_t>(gval) & 15u) == 0) &&
-                   lrow0 + R <= nloc;
-  if (vec) {
-#pragma unroll
-    for (int j = 0; j < R; j += 2) {
-      const double2 dg = __ldg(reinterpret_cast<const double2 *>(gval + row0 + lrow0 + j));
-      a0[j] = dg.x;
-      a0[j + 1] = dg.y;
-#pragma unroll
-      for (int c = 0; c < 8; ++c) {
-        const int k = P.c2s[c];
-        double2 v = make_double2(0.0, 0.0);
-        if (k >= 0)
-          v = __ldg(reinterpret_cast<const double2 *>(gval + (long long)k * n + row0 + lrow0 + j));
-        val[j][c] = v.x;
-        val[j + 1][c] = v.y;
-      }
-    }
-  } else {
-#pragma unroll
-    for (int j = 0; j < R; ++j) {
-      a0[j] = act[j] ? __ldg(gval + row0 + lrow0 + j) : 0.0;
-#pragma unroll
-      for (int c = 0; c < 8; ++c) {
-        const int k = P.c2s[c];
-        val[j][c] = (act[j] && k >= 0) ? __ldg(gval + (long long)k * n + row0 + lrow0 + j) : 0.0;
-      }
-    }
-  }
-  const double *bsys = P.b + sys * n;
-#pragma unroll
-  for (int j = 0; j < R; ++j) {
-    d[j] = jacobi_inv(P.precond, a0[j]);
-    r[j] = act[j] ? __ldg(bsys + row0 + lrow0 + j) : 0.0;
-    x[j] = (act[j] && P.x0) ? __ldg(P.x0 + sys * n + row0 + lrow0 + j) : 0.0;
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;");
-  const uint32_t tlane = *tbase_s + (static_cast<uint32_t>(32 * (warp & 3)) << 16);
-#pragma unroll
-  for (int j = 0; j < R; ++j) {
-    uint32_t w[16];
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      w[2 * c] = static_cast<uint32_t>(__double2loint(val[j][c]));
-      w[2 * c + 1] = static_cast<uint32_t>(__double2hiint(val[j][c]));
-    }
-    tmem_st16(tlane + 16 * j, w);
-  }
-  tmem_wait_st();
-  cl.sync();  // every CTA of the cluster runs (DSMEM and its mbarriers are live)
-  ClusterLineComm<NX, C> comm(sg, sred, mbar, rank, n, act);
-  auto spmv = [&](const double(&own)[R], double(&y)[R]) {
-    line_spmv<NX, NT, R, 4>(tlane, comm.gq, a0, own, y);
-  };
-  bicgstab_core<R, NT, false, 3>(P, sys, x, r, d, act, r, comm, spmv);
-  asm volatile("tcgen05.fence::before_thread_sync;");
-  cl.sync();  // peers may write into this CTA's SMEM until they are done
-  if (warp == 0)
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tbase_s), "n"(128));
-}
-
 }  // namespace bsolve

@@ -66,12 +66,8 @@ const Variant *variants_generic(int *count);
 const PVariant *variants_persist(int *count);
 const CVariant *variants_cluster(int *count);
 const CVariant *variants_cluster_tmem(int *count);
-// line-tiled cluster plan: c = CTAs, kreg = grid width NX; smem = bytes for C <= 8
-const CVariant *variants_cluster_line(int *count, int *smem_bytes);
 // 3-CTA line-tiled plan on a cluster (line3_kernel.cuh), kreg = grid width NX
 const CVariant *variants_cluster_line3(int *count, int *smem_bytes);
 const TVariant *variants_tmem(int *count);
-persist_fn variant_tmem_persist();
-persist_fn variant_line_persist(int nx, int *smem_bytes, int smem_vals, int n_pad);
 const LVariant *variants_line(int *count);
 const BVariant *variants_banded(int *count);

@@ -462,50 +462,6 @@ def test_tmem_refuses_non_stencil():
     assert S.info["kernel_mode"] == 4
 
 
-@pytest.mark.parametrize("batch", [3, 296, 1000])
-def test_tmem_persistent_repeated_launches_and_fallback(batch, monkeypatch):
-    """Default TMEM plan launches the persistent kernel (self-resetting work
-    counter, TMA prefetch of the next system): back-to-back launches on one
-    handle are identical; batches below / above the 296-CTA grid; misaligned
-    buffers take the per-system kernel with identical results."""
-    monkeypatch.setenv("BSOLVE_TMEM_PERSIST", "1")  # read at bsolve_create
-    B = X.make_batch(0, batch)
-    p = B.pattern
-    S = Solver(p.row_ptr, p.col_idx, batch)
-    assert S.info["placement"] == 5
-    v = to_dev(S.ell_values(B.values))
-    b = to_dev(B.b)
-    outs = [S.run(v, b) for _ in range(3)]
-    torch.cuda.synchronize()
-    for o in outs[1:]:
-        for a, c in zip(outs[0], o):
-            assert torch.equal(a, c)
-    g = dict(x=outs[0][0].cpu().numpy(), iters=outs[0][1].cpu().numpy(),
-             resnorm=outs[0][2].cpu().numpy(), status=outs[0][3].cpu().numpy().astype(np.int32))
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
-    vbig = torch.empty(v.numel() + 1, dtype=torch.float64, device="cuda")
-    vbig[1:] = v.reshape(-1)
-    xf, itf, rf, sf = S.run(vbig[1:].view_as(v), b)
-    torch.cuda.synchronize()
-    assert np.array_equal(itf.cpu().numpy(), g["iters"])
-    assert np.array_equal(xf.cpu().numpy(), g["x"])
-
-
-@pytest.mark.parametrize("rounds,group", [(3, 1), (3, 2)])
-def test_tmem_schedules(rounds, group, monkeypatch):
-    """TMEM plan with other row groups per tcgen05.ld wait: same parity bar."""
-    monkeypatch.setenv("BSOLVE_TMEM_ROUNDS", str(rounds))
-    monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
-    B = X.make_batch(0, 64)
-    p = B.pattern
-    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g)
-    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-3)
-    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
-    o = O.batch_bicgstab(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, maxiter=3)
-    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
-
-
 # ------------------------------------------ line-tiled TMEM kernel (mode 4) --
 def _five_point(nx, ny):
     """5-point stencil pattern (the 9-point pattern without its corners)."""
@@ -575,15 +531,12 @@ def test_line_tmem_matches_strided_plan_and_is_deterministic(monkeypatch):
     assert torch.equal(xa, xm) and torch.equal(ia, im) and torch.equal(ra, rm)
 
 
-@pytest.mark.parametrize("rows,group,nx,ny", [(8, 2, 32, 31), (4, 2, 32, 31), (4, 4, 32, 31),
-                                               (4, 2, 31, 32), (4, 2, 32, 5), (4, 2, 31, 31)])
-def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
-    """Line kernel with 8 rows x 128 threads or 4 rows x 256 threads per CTA
-    (two warps per TMEM lane quarter) and other TMEM load groups: same parity
-    bar, warm start included."""
-    monkeypatch.setenv("BSOLVE_LINE_CTAS", "2")  # geometries of the 2-CTA kernel
-    monkeypatch.setenv("BSOLVE_TMEM_GROUP", str(group))
-    monkeypatch.setenv("BSOLVE_TMEM_LINE_ROWS", str(rows))
+@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32), (32, 5), (31, 31)])
+def test_line_tmem_two_cta_kernel(nx, ny, monkeypatch):
+    """The 2-CTA line kernel (252 registers; the GMRES kernel's BiCGSTAB twin,
+    BSOLVE_LINE_CTAS=2): same parity bar, warm start included."""
+    rows = 8
+    monkeypatch.setenv("BSOLVE_LINE_CTAS", "2")
     B = X.make_batch(0, 64, nx=nx, ny=ny)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
@@ -595,15 +548,13 @@ def test_line_tmem_geometries(rows, group, nx, ny, monkeypatch):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
 
 
-@pytest.mark.parametrize("line", ["3", "1"])
 @pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4), (64, 120, 8)])
-def test_cluster_line_kernel(nx, ny, C, line, monkeypatch):
-    """Line-tiled TMEM cluster kernels: BSOLVE_CLUSTER_LINE=3 (default, the
-    3-CTA line3 kernel per cluster CTA, halo rows and reduction partials by
-    st.shared::cluster + cluster barriers) and =1 (the 2-CTA line kernel,
-    st.async + mbarrier): the plane guards carry the neighbours' halo rows;
-    same parity bar, warm start included."""
-    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", line)
+def test_cluster_line_kernel(nx, ny, C, monkeypatch):
+    """The 3-CTA line kernel on a cluster (default for 64-wide grids, n > 1024):
+    the plane guards carry the neighbours' halo rows (bulk DSMEM copies),
+    reductions in two stages over mbarriers; same parity bar, warm start
+    included."""
+    monkeypatch.setenv("BSOLVE_CLUSTER_LINE", "3")
     B = X.make_batch(0, 12, nx=nx, ny=ny)
     p = B.pattern
     g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b)
@@ -615,7 +566,7 @@ def test_cluster_line_kernel(nx, ny, C, line, monkeypatch):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
 
 
-@pytest.mark.parametrize("line", ["0", "1", "3"])
+@pytest.mark.parametrize("line", ["0", "3"])
 def test_cluster_maxiter_exhausted(line, monkeypatch):
     """Cluster plans (strided and line-tiled) when maxiter runs out: the final
     true-residual check must not wait for a halo nobody sent (regression: the

@@ -15,14 +15,22 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:bicg
     -o $OUT/prof_$TAG python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --parity none \
     > $OUT/ncu_full_$TAG.log 2>&1
 timeout 900 python bench.py --picard 5 --steps 3 --warmup 1 --out $OUT/picard_$TAG.jsonl > $OUT/picard_$TAG.log 2>&1
+timeout 600 python bench.py --precond block_jacobi --steps 10 --warmup 3 --no-e2e --parity sample --cpu-seconds 3 \
+    --out $OUT/bench_bj_$TAG.jsonl > $OUT/bench_bj_$TAG.log 2>&1
+timeout 600 python bench.py --nx 64 --ny 63 --batch 16384 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline \
+    --parity none --out $OUT/bench_n4032_$TAG.jsonl > $OUT/bench_n4032_$TAG.log 2>&1
+timeout 900 python bench.py --solver banded --steps 5 --warmup 2 --no-e2e --cpu-seconds 3 \
+    --out $OUT/bench_banded_$TAG.jsonl > $OUT/bench_banded_$TAG.log 2>&1
+bash tools/r2_table2.sh $TAG
 timeout 600 python tools/iter_sensitivity.py --gpu --n 1000 --out $OUT/iter_sensitivity_$TAG.json \
     > $OUT/iter_sensitivity_$TAG.log 2>&1
 for tool in memcheck racecheck synccheck initcheck; do
-  echo "== compute-sanitizer --tool $tool python tools/sanitize_cases.py (SAN_BATCH=3, line-tiled cases)" >> $OUT/sanitizer_$TAG.txt
-  SAN_BATCH=3 SAN_CASES=line-tiled timeout 900 compute-sanitizer --tool $tool python tools/sanitize_cases.py \
+  echo "== compute-sanitizer --tool $tool python tools/sanitize_cases.py (SAN_BATCH=3)" >> $OUT/sanitizer_$TAG.txt
+  SAN_BATCH=3 timeout 1200 compute-sanitizer --tool $tool python tools/sanitize_cases.py \
       >> $OUT/sanitizer_$TAG.txt 2>&1
   echo "rc=$?" >> $OUT/sanitizer_$TAG.txt
 done
-timeout 300 compute-sanitizer --tool synccheck tools/tmem_probe > $OUT/synccheck_tmem_probe_$TAG.txt 2>&1
-echo "rc=$?" >> $OUT/synccheck_tmem_probe_$TAG.txt
+for mode in 0 1 2 3; do
+  timeout 300 compute-sanitizer --tool racecheck tools/cluster_race_probe $mode > $OUT/race_probe_${TAG}_$mode.txt 2>&1
+done
 echo done

@@ -28,8 +28,6 @@ CASES = [
     ("persistent regs", dict(nx=32, ny=31), dict(placement="regs")),
     ("cluster C=3 (n=2112)", dict(nx=64, ny=33), dict()),
     ("line-tiled cluster C=4 (n=4032)", dict(nx=64, ny=63), dict()),
-    ("line-tiled 2-CTA cluster C=4 (st.async)", dict(nx=64, ny=63), dict(),
-     {"BSOLVE_CLUSTER_LINE": "1"}),
     ("strided cluster C=4 (st.async)", dict(nx=64, ny=63), dict(), {"BSOLVE_CLUSTER_LINE": "0"}),
 ]
 
