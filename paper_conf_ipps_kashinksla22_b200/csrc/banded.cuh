@@ -439,8 +439,11 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
         }
 #endif
         // row j leaves; row j+KL+1 (ring slot j mod R) enters as window row KL
-        v[KL] = ring[jr * RB + rcol];
-        ring[jr * RB + rcol] = 0.0;
+        // (loader lanes own no column: they keep zeros and leave the ring alone)
+        if (owns) {
+          v[KL] = ring[jr * RB + rcol];
+          ring[jr * RB + rcol] = 0.0;
+        }
         pos = t < W ? (pos == 0 ? W - 1 : pos - 1) : pos;
       }
       jr = (jr + 1 == R) ? 0 : jr + 1;
