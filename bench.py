@@ -490,14 +490,18 @@ def run_ours(args, rank, world, local_rank):
             dist.barrier()
         torch.cuda.synchronize()
 
+    nvtx = torch.cuda.nvtx  # ranges for nsys / ncu --nvtx timelines
+    nvtx.range_push("warmup")
     for _ in range(max(args.warmup, 0)):
         S.run(vals, b, None, args.tol, args.maxiter, out=out)
     barrier()
+    nvtx.range_pop()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
     launch_ms = []
     with ClockSampler(local_rank) as clk:
         barrier()
+        nvtx.range_push(f"timed {args.steps} steps")
         ev0.record(stream)
         for _ in range(args.steps):
             e_a = torch.cuda.Event(enable_timing=True)
@@ -508,6 +512,7 @@ def run_ours(args, rank, world, local_rank):
             launch_ms.append((e_a, e_b))
         ev1.record(stream)
         torch.cuda.synchronize()
+        nvtx.range_pop()
         barrier()
     total_ms = ev0.elapsed_time(ev1)
     kern_ms = [a.elapsed_time(bb) for a, bb in launch_ms]
@@ -662,10 +667,12 @@ def run_ours(args, rank, world, local_rank):
         S.run_host(vn, bn, None, args.tol, args.maxiter, out=outs)  # warm-up (allocates)
         e2e_steps = max(1, min(args.steps, 3))
         barrier()
+        nvtx.range_push("e2e (host buffers)")
         t0 = time.perf_counter()
         for _ in range(e2e_steps):
             S.run_host(vn, bn, None, args.tol, args.maxiter, out=outs)
         torch.cuda.synchronize()
+        nvtx.range_pop()
         dt = time.perf_counter() - t0
         dt = max_over_ranks(dt, device=dev)
         h2d = int(vn.nbytes + bn.nbytes)

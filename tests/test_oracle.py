@@ -389,3 +389,27 @@ def test_paper_storage_numbers():
     ell_col, src = X.ell_layout(pat.row_ptr, pat.col_idx)
     assert ell_col.size == facts["ell_slots_9pt_32x31"]["value"]
     assert int(np.sum(src < 0)) == facts["ell_padding_slots"]["value"]
+
+
+def test_paper_vector_planner_accounting():
+    """The paper's SMEM planner (Sec. IV-D): the BiCGSTAB vectors
+    (9 of n doubles, the 4 SpMV vectors first) go to shared memory in priority
+    order while they fit the per-block budget, the rest to global memory.  On
+    the V100 with the default 48 KiB budget and n = 992 that is 6 + 3
+    (golden).  The same byte accounting with B200's 227 KB opt-in
+    budget places all 9 (71.4 KB) on chip; the B200 plan goes further and
+    keeps them off the SMEM data pipe altogether (registers, TMEM; DESIGN.md
+    Kernels 12), so no planner is needed there."""
+    facts = json.load(open(os.path.join(GOLD, "paper_facts.json")))
+    nvec = facts["bicgstab_vectors"]["value"]
+    n = facts["rows"]["value"]
+    vec_bytes = 8 * n
+    def plan(budget):
+        smem = 0
+        for _ in range(nvec):  # priority order; each vector whole or not at all
+            if (smem + 1) * vec_bytes <= budget:
+                smem += 1
+        return smem, nvec - smem
+    v100 = facts["v100_smem_split"]
+    assert plan(v100["budget_bytes"]) == (v100["smem"], v100["global"])
+    assert plan(232448) == (9, 0)  # B200: 227 KB dynamic SMEM per CTA (opt-in)
