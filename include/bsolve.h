@@ -151,10 +151,13 @@ typedef struct bsolve_options {
                               1 <= m <= BSOLVE_MAX_RESTART (default 7)        */
   int direct_fallback;     /* 1: after the iterative solve, every system whose
                               status is not CONVERGED is re-solved by the
-                              banded LU in a second launch
-                              on the same stream and gets status DIRECT; a
-                              singular band keeps the iterative result.
-                              Needs status != NULL in bsolve_run (default 0) */
+                              banded LU on the same stream
+                              and gets status DIRECT; a singular band keeps
+                              the iterative result.  Two more launches per
+                              bsolve_run (a device-side list of the failed
+                              systems, one solve over that list); buffers
+                              are allocated by bsolve_create.  Needs status
+                              != NULL in bsolve_run (default 0)            */
 } bsolve_options;
 
 typedef struct bsolve_info {
@@ -205,7 +208,8 @@ void bsolve_default_options(bsolve_options *opt);
 int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t *row_ptr,
                   const int32_t *col_idx, const bsolve_options *opt);
 
-/* Solve all `batch` systems (one asynchronous kernel launch).
+/* Solve all `batch` systems (one asynchronous kernel launch; 3 with
+ * direct_fallback).
  *   values   DEVICE, batch * nnz (CSR) or batch * W * n (ELL) doubles.
  *   b        DEVICE, batch * n doubles (read only).
  *   x0       DEVICE, batch * n doubles, or NULL for the zero guess; may alias
@@ -275,10 +279,17 @@ int bsolve_ell_layout(int n, const int32_t *row_ptr, const int32_t *col_idx, int
  *           exactly zero pivot u_jj (LAPACK convention: singular).
  *   ipiv    DEVICE, batch * n int32 (out) or NULL: 0-based row interchanged
  *           with row j at step j (ipiv[j] >= j).
- *   stream  cudaStream_t or NULL.  Asynchronous: one kernel launch.
- * The handle owns a workspace of (number of resident CTAs) x n x (2 kb + 2)
- * doubles, kb = max(kl, ku) rounded up to 4, 8, 16, 33 or 65, allocated on
- * the first call.  Errors: INVALID (NULL / foreign pointers), UNSUPPORTED
+ *   stream  cudaStream_t or NULL.  Asynchronous after the first call: per
+ *           chunk of systems two kernel launches (factorisation writing U and
+ *           y to the workspace, then the back substitution; bsolve_info.
+ *           banded_launches reports the count of the last call).
+ * The FIRST call (per handle) is synchronous host work: it builds and uploads
+ * the banded pattern tables and allocates the workspace, n x (2 kb + 2)
+ * doubles per system of a chunk (whole waves of resident CTAs, at most
+ * ~8 GB), kb = max(kl, ku) rounded up to 4, 8, 16, 33 or 65.  With
+ * direct_fallback the tables are built, and the fallback's own bounded
+ * workspace (<= 256 MB) allocated, by bsolve_create; bsolve_run never
+ * allocates.  Errors: INVALID (NULL / foreign pointers), UNSUPPORTED
  * (max(kl, ku) > 65, or a row with more entries than the instance has
  * loader lanes), NOMEM, CUDA. */
 int bsolve_banded_solve(bsolve_handle h, const double *values, const double *b, double *x,
