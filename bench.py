@@ -168,7 +168,10 @@ def make_inputs(g0, count, args, pinned, picard=0):
     CH = 8192
     for c0 in range(0, count, CH):
         c1 = min(count, c0 + CH)
-        Bt = X.make_batch(g0 + c0, c1 - c0, pattern=pat, seed=args.seed, picard=picard)
+        # ranks share the host: split its cores among them for the generator
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        Bt = X.make_batch(g0 + c0, c1 - c0, pattern=pat, seed=args.seed, picard=picard,
+                          threads=max(1, min(32, host_cores() // max(1, world))))
         if args.format == "ell":
             blk = vn[c0:c1]
             blk[:, ~ok] = 0.0
