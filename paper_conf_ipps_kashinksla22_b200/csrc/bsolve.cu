@@ -516,13 +516,13 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         int cnt = 0;
         const CVariant *t = variants_cluster_line3(&cnt, &line_smem);
         const char *csenv = getenv("BSOLVE_CLUSTER_SYNC");  // "barrier": the reference exchange
-        // BSOLVE_CLUSTER_SYNC: default / "halo": bulk halo copies + two-stage
-        // reductions on mbarriers (measured fastest); "state": halo state kept
-        // per CTA, 2 exchanges per iteration (slower: element-wise pushes);
-        // "barrier": cluster barriers (the reference)
-        const int mb = !csenv ? 1 : std::strcmp(csenv, "barrier") == 0 ? 0
-                                  : std::strcmp(csenv, "state") == 0  ? 2
-                                                                       : 1;
+        // BSOLVE_CLUSTER_SYNC: default / "state": halo state kept per CTA, 2
+        // exchanges per iteration, the boundary rows riding the reductions as
+        // bulk copies (measured fastest); "halo": bulk halo copies + two-stage
+        // reductions, 4 exchanges; "barrier": cluster barriers (the reference)
+        const int mb = !csenv ? 2 : std::strcmp(csenv, "barrier") == 0 ? 0
+                                  : std::strcmp(csenv, "halo") == 0   ? 1
+                                                                       : 2;
         for (int i = 0; i < cnt && !h->cvar; ++i) {
           if (t[i].c != c) continue;
           if (t[i].rounds != mb) continue;

@@ -638,7 +638,9 @@ struct Line3ClusterComm {
   // ride along with the two reductions that follow the SpMVs.
   static constexpr bool kHalo2 = H2 != 0;
   static constexpr int HS = 66;  // halo state: [side][field][HS], sides L = 0, R = 1
-  enum { F_D = 0, F_P = 1, F_R = 2, F_V0 = 3, F_V1 = 4, F_T = 5, NF = 6 };
+  static_assert(G <= HS && (HS * 8) % 16 == 0, "halo state rows: bulk-copy granules");
+  // r and d adjacent: the pair pushed together is one bulk copy
+  enum { F_R = 0, F_D = 1, F_P = 2, F_V0 = 3, F_V1 = 4, F_T = 5, NF = 6 };
   static constexpr int NP = C * NWARP;  // partials per reduced value
   using L = LineGeom<NX, NT, R>;
   double *gq;    // sg + GQ + threadIdx.x
@@ -654,10 +656,12 @@ struct Line3ClusterComm {
   uint32_t lseg = 0, rseg = 0;  // MB = 1: bulk-copy destinations (plane 0) in the neighbours
   int n;
   double *hst = nullptr;        // H2: halo state (this CTA's copy of the neighbours' rows)
+  double *stg = nullptr;        // H2: outgoing boundary rows [2 halves][2 sides][2 * HS]
   int vk = 0;                   // H2: v exchanges so far (v is double-buffered by parity)
   __device__ __forceinline__ Line3ClusterComm(double *sg, double *sred_, uint64_t *bars_, int rank_,
                                               int n_, double *hst_ = nullptr)
-      : gq(sg + L::GQ + threadIdx.x), sred(sred_), rank(rank_), bars(bars_), n(n_), hst(hst_) {
+      : gq(sg + L::GQ + threadIdx.x), sred(sred_), rank(rank_), bars(bars_), n(n_), hst(hst_),
+        stg(hst_ ? hst_ + 2 * NF * HS : nullptr) {
     const uint32_t sg_s = smem_addr(sg);
     const int t = threadIdx.x;
     const uint32_t bars_s = smem_addr(bars);
@@ -749,33 +753,46 @@ struct Line3ClusterComm {
     sum_x<K>(v, none, 0, none);
   }
   __device__ __forceinline__ int nloc() const { return min(RPC, n - rank * RPC); }
-  // H2: the rows this thread owns that a neighbour keeps as halo state go to
-  // that neighbour's state field f (the left neighbour's right side, the
-  // right neighbour's left side), completing on its reduction barrier.  Only
-  // the threads of the first G and the last G rows (nleft / rfirst, set by
-  // init_push) send.
-  uint32_t hl = 0, hr = 0, hlb = 0, hrb = 0;  // remote state rows / barriers of this thread
+  // H2: the rows this thread owns that a neighbour keeps as halo state (the
+  // first G rows for the left neighbour, the last G for the right one; nleft /
+  // rfirst, set by init_push) are staged in stg and leave as ONE bulk copy per
+  // side and exchange (thread 32: left, thread 64: right) into the
+  // neighbour's state field, completing on its reduction barrier.  The
+  // staging is double-buffered by reduction half: half h is rewritten two
+  // exchanges later, after a reduction that needed the neighbour's partial,
+  // which it pushed only after its wait for this copy returned.
+  uint32_t hl = 0, hr = 0, hlb = 0, hrb = 0;  // remote state sides / barriers (threads 32, 64)
+  int roff = 0;                               // staging index of this thread's row 0 (right side)
   __device__ __forceinline__ void init_push() {
     const int t = threadIdx.x, nl = nloc();
-    if (rank > 0 && R * t < G) {
-      nleft = min(R, G - R * t);
-      hl = mapa_u32(smem_addr(hst + HS * NF + R * t), rank - 1);
-      hlb = mapa_u32(smem_addr(bars + 1), rank - 1);
-    }
+    if (rank > 0 && R * t < G) nleft = min(R, G - R * t);
     if (rank < C - 1 && R * t + R > nl - G && R * t < nl) {
       rfirst = max(0, nl - G - R * t);
-      hr = mapa_u32(smem_addr(hst + (R * t - (nl - G))), rank + 1);
+      roff = R * t - (nl - G);
+    }
+    if (t == 32 && rank > 0) {
+      hl = mapa_u32(smem_addr(hst + HS * NF), rank - 1);
+      hlb = mapa_u32(smem_addr(bars + 1), rank - 1);
+    }
+    if (t == 64 && rank < C - 1) {
+      hr = mapa_u32(smem_addr(hst), rank + 1);
       hrb = mapa_u32(smem_addr(bars + 1), rank + 1);
     }
   }
-  __device__ __forceinline__ void push_rows(const double (&a)[R], int f, int half) {
-    if (nleft == 0 && rfirst == R) return;
-    const uint32_t fo = 8u * static_cast<uint32_t>(f * HS), bo = 8u * static_cast<uint32_t>(half);
+  __device__ __forceinline__ void stage_rows(const double (&a)[R], int slot) {
+    double *sl = stg + buf * (4 * HS) + slot * HS;
+    double *sr = sl + 2 * HS;
 #pragma unroll
     for (int j = 0; j < R; ++j) {
-      if (j < nleft) st_async_f64(hl + fo + 8u * j, a[j], hlb + bo);
-      if (j >= rfirst) st_async_f64(hr + fo + 8u * j, a[j], hrb + bo);
+      if (j < nleft) sl[R * threadIdx.x + j] = a[j];
+      if (j >= rfirst) sr[roff + j] = a[j];
     }
+  }
+  __device__ __forceinline__ void send_rows(int f, int nfield) {
+    const uint32_t bytes = static_cast<uint32_t>(8 * HS * nfield);
+    const uint32_t fo = 8u * static_cast<uint32_t>(f * HS), bo = 8u * static_cast<uint32_t>(buf);
+    if (hl) bulk_s2c(hl + fo, smem_addr(stg + buf * (4 * HS)), bytes, hlb + bo);
+    if (hr) bulk_s2c(hr + fo, smem_addr(stg + buf * (4 * HS) + 2 * HS), bytes, hrb + bo);
   }
   // Cluster-wide sum of K values in two stages (every exchange variant uses
   // the same order, so all give the same bits): warp butterflies, the 4 warp
@@ -788,12 +805,16 @@ struct Line3ClusterComm {
                                         const double (&xb)[R]) {
     static_assert(K >= 1 && K <= 8, "cluster sum supports 1..8 values");
     uint32_t hbytes = 0;
+    int hf = 0;
     if (H2 && what) {
       const int nb = (rank > 0 ? 1 : 0) + (rank < C - 1 ? 1 : 0);
-      hbytes = static_cast<uint32_t>(8 * G * nb * (what == 2 ? 2 : 1));
-      const int f = what == 1 ? ((vk & 1) ? F_V1 : F_V0) : what == 4 ? F_T : F_R;
-      push_rows(xa, f, buf);
-      if (what == 2) push_rows(xb, F_D, buf);
+      hbytes = static_cast<uint32_t>(8 * HS * nb * (what == 2 ? 2 : 1));
+      hf = what == 1 ? ((vk & 1) ? F_V1 : F_V0) : what == 4 ? F_T : F_R;
+      if (nleft || rfirst < R) {
+        stage_rows(xa, 0);
+        if (what == 2) stage_rows(xb, 1);  // d right after r (F_D = F_R + 1)
+        fence_proxy_async_smem();          // staged rows before the async-proxy copy reads them
+      }
       if (what == 1) ++vk;
     }
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -821,6 +842,7 @@ struct Line3ClusterComm {
     if (MB && threadIdx.x == 0)
       mbar_arrive_expect_tx(bars + 1 + buf, static_cast<uint32_t>(K * C * 8) + hbytes);
     __syncthreads();
+    if (H2 && what) send_rows(hf, what == 2 ? 2 : 1);
     if (threadIdx.x < K) {  // lane k of warp 0: the CTA partial of value k, to every CTA
       const double2 w01 = reinterpret_cast<const double2 *>(Wb + threadIdx.x * NWARP)[0];
       const double2 w23 = reinterpret_cast<const double2 *>(Wb + threadIdx.x * NWARP)[1];
@@ -911,8 +933,8 @@ struct Line3ClusterGeom {
   static constexpr int R = 8, NT = 128;
   static constexpr int OFF_RED = G3::OFF_RED;                         // [2][8][C*4]
   static constexpr int OFF_X = (OFF_RED + 2 * 8 * (4 + C) + 1) & ~1;  // scratch [2][8][4 + C]
-  static constexpr int OFF_HS = OFF_X + R * NT;       // halo state [2][6][66] (H2)
-  static constexpr int OFF_BAR = OFF_HS + 2 * 6 * 66;  // 3 mbarriers (MB = 1)
+  static constexpr int OFF_HS = OFF_X + R * NT;  // halo state [2][6][66], staging [2][2][2][66] (H2)
+  static constexpr int OFF_BAR = OFF_HS + 2 * 6 * 66 + 8 * 66;  // 3 mbarriers (MB = 1)
   static constexpr int SMEM_BYTES = (OFF_BAR + 3) * 8 + 16;
 };
 
@@ -951,7 +973,7 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const So
     sg[pl * L::S + (q < L::GQ ? q : q + NT)] = 0.0;
   }
   if (H2)
-    for (int i = tid; i < 2 * 6 * 66; i += NT) hst[i] = 0.0;
+    for (int i = tid; i < 2 * 6 * 66 + 8 * 66; i += NT) hst[i] = 0.0;  // state + staging
   if (rank == 0 && tid == 0 && P.pf_ahead > 0 && sys + P.pf_ahead < P.batch) {
     const long long ns = sys + P.pf_ahead;
     const void *va = P.values + ns * P.sys_stride;
