@@ -114,9 +114,10 @@ enum {
   BSOLVE_PREC_BLOCK_JACOBI = 2 /* M = block diagonal of A with
                               blocks of 8 consecutive rows, each solved exactly
                               (R30).  BiCGSTAB on the line-tiled TMEM
-                              plan only (2D 9-point stencils, grid width 31 or
-                              32, n <= 1024, where every block is tridiagonal);
-                              UNSUPPORTED elsewhere                           */
+                              plans only (2D 9-point stencils, where every block
+                              is tridiagonal: grid width 31 or 32 with n <= 1024,
+                              or width 64 with 1024 < n <= 8192 on the cluster
+                              plan); UNSUPPORTED elsewhere                    */
 };
 
 /* Per-system outcome written to status[] (R10). */

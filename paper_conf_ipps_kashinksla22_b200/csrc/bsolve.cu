@@ -512,17 +512,24 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
         }
         return true;
       };
+      const bool cbj = opt.precond == BSOLVE_PREC_BLOCK_JACOBI;
+      if (cbj && !(ctmem && cl_line == 3))
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                              "block-Jacobi on the cluster plan needs the line kernel (TMEM values)"));
       if (ctmem && cl_line == 3) {
         int cnt = 0;
-        const CVariant *t = variants_cluster_line3(&cnt, &line_smem);
+        const CVariant *t = cbj ? variants_cluster_line3_bj(&cnt, &line_smem)
+                                : variants_cluster_line3(&cnt, &line_smem);
         const char *csenv = getenv("BSOLVE_CLUSTER_SYNC");  // "barrier": the reference exchange
         // BSOLVE_CLUSTER_SYNC: default / "state": halo state kept per CTA, 2
         // exchanges per iteration, the boundary rows riding the reductions as
         // bulk copies (measured fastest); "halo": bulk halo copies + two-stage
         // reductions, 4 exchanges; "barrier": cluster barriers (the reference)
-        const int mb = !csenv ? 2 : std::strcmp(csenv, "barrier") == 0 ? 0
-                                  : std::strcmp(csenv, "halo") == 0   ? 1
-                                                                       : 2;
+        const int mb = cbj     ? 1  // block-Jacobi: the halo exchange only
+                       : !csenv ? 2
+                       : std::strcmp(csenv, "barrier") == 0 ? 0
+                       : std::strcmp(csenv, "halo") == 0    ? 1
+                                                            : 2;
         for (int i = 0; i < cnt && !h->cvar; ++i) {
           if (t[i].c != c) continue;
           if (t[i].rounds != mb) continue;
@@ -534,6 +541,10 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
           for (int cc = 0; cc < 8; ++cc) h->c2s[cc] = c2s[cc];
         }
       }
+      if (cbj && !h->cvar)
+        return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
+                              "block-Jacobi on the cluster plan needs a 9-point stencil on a "
+                              "64-wide grid"));
       if (ctmem && !h->cvar) {
         int cnt = 0;
         const CVariant *t = variants_cluster_tmem(&cnt);
@@ -641,10 +652,11 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
     }
   }
-  if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && !line_v)
+  if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && !line_v && h->place != PLACE_CLUSTER)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "block-Jacobi needs the line-tiled plan: a 2D 9-point stencil on a grid "
-                          "of width 31 or 32, n <= 1024, placement AUTO or TMEM"));
+                          "of width 31 or 32 (n <= 1024, placement AUTO or TMEM) or 64 (cluster "
+                          "plan, 1024 < n <= 8192)"));
   if (opt.solver == BSOLVE_SOLVER_GMRES && !line_v)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "GMRES needs a 2D stencil pattern (9- or 5-point, grid width 31 or "

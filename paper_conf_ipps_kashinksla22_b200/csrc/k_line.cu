@@ -48,6 +48,16 @@ static const CVariant kL3CVariants[] = {
     L3CV_(64, 5, 1), L3CV_(64, 6, 1), L3CV_(64, 7, 1), L3CV_(64, 8, 1), L3CV_(64, 2, 0),
     L3CV_(64, 3, 0), L3CV_(64, 4, 0), L3CV_(64, 5, 0), L3CV_(64, 6, 0), L3CV_(64, 7, 0),
     L3CV_(64, 8, 0)};
+// block-Jacobi (PRE = 1) on the cluster plan: halo exchange (rounds field 1)
+#define L3CVB_(NX, C) {C, NX, 1, (solve_fn)bicgstab_line3_cluster_kernel<NX, C, 1, 0, 2, 1>}
+static const CVariant kL3CBVariants[] = {L3CVB_(64, 2), L3CVB_(64, 3), L3CVB_(64, 4),
+                                         L3CVB_(64, 5), L3CVB_(64, 6), L3CVB_(64, 7),
+                                         L3CVB_(64, 8)};
+const CVariant *variants_cluster_line3_bj(int *count, int *smem_bytes) {
+  *count = (int)(sizeof(kL3CBVariants) / sizeof(kL3CBVariants[0]));
+  *smem_bytes = Line3ClusterGeom<64, 8, 1>::SMEM_BYTES;
+  return kL3CBVariants;
+}
 const CVariant *variants_cluster_line3(int *count, int *smem_bytes) {
   *count = (int)(sizeof(kL3CVariants) / sizeof(kL3CVariants[0]));
   *smem_bytes = Line3ClusterGeom<64, 8>::SMEM_BYTES;

@@ -927,21 +927,27 @@ struct Line3ClusterComm {
   __device__ __forceinline__ void sync_local() { __syncthreads(); }
 };
 
-template <int NX, int C>
+template <int NX, int C, int PRE = 0>
 struct Line3ClusterGeom {
   using G3 = Line3Geom<NX, 0>;
   static constexpr int R = 8, NT = 128;
   static constexpr int OFF_RED = G3::OFF_RED;                         // [2][8][C*4]
   static constexpr int OFF_X = (OFF_RED + 2 * 8 * (4 + C) + 1) & ~1;  // scratch [2][8][4 + C]
   static constexpr int OFF_HS = OFF_X + R * NT;  // halo state [2][6][66], staging [2][2][2][66] (H2)
-  static constexpr int OFF_BAR = OFF_HS + 2 * 6 * 66 + 8 * 66;  // 3 mbarriers (MB = 1)
+  static constexpr int OFF_F = OFF_HS + 2 * 6 * 66 + 8 * 66;  // PRE = 1: block-Jacobi factors [22][NT]
+  static constexpr int OFF_BAR = OFF_F + (PRE ? 22 * NT : 0);  // 3 mbarriers (MB = 1)
   static constexpr int SMEM_BYTES = (OFF_BAR + 3) * 8 + 16;
 };
 
 // One system per cluster of C CTAs x 1024 rows (blockIdx.x / C = system).
-template <int NX, int C, int MB = 1, int H2 = 1, int ROUNDS = 2>
+// PRE = 1: block-Jacobi (R30) with the thread's 8 rows as its block, as in the
+// single-CTA kernel; the guards then hold p^ = M^-1 p and s^ = M^-1 s, which
+// a neighbour cannot recompute from the row state alone, so PRE = 1 runs the
+// halo exchange (H2 = 0).
+template <int NX, int C, int MB = 1, int H2 = 1, int ROUNDS = 2, int PRE = 0>
 __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const SolveParams P) {
-  using CG = Line3ClusterGeom<NX, C>;
+  static_assert(!(PRE && H2), "block-Jacobi guards are exchanged, not recomputed");
+  using CG = Line3ClusterGeom<NX, C, PRE>;
   constexpr int R = 8, NT = 128;
   using L = LineGeom<NX, NT, R>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -1004,8 +1010,8 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_cluster_kernel(const So
   const uint32_t trh = tbase_s[1] + lane_hi;
   const uint32_t ta0 = trh + 16;
   Line3ClusterComm<NX, C, MB, H2> comm(sg, sred, bars, rank, n, hst);
-  line3_solve<NX, ROUNDS, 0>(P, sys, grow0, rank == 0 && tid == 0, act, comm, nullptr, sx2, tval,
-                             trh, ta0);
+  line3_solve<NX, ROUNDS, PRE>(P, sys, grow0, rank == 0 && tid == 0, act, comm,
+                               PRE ? sg + CG::OFF_F + tid : nullptr, sx2, tval, trh, ta0);
   asm volatile("tcgen05.fence::before_thread_sync;");
   // no CTA leaves while a peer may still store into its SMEM.  MB = 1: the
   // last exchange is a reduction whose pushes into this CTA all completed on

@@ -68,6 +68,8 @@ const CVariant *variants_cluster(int *count);
 const CVariant *variants_cluster_tmem(int *count);
 // 3-CTA line-tiled plan on a cluster (line3_kernel.cuh), kreg = grid width NX
 const CVariant *variants_cluster_line3(int *count, int *smem_bytes);
+// the same with block-Jacobi (PRE = 1, halo exchange)
+const CVariant *variants_cluster_line3_bj(int *count, int *smem_bytes);
 const TVariant *variants_tmem(int *count);
 const LVariant *variants_line(int *count);
 const BVariant *variants_banded(int *count);
