@@ -37,6 +37,7 @@
 //    the band and x_j travels by shuffle (no CTA barrier per step).
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 #ifndef BBAND_LDS64
@@ -460,6 +461,187 @@ __global__ void __launch_bounds__(SPLIT ? Geo<KL, KU>::NTF : Geo<KL, KU>::NT, MI
       }
     }
     ++k;
+  }
+}
+
+// ---- one warp per system (split mode factorisation) --
+// The same dgbtf2 step as banded_lu_kernel, with the W + 1 "virtual column
+// threads" vt = 0..W (vt = W: b) folded onto NCL lanes, CPL columns per lane
+// (vt = lane + NCL s, s < CPL).  One multiplier load then feeds CPL columns,
+// the step needs no CTA barrier (one __syncwarp), and every SMEM broadcast
+// reaches one warp instead of ceil((W + 2) / 32): per elimination step of a
+// K = 33 system 17 LDS.128 + 17 STS.128 instead of 51 + 17.  The pivot
+// column vt = j mod W is warp-uniform, so the lane and slot are known to all;
+// its lane runs the IDAMAX test and publishes as before.  Lanes e <= E load
+// pattern entry e of the rows entering the ring (E + 1 <= 32).
+// (A look-ahead variant -- the next pivot column updated first and its test
+// overlapped with the other columns' FMAs -- needs ~20 more registers than
+// the 255 this one uses and spilled: 0.73 vs 0.94 M sys/s; DESIGN.md f4 log.)
+template <int KL, int KU>
+struct WGeo {
+  static constexpr int R = KL + 1, W = KL + KU + 1;
+  static constexpr int CPL = (W + 1 + 31) / 32;           // columns per lane
+  static constexpr int NCL = (W + 1 + CPL - 1) / CPL;     // lanes owning columns
+  static constexpr int D = R - 2 < 4 ? R - 2 : 4;         // row prefetch distance
+  static constexpr int RB = W + 2;                        // ring stride (+ a dummy slot)
+  static constexpr int RP = (R + 1) & ~1;
+  static constexpr int OFF_CB = (R * RB + 1) & ~1;        // colbuf [2][RP] (16-byte aligned)
+  static constexpr int smem_bytes = (OFF_CB + 2 * RP + 3) * 8;  // + s_p[2], s_rp[2]
+  static_assert(NCL <= 32 && D >= 1, "one warp per system");
+};
+
+template <int KL, int KU, int MINB>
+__global__ void __launch_bounds__(32, MINB) banded_lu_warp_kernel(const BandParams P) {
+  using G = WGeo<KL, KU>;
+  constexpr int R = G::R, W = G::W, CPL = G::CPL, NCL = G::NCL, D = G::D, RB = G::RB;
+  constexpr int RP = G::RP;
+  extern __shared__ __align__(16) double wsm[];
+  double *ring = wsm;                 // [R][RB]
+  double *colbuf = wsm + G::OFF_CB;   // [2][RP]: pivot column rows 1..KL (index k-1)
+  int *s_p = reinterpret_cast<int *>(colbuf + 2 * RP);
+  double *s_rp = colbuf + 2 * RP + 1;  // [2]
+  const int l = threadIdx.x;
+  const int n = P.n;
+  const size_t ws_sys = (size_t)n * W + n;
+  for (int i = l; i < R * RB; i += 32) ring[i] = 0.0;
+  __syncwarp();
+  int vt[CPL];
+#pragma unroll
+  for (int s = 0; s < CPL; ++s) vt[s] = l + NCL * s <= W && l < NCL ? l + NCL * s : -1;
+  const bool loader = l <= P.E;  // pattern entry l (l == E: b)
+  const long long cnt = P.list ? *P.list_len : P.batch;
+  for (long long it = blockIdx.x; it < cnt; it += gridDim.x) {
+    const long long sys = P.list ? P.list[it] : it;
+    if (P.only && P.only[sys] == 0) continue;  // converged iteratively
+    double *U = P.ws + (size_t)sys * ws_sys;
+    double *Y = U + (size_t)n * W;
+    const double *val = P.values + sys * P.sys_stride;
+    const double *bb = P.b + sys * n;
+    int info = 0;  // this lane's first zero pivot (j + 1)
+    // ---- prologue: rows 0..KL straight into the registers -----------------
+    if (loader) {
+#pragma unroll 1
+      for (int r = 0; r < R; ++r) load_entry<KL, KU>(P, val, bb, ring, r, r, l, load_pk(P, r, l));
+      cp_commit();
+      cp_wait<0>();
+    }
+    __syncwarp();
+    double v[CPL][R];
+#pragma unroll
+    for (int s = 0; s < CPL; ++s)
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        v[s][r] = vt[s] >= 0 ? ring[r * RB + vt[s]] : 0.0;
+        if (vt[s] >= 0) ring[r * RB + vt[s]] = 0.0;
+      }
+    __syncwarp();
+    int pk = -1;
+    if (loader) {
+#pragma unroll
+      for (int d = 1; d <= D; ++d) {
+        load_entry<KL, KU>(P, val, bb, ring, (KL + d) % R, KL + d, l, load_pk(P, KL + d, l));
+        cp_commit();
+      }
+      pk = load_pk(P, KL + 1 + D, l);
+    }
+    int pos[CPL];
+#pragma unroll
+    for (int s = 0; s < CPL; ++s) pos[s] = vt[s];  // column j + pos (b: W; unused: -1)
+    int jr = 0;       // j mod R
+    int pt = 0;       // pivot virtual thread j mod W
+    double *Urow = U;
+#pragma unroll 1
+    for (int j = 0; j < n; ++j) {
+      const int jb = j & 1;
+      const int pl = pt % NCL, ps = pt / NCL;  // pivot lane and slot (warp-uniform)
+      if (l == pl) {
+#pragma unroll
+        for (int s = 0; s < CPL; ++s) {
+          if (s != ps) continue;
+          bool diag_max[4] = {true, true, true, true};
+#pragma unroll
+          for (int kk = 1; kk < R; ++kk)
+            diag_max[kk & 3] = diag_max[kk & 3] && (fabs(v[s][0]) >= fabs(v[s][kk]));
+          int p = 0;
+          if (!(diag_max[0] && diag_max[1] && diag_max[2] && diag_max[3])) p = argmax_abs<R>(v[s]);
+          double pv = v[s][0];
+          double2 *cbw = reinterpret_cast<double2 *>(colbuf + jb * RP);
+#pragma unroll
+          for (int kk = 1; kk < R; kk += 2)
+            cbw[(kk - 1) / 2] = make_double2(v[s][kk], kk + 1 < R ? v[s][kk + 1] : 0.0);
+          if (p != 0) {
+            pv = colbuf[jb * RP + p - 1];
+            colbuf[jb * RP + p - 1] = v[s][0];  // row swap in the published column
+          }
+          const double rp = pv != 0.0 ? __drcp_rn(pv) : 0.0;
+          s_p[jb] = p;
+          s_rp[jb] = rp;
+          Urow[0] = rp;
+          if (P.ipiv) P.ipiv[sys * n + j] = j + p;
+          if (pv == 0.0 && info == 0) info = j + 1;
+        }
+      }
+      if (loader) {
+        int slot = jr + D;
+        if (slot >= R) slot -= R;
+        load_entry<KL, KU>(P, val, bb, ring, slot, j + KL + 1 + D, l, pk);
+        pk = load_pk(P, j + KL + 2 + D, l);
+        cp_commit();
+        cp_wait<D>();
+      }
+      __syncwarp();
+      const int p = s_p[jb];
+      const double rp = s_rp[jb];
+      if (p != 0) {  // row swap j <-> j+p (uniform branch)
+#pragma unroll
+        for (int s = 0; s < CPL; ++s) {
+          const double a = v[s][0];
+          double bsel = a;
+#pragma unroll
+          for (int kk = 1; kk < R; ++kk) bsel = (p == kk) ? v[s][kk] : bsel;
+#pragma unroll
+          for (int kk = 1; kk < R; ++kk) v[s][kk] = (p == kk) ? a : v[s][kk];
+          v[s][0] = bsel;
+        }
+      }
+      double w[CPL];
+#pragma unroll
+      for (int s = 0; s < CPL; ++s) {
+        const double uc = v[s][0];
+        double *dst = pos[s] == W ? Y + j : Urow + pos[s];
+        if (pos[s] == W || (pos[s] >= 1 && pos[s] < n - j)) *dst = uc;
+        w[s] = pos[s] == 0 ? 1.0 : uc * rp;  // pivot column: exact zeros
+      }
+      const double2 *cb = reinterpret_cast<const double2 *>(colbuf + jb * RP);
+#pragma unroll
+      for (int kk = 1; kk < R; kk += 2) {
+        const double2 m = cb[(kk - 1) / 2];
+#pragma unroll
+        for (int s = 0; s < CPL; ++s) {
+          v[s][kk - 1] = fma(-m.x, w[s], v[s][kk]);
+          if (kk + 1 < R) v[s][kk] = fma(-m.y, w[s], v[s][kk + 1]);
+        }
+        if ((kk - 1) % 6 == 4) asm volatile("" ::: "memory");  // <= 3 multiplier pairs in flight
+      }
+      // row j+KL+1 (ring slot j mod R) enters as window row KL
+#pragma unroll
+      for (int s = 0; s < CPL; ++s) {
+        if (vt[s] >= 0) {
+          v[s][KL] = ring[jr * RB + vt[s]];
+          ring[jr * RB + vt[s]] = 0.0;
+        } else {
+          v[s][KL] = 0.0;
+        }
+        pos[s] = (vt[s] >= 0 && vt[s] < W) ? (pos[s] == 0 ? W - 1 : pos[s] - 1) : pos[s];
+      }
+      jr = (jr + 1 == R) ? 0 : jr + 1;
+      pt = (pt + 1 == W) ? 0 : pt + 1;
+      Urow += W;
+    }
+    if (loader) cp_wait<0>();
+    __syncwarp();  // every ring read of this system done before the next prologue
+    const unsigned first = __reduce_min_sync(0xffffffffu, info ? static_cast<unsigned>(info) : ~0u);
+    if (l == 0 && P.info) P.info[sys] = first == ~0u ? 0 : static_cast<int>(first);
   }
 }
 

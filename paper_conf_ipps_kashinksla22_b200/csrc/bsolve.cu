@@ -1350,11 +1350,19 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
       (int)std::min<long long>(4, (long long)h->smem_optin / ((long long)(n + Wb) * 8));
   const char *senv = getenv("BSOLVE_BANDED_SPLIT");
   const bool split = !(senv && atoi(senv) == 0) && bs_warps >= 1;
-  banded_fn fact = split ? bv->fn_split : bv->fn;
-  const int nt = split ? bv->nt_split : bv->nt;
+  // split mode factorisation: one warp per system (banded_lu_warp_kernel) when
+  // the instance has one and a row's entries + b fit the 32 loader lanes;
+  // developer knob BSOLVE_BANDED_WARP=0 keeps the multi-warp CTA kernel
+  const char *wenv = getenv("BSOLVE_BANDED_WARP");
+  const bool warp = split && bv->fn_warp && h->W + 1 <= 32 && !(wenv && atoi(wenv) == 0);
+  banded_fn fact = warp ? bv->fn_warp : split ? bv->fn_split : bv->fn;
+  const int nt = warp ? 32 : split ? bv->nt_split : bv->nt;
+  const int fsmem = warp ? bv->smem_warp : bv->smem_bytes;
+  if (warp)
+    cudaFuncSetAttribute((const void *)fact, cudaFuncAttributePreferredSharedMemoryCarveout,
+                         cudaSharedmemCarveoutMaxShared);
   int occ = 0;
-  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)fact, nt,
-                                                         bv->smem_bytes));
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void *)fact, nt, fsmem));
   if (occ < 1) return fail(BSOLVE_ERR_UNSUPPORTED, "banded kernel cannot be resident");
   const long long resident = (long long)occ * h->num_sms;
   long long chunk = count;
@@ -1401,7 +1409,7 @@ static int launch_banded(bsolve_handle h, const double *values, const double *b,
       Q.info = info ? info + c0 : nullptr;
       Q.ipiv = ipiv ? ipiv + c0 * n : nullptr;
       Q.batch = cnt;
-      fact<<<(int)std::min<long long>(resident, cnt), nt, bv->smem_bytes, stream>>>(Q);
+      fact<<<(int)std::min<long long>(resident, cnt), nt, fsmem, stream>>>(Q);
       const int gb =
           (int)std::min<long long>((cnt + bs_warps - 1) / bs_warps, (long long)h->num_sms * 16);
       bv->fn_backsub<<<gb, 32 * bs_warps, sbs, stream>>>(Q);

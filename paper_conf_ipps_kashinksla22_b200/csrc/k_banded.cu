@@ -9,13 +9,16 @@
 
 using namespace bband;
 
-#define BV_(K, MINB, MINB_SPLIT)                                                  \
+#define BV_(K, MINB, MINB_SPLIT, WARP)                                            \
   {K, Geo<K, K>::NT, Geo<K, K>::NTF - Geo<K, K>::W - 1, Geo<K, K>::smem_bytes,    \
    (banded_fn)banded_lu_kernel<K, K, MINB>, Geo<K, K>::NTF,                       \
    (banded_fn)banded_lu_kernel<K, K, MINB_SPLIT, true>,                          \
-   (banded_fn)banded_backsub_kernel<K, K>}
-static const BVariant kBVariants[] = {BV_(4, 8, 8), BV_(8, 8, 8), BV_(16, 5, 8),
-                                      BV_(33, 5, 8), BV_(65, 1, 1)};
+   (banded_fn)banded_backsub_kernel<K, K>, WARP}
+#define BW_(K) (banded_fn) banded_lu_warp_kernel<K, K, 8>, WGeo<K, K>::smem_bytes
+#define BW_NONE nullptr, 0
+static const BVariant kBVariants[] = {BV_(4, 8, 8, BW_(4)), BV_(8, 8, 8, BW_(8)),
+                                      BV_(16, 5, 8, BW_(16)), BV_(33, 5, 8, BW_(33)),
+                                      BV_(65, 1, 1, BW_NONE)};
 
 const BVariant *variants_banded(int *count) {
   *count = (int)(sizeof(kBVariants) / sizeof(kBVariants[0]));

@@ -60,6 +60,8 @@ struct BVariant {
   int nt_split;    // split mode: factor-only CTA size
   banded_fn fn_split;    // split mode: factorisation (U, y to a per-system workspace)
   banded_fn fn_backsub;  // split mode: one warp per system back substitution
+  banded_fn fn_warp;     // split mode: one warp per system factorisation (nullptr: none)
+  int smem_warp;         // its dynamic SMEM
 };
 
 const Variant *variants_generic(int *count);

@@ -301,3 +301,32 @@ def test_banded_large_grid_backsub_smem():
     assert np.all(info == 0)
     xo, io, _ = oracle_banded(pat.row_ptr, pat.col_idx, B.values, B.b)
     assert np.max(np.linalg.norm(x - xo, axis=1) / np.linalg.norm(xo, axis=1)) <= 1e-12
+
+
+@pytest.mark.parametrize("nx,ny,pivot", [(32, 31, False), (32, 31, True), (12, 9, True),
+                                         (17, 6, True), (5, 4, True), (31, 32, False)])
+def test_warp_kernel_bitwise_equals_cta_kernel(nx, ny, pivot, monkeypatch):
+    """The one-warp-per-system factorisation (banded_lu_warp_kernel, default in
+    split mode) does every column's operations in the CTA kernel's order, so x,
+    info and ipiv agree bit for bit with BSOLVE_BANDED_WARP=0 (instances KB =
+    4, 16, 33; pivoting-heavy and XGC values), and both match the oracle."""
+    pat = X.stencil_pattern(nx, ny)
+    if pivot:
+        rng = np.random.default_rng(nx * 7 + ny)
+        v = rng.standard_normal((24, pat.nnz))
+        v[:, pat.col_idx == np.repeat(np.arange(pat.n), np.diff(pat.row_ptr))] *= 1e-2
+        b = rng.standard_normal((24, pat.n))
+    else:
+        B = X.make_batch(0, 24, nx=nx, ny=ny)
+        v, b = B.values, B.b
+    outs = []
+    for knob in (None, "0"):
+        if knob is None:
+            monkeypatch.delenv("BSOLVE_BANDED_WARP", raising=False)
+        else:
+            monkeypatch.setenv("BSOLVE_BANDED_WARP", knob)
+        outs.append(gpu_banded(pat.row_ptr, pat.col_idx, v, b))
+    for a, c in zip(outs[0], outs[1]):
+        assert np.array_equal(a, c)
+    xo, io, po = oracle_banded(pat.row_ptr, pat.col_idx, v, b)
+    assert np.array_equal(outs[0][1], io) and np.array_equal(outs[0][2], po)

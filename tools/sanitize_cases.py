@@ -28,6 +28,10 @@ CASES = [
     ("persistent regs", dict(nx=32, ny=31), dict(placement="regs")),
     ("cluster C=3 (n=2112)", dict(nx=64, ny=33), dict()),
     ("line-tiled cluster C=4 (n=4032)", dict(nx=64, ny=63), dict()),
+    ("line-tiled cluster C=4, halo exchange", dict(nx=64, ny=63), dict(),
+     {"BSOLVE_CLUSTER_SYNC": "halo"}),
+    ("line-tiled block-Jacobi", dict(nx=32, ny=31), dict(precond="block_jacobi")),
+    ("line-tiled cluster C=4 block-Jacobi", dict(nx=64, ny=63), dict(precond="block_jacobi")),
     ("strided cluster C=4 (st.async)", dict(nx=64, ny=63), dict(), {"BSOLVE_CLUSTER_LINE": "0"}),
 ]
 
@@ -36,8 +40,16 @@ def banded_cases():
     """f4 banded LU (bsolve_banded_solve): XGC systems (KB = 33), pivoting-heavy
     random values (KB = 8, swaps every step), more systems than CTAs."""
     bad = 0
-    for name, grid, pivot, batch in (("banded 32x31 (KB=33)", dict(nx=32, ny=31), False, 3),
-                                     ("banded 7x5 pivoting (KB=8)", dict(nx=7, ny=5), True, 5)):
+    for name, grid, pivot, batch, knob in (
+            ("banded 32x31 (KB=33), warp kernel", dict(nx=32, ny=31), False, 3, None),
+            ("banded 32x31 (KB=33), CTA kernel", dict(nx=32, ny=31), False, 3, "0"),
+            ("banded 7x5 pivoting (KB=8), warp", dict(nx=7, ny=5), True, 5, None),
+            ("banded 7x5 pivoting (KB=8), CTA", dict(nx=7, ny=5), True, 5, "0")):
+        # BSOLVE_BANDED_WARP is read at launch: 0 = the multi-warp CTA kernel
+        if knob is None:
+            os.environ.pop("BSOLVE_BANDED_WARP", None)
+        else:
+            os.environ["BSOLVE_BANDED_WARP"] = knob
         pat = X.stencil_pattern(**grid)
         B = X.make_batch(0, batch, pattern=pat)
         vals = B.values.copy()
@@ -56,6 +68,7 @@ def banded_cases():
             xo, io, po = O.banded_factor_solve(pat.row_ptr, pat.col_idx, vals[k], B.b[k])
             err = max(err, np.linalg.norm(x[k] - xo) / np.linalg.norm(xo))
             same = same and np.array_equal(piv[k], po)
+        os.environ.pop("BSOLVE_BANDED_WARP", None)
         ok = err <= 1e-10 and same and int(info.abs().sum()) == 0
         bad += not ok
         print(f"{name:32s} fwd_err_vs_oracle={err:.2e} ipiv_equal={same} {'ok' if ok else 'FAIL'}",
