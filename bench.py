@@ -296,6 +296,24 @@ def run_reference(args, rank, world):
     emit(line, args)
 
 
+def h2d_copy_gbs(dev, nbytes=1 << 30, reps=3):
+    """Measured pinned host -> device copy rate (GB/s, best of reps, CUDA
+    events): the link bound of every e2e number (inputs cross it once)."""
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    best = 0.0
+    for _ in range(reps + 1):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        d.copy_(h, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        best = max(best, nbytes / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+    del h, d
+    return best
+
+
 def rank_slice_count(args, world):
     from paper_conf_ipps_kashinksla22_b200.parallel import rank_slice
     return rank_slice(args.batch, 0, world, args.scaling).count
@@ -680,8 +698,11 @@ def run_ours(args, rank, world, local_rank):
         dt = max_over_ranks(dt, device=dev)
         h2d = int(vn.nbytes + bn.nbytes)
         d2h = int(x_h.nbytes + i_h.nbytes + r_h.nbytes + s_h.nbytes)
+        link = h2d_copy_gbs(dev)
         e2e = {"value": sl.total * e2e_steps / dt, "unit": UNIT,
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+               "h2d_gbs": h2d * e2e_steps / dt / 1e9, "h2d_copy_gbs_measured": link,
+               "link_frac": h2d * e2e_steps / dt / 1e9 / link,
                "api": "bsolve_run_host (C ABI, chunked H2D/solve/D2H pipeline)",
                "bitwise_equal_to_device_path": bool(np.array_equal(i_h, it_h) and
                                                     np.array_equal(r_h, res_h))}
@@ -937,9 +958,13 @@ def run_banded(args, rank, world, local_rank):
             S.banded_solve_host(vn, bn, out=(xh, ih))
         torch.cuda.synchronize()
         dt = max_over_ranks(time.perf_counter() - t0, device=dev)
+        link = h2d_copy_gbs(dev)
+        h2d = int(vn.nbytes + bn.nbytes)
         e2e = {"value": sl.total * steps / dt, "unit": UNIT,
-               "h2d_bytes_per_step": int(vn.nbytes + bn.nbytes),
+               "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": int(xh.nbytes + ih.nbytes), "steps": steps,
+               "h2d_gbs": h2d * steps / dt / 1e9, "h2d_copy_gbs_measured": link,
+               "link_frac": h2d * steps / dt / 1e9 / link,
                "api": "bsolve_banded_solve_host (C ABI, chunked H2D/solve/D2H pipeline)",
                "bitwise_equal_to_device_path": bool(np.array_equal(
                    xh[:2000], x[:2000].cpu().numpy()))}
