@@ -649,8 +649,16 @@ def run_ours(args, rank, world, local_rank):
                     "wherever they live; effective on-chip bandwidth, can exceed 1"},
     }
     # traffic from the committed ncu --set full capture of this kernel on this
-    # workload (profiles/ncu_traffic.json), scaled to this launch's systems
+    # workload (profiles/ncu_traffic.json), scaled to this launch's systems; the
+    # capture is of the default workload only (another grid, preconditioner,
+    # solver or placement runs another kernel: no traffic / physical fields)
+    default_workload = ((args.nx, args.ny) == (32, 31) and args.precond == "jacobi" and
+                        args.solver == "bicgstab" and args.format == "ell" and
+                        args.placement == "auto" and not args.block_threads and
+                        not args.reg_slots)
     try:
+        if not default_workload:
+            raise LookupError("no committed capture for this workload")
         tr = _json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
         scale = per_rank / tr["systems_per_launch"]
         roofline["traffic"] = tr["smem_data_pipe_bytes_per_launch"] * scale

@@ -19,7 +19,9 @@ timeout 600 python bench.py --precond block_jacobi --steps 10 --warmup 3 --no-e2
     --out $OUT/bench_bj_$TAG.jsonl > $OUT/bench_bj_$TAG.log 2>&1
 timeout 600 python bench.py --nx 64 --ny 63 --batch 16384 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline \
     --parity none --out $OUT/bench_n4032_$TAG.jsonl > $OUT/bench_n4032_$TAG.log 2>&1
-timeout 900 python bench.py --solver banded --steps 5 --warmup 2 --no-e2e --cpu-seconds 3 \
+timeout 600 python bench.py --nx 64 --ny 63 --batch 16384 --steps 10 --warmup 3 --no-e2e --no-cpu-baseline \
+    --parity none --precond block_jacobi --out $OUT/bench_n4032_bj_$TAG.jsonl > $OUT/bench_n4032_bj_$TAG.log 2>&1
+timeout 900 python bench.py --solver banded --steps 5 --warmup 2 --cpu-seconds 3 \
     --out $OUT/bench_banded_$TAG.jsonl > $OUT/bench_banded_$TAG.log 2>&1
 bash tools/r2_table2.sh $TAG
 timeout 600 python tools/iter_sensitivity.py --gpu --n 1000 --out $OUT/iter_sensitivity_$TAG.json \
