@@ -189,6 +189,12 @@ typedef struct bsolve_info {
   int occupancy_api;       /* cudaOccupancyMaxActiveBlocksPerMultiprocessor for
                               it (TMEM plans; ctas_per_sm is computed from the
                               register, SMEM, thread and TMEM-column limits) */
+  int line_width;          /* kernel_mode 4: the 2D grid width the line-tiled
+                              kernel runs (a compile-time width: 31, 32, 64;
+                              or any width <= 120 through the generic-width
+                              instances), else 0                             */
+  int line_generic;        /* 1: the generic-width instance (width mod 8 at
+                              compile time, width / 8 at run time), else 0  */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

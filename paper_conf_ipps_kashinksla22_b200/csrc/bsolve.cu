@@ -98,6 +98,8 @@ struct bsolve_plan {
   const CVariant *cvar = nullptr;    // cluster kernel when place == PLACE_CLUSTER
   solve_fn var_tmem = nullptr;       // TMEM kernel when place == PLACE_TMEM
   int line_nx = 0;                   // > 0: line-tiled TMEM kernel for an NX-wide 9-point grid
+  int line_a = 0;                    // generic-width line kernel: line_nx / 8 (else 0)
+  int line_generic = 0;              // 1: the generic-width line kernel
   int line_ctas = 0;                 // its resident CTAs per SM (launch bounds)
   int st_ok = 0;                     // pattern is a uniform-offset stencil (st_doff valid)
   int st_doff[kMaxW] = {};           // byte offset d_k * 8 of ELL slot k (stencils)
@@ -602,6 +604,7 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   // applies.  Developer knob: BSOLVE_TMEM_LINE=0 keeps the strided kernel.
   const LVariant *line_v = nullptr;
   int line_c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
+  int line_width = 0;  // the grid width the chosen line kernel runs
   {
     const char *lenv = getenv("BSOLVE_TMEM_LINE");
     const bool gm = opt.solver == BSOLVE_SOLVER_GMRES;
@@ -621,8 +624,31 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     const int lctas = ctasenv ? atoi(ctasenv) : 3;
     const char *roundsenv = getenv("BSOLVE_ROUNDS");
     const int lrounds = roundsenv ? atoi(roundsenv) : (lctas == 3 ? 2 : 3);
+    // slot k -> canonical stencil slot of an NX-wide 2D grid (false: not that grid)
+    std::vector<char> real_slot(W, 0);  // slot k holds at least one entry of the pattern
+    if (line_on)
+      for (int k = 1; k < W; ++k)
+        for (int r = 0; r < n && !real_slot[k]; ++r)
+          real_slot[k] = h->h_csr2ell[(size_t)k * n + r] >= 0;
+    auto map_grid = [&](int NX, int (&c2s)[8]) {
+      const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
+      for (int c = 0; c < 8; ++c) c2s[c] = -1;
+      for (int k = 1; k < W; ++k) {
+        if (!real_slot[k]) continue;
+        const int o = h->st_doff[k] / 8;
+        int c = 0;
+        while (c < 8 && canon[c] != o) ++c;
+        if (c == 8 || c2s[c] >= 0) return false;
+        c2s[c] = k;
+      }
+      return true;
+    };
+    // developer knob BSOLVE_LINE_GENERIC=1: the generic-width instance even
+    // where a compile-time width exists (tests compare the two bit for bit)
+    const char *genv = getenv("BSOLVE_LINE_GENERIC");
+    const bool force_generic = genv && atoi(genv) == 1;
     // first pass: the requested geometry; second pass: any 2-CTA variant for the grid
-    for (int i = 0; i < 2 * lcnt && !line_v; ++i) {
+    for (int i = 0; i < 2 * lcnt && !line_v && !force_generic; ++i) {
       const LVariant &cand = lv[i % lcnt];
       if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
       if (!gm && !bj && cand.rounds != lrounds) continue;
@@ -633,24 +659,27 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       } else if (cand.ctas != 2) {
         continue;
       }
-      const int NX = cand.nx;
-      const int canon[8] = {-NX - 1, -NX, -NX + 1, -1, 1, NX - 1, NX, NX + 1};
-      int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};
-      bool ok = true;
-      for (int k = 1; k < W && ok; ++k) {
-        bool real = false;  // slot k holds at least one entry of the pattern
-        for (int r = 0; r < n && !real; ++r) real = h->h_csr2ell[(size_t)k * n + r] >= 0;
-        if (!real) continue;
-        const int o = h->st_doff[k] / 8;
-        int c = 0;
-        while (c < 8 && canon[c] != o) ++c;
-        if (c == 8 || c2s[c] >= 0) ok = false;
-        else c2s[c] = k;
-      }
-      if (!ok) continue;
+      int c2s[8];
+      if (!map_grid(cand.nx, c2s)) continue;
       line_v = &cand;
+      line_width = cand.nx;
       for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
     }
+    // generic-width 3-CTA instances (k_line_generic.cu): any width NX =
+    // B (mod 8), 3 <= NX <= nxmax (block-Jacobi: NX >= 9, tridiagonal blocks)
+    int gcnt = 0;
+    const LVariant *gv = (line_on && !gm && (bj || (lctas == 3 && lrounds == 2)))
+                             ? variants_line_generic(&gcnt) : nullptr;
+    for (int nx = bj ? 9 : 3; gv && !line_v && nx <= gv[0].nxmax; ++nx)
+      for (int i = 0; i < gcnt && !line_v; ++i) {
+        const LVariant &cand = gv[i];
+        if (cand.nx != nx % 8 || cand.pre != (bj ? 1 : 0) || nx > cand.nxmax) continue;
+        int c2s[8];
+        if (!map_grid(nx, c2s)) continue;
+        line_v = &cand;
+        line_width = nx;
+        for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
+      }
   }
   if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && !line_v && h->place != PLACE_CLUSTER)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
@@ -672,7 +701,9 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
     h->n_pad = (n + 1) & ~1;
     h->smem_vals = (int)((h->sys_stride + 1) & ~1LL);
     if (line_v) {
-      h->line_nx = line_v->nx;
+      h->line_nx = line_width;
+      h->line_a = line_v->nxmax ? line_width / 8 : 0;
+      h->line_generic = line_v->nxmax ? 1 : 0;
       h->var_tmem = line_v->fn;
       h->smem_bytes = line_v->smem_bytes;
       for (int c = 0; c < 8; ++c) h->c2s[c] = line_c2s[c];
@@ -914,6 +945,8 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->ctas_per_sm = h->ctas_per_sm;
   info->regs_per_thread = h->regs;
   info->occupancy_api = h->occ_api;
+  info->line_width = h->line_nx;
+  info->line_generic = h->line_generic;
   info->num_sms = h->num_sms;
   info->grid = h->place == PLACE_REGS      ? (int)std::min<long long>(h->grid_persist, h->batch)
                : h->place == PLACE_CLUSTER ? h->batch * h->cluster
@@ -961,7 +994,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
                         double tol, int maxiter, double *x, int32_t *iters, double *resnorm,
                         int8_t *status, int count, cudaStream_t stream, int slot = -1) {
   if (count <= 0) return BSOLVE_OK;
-  SolveParams P;
+  SolveParams P = {};
   P.values = values;
   P.b = b;
   P.x0 = x0;
@@ -995,6 +1028,7 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
     const char *pe = getenv("BSOLVE_L2_PREFETCH");
     const int k = pe ? atoi(pe) : 2;  // systems ahead, in units of #SMs
     P.pf_ahead = (h->line_nx && k > 0) ? k * h->num_sms : 0;
+    P.line_a = h->line_a;
   }
   const bool aligned = ((reinterpret_cast<uintptr_t>(values) | reinterpret_cast<uintptr_t>(b) |
                          reinterpret_cast<uintptr_t>(x0)) & 15u) == 0;

@@ -12,7 +12,7 @@ using namespace bsolve;
 
 #define LSMEM_(NX, R) ((R * LineGeom<NX, 1024 / R, R>::S + 16 * (1024 / R / 32)) * 8 + 16)
 #define LV_(NX, R, G) {NX, R, G, SOLVER_BICGSTAB, LSMEM_(NX, R), 3, \
-                       (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB>, 2}
+                       (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_BICGSTAB>, 2, 0, 0}
 // 3 CTAs per SM (line3_kernel.cuh, the default plan): r^, a_ii in TMEM, x in
 // SMEM, <= 168 registers, 3 partial sums per SpMV row.  RD = 2: rho and ||r||
 // from the omega round (R29, default); RD = 3: the literal 3-round
@@ -20,14 +20,14 @@ using namespace bsolve;
 // one FMA chain per row, a shallower one-value reduction, gathers one row
 // ahead -- DESIGN.md perf log.)
 #define LV3_(NX, RD) {NX, 8, 3, SOLVER_BICGSTAB, Line3Geom<NX>::SMEM_BYTES, RD, \
-                      (solve_fn)bicgstab_line3_kernel<NX, RD>, 3, 0}
+                      (solve_fn)bicgstab_line3_kernel<NX, RD>, 3, 0, 0}
 // block-Jacobi preconditioner, one 8-row tridiagonal block per thread (f3, R30)
 #define LV3B_(NX) {NX, 8, 3, SOLVER_BICGSTAB, Line3Geom<NX, 1>::SMEM_BYTES, 2, \
-                   (solve_fn)bicgstab_line3_kernel<NX, 2, 1>, 3, 1}
+                   (solve_fn)bicgstab_line3_kernel<NX, 2, 1>, 3, 1, 0}
 // GMRES: + the Krylov basis and the triangular factor in SMEM
 #define LVG_(NX, R, G) {NX, R, G, SOLVER_GMRES,                                          \
                         LSMEM_(NX, R) + (kMaxRestart * 1024 + kMaxRestart * kMaxRestart) * 8, 0, \
-                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_GMRES>, 2}
+                        (solve_fn)bicgstab_tmem_line_kernel<NX, R, G, SOLVER_GMRES>, 2, 0, 0}
 static const LVariant kLVariants[] = {LV_(32, 8, 4),  LV_(31, 8, 4),  LVG_(32, 8, 2),
                                       LVG_(31, 8, 2), LV3_(32, 2),    LV3_(31, 2),
                                       LV3_(32, 3),    LV3_(31, 3),    LV3B_(32),

@@ -65,6 +65,7 @@ struct SolveParams {
   int precond;              // PREC_JACOBI (d = 1 / a_ii) or PREC_NONE (d = 1)
   int restart;              // GMRES: Krylov steps per restart cycle (1 .. kMaxRestart)
   int pf_ahead;             // line plan: prefetch system sys + pf_ahead into L2 (0: off)
+  int line_a;               // generic-width line kernels: grid width / 8 (0: compile-time width)
 };
 
 // Jacobi entry d_i for diagonal a (R11: zero diagonal -> 1); 1 without preconditioner.

@@ -58,18 +58,24 @@ __device__ __forceinline__ void tmem_regs_ready2(uint32_t (&r)[2]) {
 // (line above | own line | line below) added at the end -- the 9-term FMA
 // chain of one row was the latency bound (ncu "wait" stalls; DESIGN.md perf
 // log).  The row sum is a fixed order, so results are deterministic.
-template <int NX>
+// Grid width: NX at compile time (NXG = NX, A = 0), or -- the generic-width
+// instances -- NX = B = width mod 8 with A = width / 8 at run time and the
+// plane geometry of the widest grid NXG: row 8t + o with o = +-(8A + B) + d
+// sits at idx(+-B + d) +- A (idx(8k + x) = idx(x) + k), so only the column
+// shift of the two neighbour lines is a run-time offset.
+template <int NX, int NXG = NX>
 __device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const double *gq,
                                            const double (&dd)[8], const double (&g)[8],
-                                           double (&y)[8]) {
+                                           double (&y)[8], int A = 0) {
   constexpr int R = 8;
-  using L = LineGeom<NX, 128, R>;
+  using L = LineGeom<NXG, 128, R>;
   uint32_t w[16], aw[2];
   double gm[R + 2], gp[R + 2], gr = 0.0;
+  const double *gqm = gq - A, *gqp = gq + A;  // the line below / above
 #pragma unroll
   for (int e = 0; e < 3; ++e) {
-    gm[e] = gq[L::idx(-NX + e - 1)];
-    gp[e] = gq[L::idx(NX + e - 1)];
+    gm[e] = gqm[L::idx(-NX + e - 1)];
+    gp[e] = gqp[L::idx(NX + e - 1)];
   }
   const double gl = gq[L::idx(-1)];
 #pragma unroll
@@ -77,8 +83,8 @@ __device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const do
     tmem_ld16(tval + 16 * j, w);
     tmem_ld2(ta0 + 2 * j, aw);
     if (j > 0) {  // the two operands row j is the first to need
-      gm[j + 2] = gq[L::idx(-NX + j + 1)];
-      gp[j + 2] = gq[L::idx(NX + j + 1)];
+      gm[j + 2] = gqm[L::idx(-NX + j + 1)];
+      gp[j + 2] = gqp[L::idx(NX + j + 1)];
     }
     if (j == R - 1) gr = gq[L::idx(R)];
     tmem_wait_ld();
@@ -106,11 +112,11 @@ __device__ __forceinline__ void line3_spmv(uint32_t tval, uint32_t ta0, const do
 // global row index is grow0 + 8 t + j; the communication policy Comm
 // (LineComm: CTA-local; Line3ClusterComm: halo rows and reduction partials
 // through distributed shared memory) publishes, synchronises and reduces.
-template <int NX, int ROUNDS, int PRE, class Comm>
+template <int NX, int ROUNDS, int PRE, class Comm, int NXG = NX>
 __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys, int grow0,
                                             bool leader, const bool (&act)[8], Comm &comm,
                                             double *sf, double2 *sx2, uint32_t tval,
-                                            uint32_t trh, uint32_t ta0) {
+                                            uint32_t trh, uint32_t ta0, int A = 0) {
   constexpr int R = 8, NT = 128;
   const int n = P.n;
   const int row0 = grow0 + R * threadIdx.x;  // global index of this thread's first row
@@ -208,7 +214,7 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
 
   const double one[R] = {1, 1, 1, 1, 1, 1, 1, 1};
   auto spmv = [&](const double(&dd)[R], const double(&g)[R], double(&y)[R]) {
-    line3_spmv<NX>(tval, ta0, comm.gq, dd, g, y);
+    line3_spmv<NX, NXG>(tval, ta0, comm.gq, dd, g, y, A);
   };
   auto x_load = [&](double(&xx)[R]) {
 #pragma unroll
@@ -516,9 +522,11 @@ __device__ __forceinline__ void line3_solve(const SolveParams &P, long long sys,
 // l_j = a_(j,j-1) / u_(j-1), u_j = a_jj - l_j a_(j-1,j); a zero or non-finite
 // pivot makes the block the identity) into thread-private SMEM, and every
 // application is a forward and a back substitution in registers.
-template <int NX, int ROUNDS = 2, int PRE = 0>
+// NXG > NX: a generic-width instance (NX = width mod 8, A = P.line_a = width
+// / 8, any width <= NXG; see line3_spmv).
+template <int NX, int ROUNDS = 2, int PRE = 0, int NXG = NX>
 __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParams P) {
-  using G3 = Line3Geom<NX, PRE>;
+  using G3 = Line3Geom<NXG, PRE>;
   constexpr int R = G3::R, NT = G3::NT;
   using L = typename G3::L;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -575,8 +583,10 @@ __global__ void __launch_bounds__(128, 3) bicgstab_line3_kernel(const SolveParam
   const uint32_t trh = tbase_s[1] + lane_hi;   // r^ (8 doubles)
   const uint32_t ta0 = trh + 16;               // a_jj (8 doubles)
 
-  LineComm<NX, NT, R> comm(sg, sred, act);
-  line3_solve<NX, ROUNDS, PRE>(P, sys, 0, tid == 0, act, comm, sf, sx2, tval, trh, ta0);
+  LineComm<NXG, NT, R> comm(sg, sred, act);
+  line3_solve<NX, ROUNDS, PRE, LineComm<NXG, NT, R>, NXG>(P, sys, 0, tid == 0, act, comm, sf, sx2,
+                                                          tval, trh, ta0,
+                                                          NXG == NX ? 0 : P.line_a);
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 0) {

@@ -48,6 +48,7 @@ struct LVariant {
   solve_fn fn;
   int ctas;        // resident CTAs per SM the kernel is built for (launch bounds)
   int pre;         // 0: scalar preconditioner (Jacobi / none), 1: block-Jacobi (8 rows)
+  int nxmax;       // 0: grid width nx; > 0: any width = nx (mod 8) up to nxmax (generic)
 };
 
 // batched banded LU (dgbsv analogue), k_banded.cu
@@ -74,4 +75,6 @@ const CVariant *variants_cluster_line3(int *count, int *smem_bytes);
 const CVariant *variants_cluster_line3_bj(int *count, int *smem_bytes);
 const TVariant *variants_tmem(int *count);
 const LVariant *variants_line(int *count);
+// generic-width 3-CTA line kernels (nxmax > 0), k_line_generic.cu
+const LVariant *variants_line_generic(int *count);
 const BVariant *variants_banded(int *count);

@@ -548,6 +548,66 @@ def test_line_tmem_two_cta_kernel(nx, ny, monkeypatch):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o, check_direct=False)
 
 
+@pytest.mark.parametrize("nx,ny", [(24, 40), (17, 60), (45, 22), (9, 100), (100, 10),
+                                   (120, 8), (5, 7), (3, 3), (63, 16), (40, 25)])
+def test_generic_width_line_kernel(nx, ny):
+    """Any 2D 9-point grid with n <= 1024 and width <= 120 runs the 3-CTA line
+    kernel: the generic-width instance for width mod 8 with width / 8 as a
+    run-time column shift of the neighbour lines (every residue 0..7, widths
+    from 3 to 120, ragged last thread); parity vs the oracle incl. warm start."""
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 24, pattern=pat)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b)
+    i = g["info"]
+    assert i["kernel_mode"] == 4 and i["line_generic"] == 1 and i["line_width"] == nx, i
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g)
+    x0 = O.batch_banded(pat.row_ptr, pat.col_idx, B.values, B.b) * (1 + 1e-4)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, x0=x0)
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g, x0=x0)
+
+
+@pytest.mark.parametrize("nx,ny", [(24, 40), (45, 22)])
+def test_generic_width_five_point_and_block_jacobi(nx, ny):
+    """The generic-width kernels with a 5-point stencil (corner slots absent)
+    and with block-Jacobi (R30; blocks tridiagonal for widths >= 9).  (A
+    5-point grid of width 33 has offsets +-1, +-33 only, which the compiled
+    NX = 32 kernel gathers exactly as its +-(NX + 1) slots: it takes it.)"""
+    rp, ci = _five_point(nx, ny)
+    vals = X.random_dd_values(rp, ci, 16, seed=nx, margin=0.5)
+    b = X.random_rhs(16, nx * ny, seed=ny)
+    g = gpu_solve(rp, ci, vals, b)
+    assert g["info"]["line_generic"] == 1
+    compare(rp, ci, vals, b, g)
+    pat = X.stencil_pattern(nx, ny)
+    B = X.make_batch(0, 24, pattern=pat)
+    g = gpu_solve(pat.row_ptr, pat.col_idx, B.values, B.b, precond="block_jacobi")
+    assert g["info"]["line_generic"] == 1 and g["info"]["precond"] == 2
+    o = O.batch_krylov(pat.row_ptr, pat.col_idx, B.values, B.b, precond=O.block_jacobi(8))
+    compare(pat.row_ptr, pat.col_idx, B.values, B.b, g, o=o)
+
+
+@pytest.mark.parametrize("nx,ny,precond", [(32, 31, "jacobi"), (31, 32, "jacobi"),
+                                           (32, 31, "block_jacobi")])
+def test_generic_width_equals_compiled_width_bitwise(nx, ny, precond, monkeypatch):
+    """On the paper's grid the generic-width instance (BSOLVE_LINE_GENERIC=1)
+    runs the same arithmetic as the compile-time width: bitwise equal x,
+    iters, resnorm and status, warm start and maxiter exhaustion included."""
+    B = X.make_batch(0, 64, nx=nx, ny=ny)
+    p = B.pattern
+    x0 = O.batch_banded(p.row_ptr, p.col_idx, B.values, B.b) * (1 + 1e-4)
+    outs = []
+    for knob in ("0", "1"):
+        monkeypatch.setenv("BSOLVE_LINE_GENERIC", knob)
+        g = [gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, precond=precond),
+             gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, x0=x0, precond=precond),
+             gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, maxiter=5, precond=precond)]
+        assert g[0]["info"]["line_generic"] == int(knob) and g[0]["info"]["line_width"] == nx
+        outs.append(g)
+    for a, c in zip(outs[0], outs[1]):
+        for k in ("x", "iters", "resnorm", "status"):
+            assert np.array_equal(a[k], c[k]), k
+
+
 @pytest.mark.parametrize("nx,ny,C", [(64, 32, 2), (64, 33, 3), (64, 63, 4), (64, 120, 8)])
 def test_cluster_line_kernel(nx, ny, C, monkeypatch):
     """The 3-CTA line kernel on a cluster (default for 64-wide grids, n > 1024):

@@ -17,6 +17,8 @@ from paper_conf_ipps_kashinksla22_b200 import Solver  # noqa: E402
 CASES = [
     ("line-tiled tmem (bench default)", dict(nx=32, ny=31), dict()),
     ("line-tiled tmem, grid 31x32", dict(nx=31, ny=32), dict()),
+    ("line-tiled generic width 40x25", dict(nx=40, ny=25), dict()),
+    ("line-tiled generic width 5x7", dict(nx=5, ny=7), dict()),
     ("line-tiled GMRES(7)", dict(nx=32, ny=31), dict(solver="gmres")),
     ("line-tiled + direct fallback", dict(nx=32, ny=31), dict(direct_fallback=True)),
     ("strided tmem (line off)", dict(nx=32, ny=31), dict(), {"BSOLVE_TMEM_LINE": "0"}),
