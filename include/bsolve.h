@@ -115,7 +115,7 @@ enum {
                               blocks of 8 consecutive rows, each solved exactly
                               (R30).  BiCGSTAB on the line-tiled TMEM
                               plans only (2D 9-point stencils, where every block
-                              is tridiagonal: grid width 31 or 32 with n <= 1024,
+                              is tridiagonal: grid width 9..120 with n <= 1024,
                               or width 64 with 1024 < n <= 8192 on the cluster
                               plan); UNSUPPORTED elsewhere                    */
 };

@@ -665,15 +665,17 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       line_width = cand.nx;
       for (int c = 0; c < 8; ++c) line_c2s[c] = c2s[c];
     }
-    // generic-width 3-CTA instances (k_line_generic.cu): any width NX =
-    // B (mod 8), 3 <= NX <= nxmax (block-Jacobi: NX >= 9, tridiagonal blocks)
+    // generic-width instances (k_line_generic.cu): any width NX = B (mod 8),
+    // 3 <= NX <= nxmax (block-Jacobi: NX >= 9, tridiagonal blocks); BiCGSTAB
+    // on the 3-CTA kernel, GMRES on the 2-CTA one
     int gcnt = 0;
-    const LVariant *gv = (line_on && !gm && (bj || (lctas == 3 && lrounds == 2)))
+    const LVariant *gv = (line_on && (gm || bj || (lctas == 3 && lrounds == 2)))
                              ? variants_line_generic(&gcnt) : nullptr;
     for (int nx = bj ? 9 : 3; gv && !line_v && nx <= gv[0].nxmax; ++nx)
       for (int i = 0; i < gcnt && !line_v; ++i) {
         const LVariant &cand = gv[i];
         if (cand.nx != nx % 8 || cand.pre != (bj ? 1 : 0) || nx > cand.nxmax) continue;
+        if (cand.solver != (gm ? SOLVER_GMRES : SOLVER_BICGSTAB)) continue;
         int c2s[8];
         if (!map_grid(nx, c2s)) continue;
         line_v = &cand;
@@ -684,12 +686,12 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
   if (opt.precond == BSOLVE_PREC_BLOCK_JACOBI && !line_v && h->place != PLACE_CLUSTER)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
                           "block-Jacobi needs the line-tiled plan: a 2D 9-point stencil on a grid "
-                          "of width 31 or 32 (n <= 1024, placement AUTO or TMEM) or 64 (cluster "
+                          "of width 9..120 (n <= 1024, placement AUTO or TMEM) or 64 (cluster "
                           "plan, 1024 < n <= 8192)"));
   if (opt.solver == BSOLVE_SOLVER_GMRES && !line_v)
     return fail_free(fail(BSOLVE_ERR_UNSUPPORTED,
-                          "GMRES needs a 2D stencil pattern (9- or 5-point, grid width 31 or "
-                          "32) with n <= 1024 and placement AUTO or TMEM"));
+                          "GMRES needs a 2D stencil pattern (9- or 5-point, grid width 3..120) "
+                          "with n <= 1024 and placement AUTO or TMEM"));
   const bool tmem_ok = (h->kfmt == FMT_DIA && W == 9 && n <= 1024) || line_v;
   const bool tmem_auto = opt.placement == BSOLVE_PLACE_AUTO && opt.block_threads == 0 &&
                          opt.reg_slots == 0 && tmem_ok;

@@ -103,10 +103,12 @@ __device__ __forceinline__ double tmem_f64(const uint32_t (&w)[16], int c) {
 
 // y = A g for rows Rt .. Rt+R-1.  gq = sg + GQ + t; own[j] = g[Rt + j].
 // G rows per tcgen05.ld group; group k+1 is in flight while group k's FMAs run.
-template <int NX, int NT, int R, int G>
+// NXG > NX: generic width (NX = width mod 8, A = width / 8 at run time, the
+// plane geometry of width NXG; line3_kernel.cuh line3_spmv explains the shift)
+template <int NX, int NT, int R, int G, int NXG = NX>
 __device__ __forceinline__ void line_spmv(uint32_t tlane, const double *gq, const double (&a0)[R],
-                                          const double (&own)[R], double (&y)[R]) {
-  using L = LineGeom<NX, NT, R>;
+                                          const double (&own)[R], double (&y)[R], int A = 0) {
+  using L = LineGeom<NXG, NT, R>;
   constexpr int NG = R / G;
   static_assert(R % G == 0, "G must divide R");
   uint32_t w[2][G][16];
@@ -115,8 +117,8 @@ __device__ __forceinline__ void line_spmv(uint32_t tlane, const double *gq, cons
   double gm[R + 2], gp[R + 2];
 #pragma unroll
   for (int e = 0; e < R + 2; ++e) {
-    gm[e] = gq[L::idx(-NX + e - 1)];
-    gp[e] = gq[L::idx(NX + e - 1)];
+    gm[e] = gq[L::idx(-NX + e - 1) - A];
+    gp[e] = gq[L::idx(NX + e - 1) + A];
   }
   const double gl = gq[L::idx(-1)], gr = gq[L::idx(R)];
   tmem_wait_ld();
@@ -173,11 +175,12 @@ __device__ __forceinline__ void line_spmv(uint32_t tlane, const double *gq, cons
 //   SMEM: [gather planes: R * S] [reduction scratch: 16 * NWARP] [TMEM base: 16 B]
 //         GMRES only: [Krylov basis: kMaxRestart * R * NT] [R factor: kMaxRestart^2]
 // SOLVER: SOLVER_BICGSTAB (Algorithm 1) or SOLVER_GMRES (gmres.cuh).
-template <int NX, int R, int G, int SOLVER = SOLVER_BICGSTAB, int MINB = 2, int ROUNDS = 3>
+template <int NX, int R, int G, int SOLVER = SOLVER_BICGSTAB, int MINB = 2, int ROUNDS = 3,
+          int NXG = NX>
 __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(const SolveParams P) {
   constexpr int NT = 1024 / R, NWARP = NT / 32;
   static_assert(R == 4 || R == 8, "4 or 8 rows per thread");
-  using L = LineGeom<NX, NT, R>;
+  using L = LineGeom<NXG, NT, R>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double *sg = reinterpret_cast<double *>(smem_raw);
   double *sred = sg + R * L::S;
@@ -288,9 +291,10 @@ __global__ void __launch_bounds__(1024 / R, MINB) bicgstab_tmem_line_kernel(cons
   }
   tmem_wait_st();
 
-  LineComm<NX, NT, R> comm(sg, sred, act);
+  LineComm<NXG, NT, R> comm(sg, sred, act);
+  const int A = NXG == NX ? 0 : P.line_a;
   auto spmv = [&](const double(&own)[R], double(&y)[R]) {
-    line_spmv<NX, NT, R, G>(tlane, comm.gq, a0, own, y);
+    line_spmv<NX, NT, R, G, NXG>(tlane, comm.gq, a0, own, y, A);
   };
   if constexpr (SOLVER == SOLVER_GMRES) {
     double *sV = sred + 16 * NWARP + 2;

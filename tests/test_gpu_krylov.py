@@ -47,6 +47,34 @@ def test_gmres_line_kernel(restart, nx, ny):
     compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
 
 
+@pytest.mark.parametrize("nx,ny,restart", [(40, 25, 7), (24, 40, 4), (5, 7, 7), (100, 10, 3)])
+def test_gmres_generic_width(nx, ny, restart):
+    """GMRES(m) on grid widths other than the compiled 31 / 32: the generic-
+    width instance of the 2-CTA line kernel (width mod 8 compiled)."""
+    B = X.make_batch(0, 32, nx=nx, ny=ny)
+    p = B.pattern
+    g = gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, solver="gmres", restart=restart,
+                  maxiter=4000)
+    i = g["info"]
+    assert i["solver"] == 1 and i["kernel_mode"] == 4 and i["line_generic"] == 1, i
+    assert i["line_width"] == nx
+    o = _oracle(p, B, "gmres", restart=restart, maxiter=4000)
+    compare(p.row_ptr, p.col_idx, B.values, B.b, g, o=o)
+
+
+@pytest.mark.parametrize("nx,ny", [(32, 31), (31, 32)])
+def test_gmres_generic_equals_compiled_width_bitwise(nx, ny, monkeypatch):
+    B = X.make_batch(0, 32, nx=nx, ny=ny)
+    p = B.pattern
+    outs = []
+    for knob in ("0", "1"):
+        monkeypatch.setenv("BSOLVE_LINE_GENERIC", knob)
+        outs.append(gpu_solve(p.row_ptr, p.col_idx, B.values, B.b, solver="gmres", restart=5))
+        assert outs[-1]["info"]["line_generic"] == int(knob)
+    for k in ("x", "iters", "resnorm", "status"):
+        assert np.array_equal(outs[0][k], outs[1][k]), k
+
+
 def test_gmres_warm_start_maxiter_and_edge_cases():
     B = X.make_batch(0, 40, picard=2)
     p = B.pattern
