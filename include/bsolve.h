@@ -195,6 +195,8 @@ typedef struct bsolve_info {
                               instances), else 0                             */
   int line_generic;        /* 1: the generic-width instance (width mod 8 at
                               compile time, width / 8 at run time), else 0  */
+  int max_active_clusters; /* PLACE_CLUSTER: cudaOccupancyMaxActiveClusters of
+                              the cluster kernel (systems in flight), else 0 */
 } bsolve_info;
 
 typedef struct bsolve_plan *bsolve_handle; /* opaque; owns pattern + plan     */

@@ -51,7 +51,8 @@ class Info(C.Structure):
         "n", "nnz", "batch", "ell_width", "format", "placement", "block_threads",
         "rows_per_thread", "smem_bytes", "ctas_per_sm", "num_sms", "grid", "kl", "ku", "device",
         "kernel_mode", "cluster", "solver", "precond", "restart", "banded_launches",
-        "regs_per_thread", "occupancy_api", "line_width", "line_generic")]
+        "regs_per_thread", "occupancy_api", "line_width", "line_generic",
+        "max_active_clusters")]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -108,6 +108,7 @@ struct bsolve_plan {
   int c2s[8] = {-1, -1, -1, -1, -1, -1, -1, -1};  // its canonical offset -> ELL slot map
   int cluster = 0;                   // CTAs per system (cluster plan)
   int smem_bytes_fallback = 0, grid_persist = 0;
+  int max_clusters = 0;  // PLACE_CLUSTER: cudaOccupancyMaxActiveClusters
   unsigned long long *d_ctr = nullptr;  // persistent work counter + finished-CTA count
   std::vector<int32_t> h_ell_col;  // [W][n]
   std::vector<int32_t> h_csr2ell;  // [W][n] -> CSR entry held by the slot, -1 = padding
@@ -592,8 +593,24 @@ extern "C" int bsolve_create(bsolve_handle *out, int n, int batch, const int32_t
       if (ce != cudaSuccess || ncl < 1)
         return fail_free(fail(BSOLVE_ERR_UNSUPPORTED, "cluster of %d CTAs cannot be resident: %s",
                               c, cudaGetErrorString(ce)));
-      h->ctas_per_sm = std::max(1, ncl * c / h->num_sms);
       h->grid_persist = ncl;
+      h->max_clusters = ncl;  // (the API's figure; the hardware places CTAs by the limits below)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->occ_api, (const void *)h->cvar->fn, 128,
+                                                    h->smem_bytes);
+      // resident CTAs per SM from the kernel's own limits, as for the TMEM
+      // plan below (registers, SMEM + 1 KB reservation, TMEM columns: the line
+      // cluster kernel allocates 128 + 32 per CTA)
+      cudaFuncAttributes fa = {};
+      if (cudaFuncGetAttributes(&fa, (const void *)h->cvar->fn) == cudaSuccess && fa.numRegs > 0) {
+        h->regs = fa.numRegs;
+        const int warp_regs = (fa.numRegs * 32 + 255) / 256 * 256;
+        const int by_regs = prop.regsPerMultiprocessor / (warp_regs * 4);
+        const int by_smem = (int)(prop.sharedMemPerMultiprocessor / (h->smem_bytes + 1024));
+        const int by_tmem = h->line_nx ? 512 / 160 : 512 / 128;
+        h->ctas_per_sm = std::max(1, std::min(std::min(by_regs, by_smem), by_tmem));
+      } else {
+        h->ctas_per_sm = std::max(1, (ncl * c + h->num_sms - 1) / h->num_sms);
+      }
     }
   }
   // ---- TMEM plan: values in tensor memory (DESIGN.md "Kernels" 9, 10) -----
@@ -949,6 +966,7 @@ extern "C" int bsolve_query(bsolve_handle h, bsolve_info *info) {
   info->occupancy_api = h->occ_api;
   info->line_width = h->line_nx;
   info->line_generic = h->line_generic;
+  info->max_active_clusters = h->max_clusters;
   info->num_sms = h->num_sms;
   info->grid = h->place == PLACE_REGS      ? (int)std::min<long long>(h->grid_persist, h->batch)
                : h->place == PLACE_CLUSTER ? h->batch * h->cluster
@@ -1028,7 +1046,8 @@ static int launch_solve(bsolve_handle h, const double *values, const double *b, 
   // start-up loads hit L2 instead of HBM (BSOLVE_L2_PREFETCH=0 disables)
   {
     const char *pe = getenv("BSOLVE_L2_PREFETCH");
-    const int k = pe ? atoi(pe) : 2;  // systems ahead, in units of #SMs
+    // systems ahead, in units of #SMs (cluster plan: off, measured 1.29 vs 1.27 M sys/s at n = 4032)
+    const int k = pe ? atoi(pe) : (h->place == PLACE_CLUSTER ? 0 : 2);
     P.pf_ahead = (h->line_nx && k > 0) ? k * h->num_sms : 0;
     P.line_a = h->line_a;
   }
